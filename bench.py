@@ -1,0 +1,386 @@
+#!/usr/bin/env python
+"""bench.py — swap-in throughput of the B200 swap-image engine (BASELINE.json metric:
+"model swap-in latency (s) and restore GB/s per GPU vs host-link roofline, 1/2/4/8 B200").
+
+One step = one pass of the whole hot path over the engine image:
+  a3 checkpoint (gather + fused chunk checksums)  -> a4 manifest seal (swap_sync)
+  -> a5 summary all-gather (N>1)  -> a6 poison the regions (harness; outside the swap-in clock)
+  -> a7 restore (scatter + fused compare) -> a8 HBM verify pass -> a9 mismatch all-reduce (N>1).
+value = whole-job swap-in throughput: sum over ranks of image payload bytes / max over ranks of
+the mean device time of (restore + verify), CUDA events on the launching stream.
+
+    python bench.py [--gpus N --steps K --warmup W] [--impl reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...   (one rank per GPU, NCCL)
+
+Workload (config.workload): N=1 -> BASELINE.json configs[1] (Llama-3.1-8B bf16 engine, 291
+regions, 52.57 GB); N>1 -> each rank its shard of configs[3] (Llama-3.1-70B TP=8, 627 regions,
+30.53 GB/rank; weak scaling). Inputs are far larger than the 126 MB L2, so no flush is needed.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+GB = 1e9
+PCIE_GEN5_X16_GBPS = 63.015  # 64 GB/s x 128/130 (nominal, per direction)
+MEASURED_PEAKS = os.path.join(ROOT, "MEASURED_PEAKS.json")
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="auto", choices=["auto", "A", "B", "C", "D"])
+    ap.add_argument("--mechanism", default="sm", choices=["sm", "ce_region", "ce_chunk", "ce_batch", "sm_nocheck"])
+    ap.add_argument("--checksum", default="crc32c", choices=["crc32c", "xxh64"])
+    ap.add_argument("--chunk", type=int, default=1 << 20)
+    ap.add_argument("--grid", type=int, default=0)
+    ap.add_argument("--no-compare", action="store_true", help="skip the other-mechanism comparison")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--sample-bytes", type=int, default=1 << 30, help="oracle sample size per step")
+    ap.add_argument("--out", default=None, help="also append the JSON line to this file")
+    return ap.parse_args()
+
+
+def workload(cfg: str, rank: int, world: int):
+    if cfg == "auto":
+        cfg = "B" if world == 1 else "D"
+    if cfg == "A":
+        return "A", W.config_a(rank), "synthetic 64 MiB image, 16 random-size regions (BASELINE configs[0])"
+    if cfg == "B":
+        return "B", W.config_b(), "Llama-3.1-8B bf16 engine image: 195 weight + 32 KV + 64 workspace regions (BASELINE configs[1])"
+    if cfg == "C":
+        return "C", W.config_c(rank), "Qwen2.5-32B bf16 TP=2 engine shard per rank (BASELINE configs[2])"
+    return "D", W.config_d(rank), "Llama-3.1-70B bf16 TP=8 engine shard per rank (BASELINE configs[3])"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "200"], stdout=self.f,
+                                      stderr=subprocess.DEVNULL)
+        except OSError:
+            self.p = None
+
+    def stop(self) -> dict:
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        self.p.wait(5)
+        self.f.flush()
+        rows = []
+        with open(self.f.name) as fh:
+            for line in fh:
+                parts = [x.strip() for x in line.split(",")]
+                if len(parts) == 8 and parts[1].replace(".", "").isdigit():
+                    rows.append(parts)
+        os.unlink(self.f.name)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[4 + i].lower().startswith("active")})
+        return {"sm_mhz": statistics.median(float(r[1]) for r in rows), "sm_max_mhz": float(rows[0][2]),
+                "power_w_max": max(float(r[3]) for r in rows if r[3].replace(".", "").isdigit()) if rows else None,
+                "samples": len(rows), "reasons": reasons}
+
+
+def oracle_sample_specs(specs, limit: int):
+    """A prefix of the workload's regions, at most `limit` bytes (bounded CPU sample)."""
+    out, tot = [], 0
+    for r in specs:
+        if tot + r.nbytes > limit and out:
+            break
+        out.append(r)
+        tot += r.nbytes
+    return out, tot
+
+
+def time_oracle_restore(orc, specs, host, offs, threads: int, reps: int):
+    """Oracle restore (memcpy + chunk checksum compare) of the sample; returns (GB/s list, bytes)."""
+    base = 1 << 40
+    regs = [(i, base + o, r.nbytes, r.kind) for i, (r, o) in enumerate(zip(specs, offs))]
+    rc, image, moff = orc.checkpoint(regs, host, base, 1, 1 << 20, 4096, threads=threads)
+    assert rc == 0
+    payload = sum(r.nbytes for r in specs)
+    rates = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        rc, nbad, _ = orc.restore(image, moff, host, base, threads=threads)
+        dt = time.perf_counter() - t0
+        assert rc == 0 and nbad == 0
+        rates.append(payload / dt / GB)
+    return rates, payload
+
+
+def cpu_threads() -> int:
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+# ---------------------------------------------------------------------------- reference arm
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return  # the reference arm is the CPU oracle: rank 0 alone runs it
+    import oracle
+
+    world = args.gpus
+    name, specs, desc = workload(args.config, 0, world)
+    sample, sbytes = oracle_sample_specs(specs, args.sample_bytes)
+    host, offs = W.host_arena(sample, 0)
+    th = cpu_threads()
+    rates, payload = time_oracle_restore(oracle, sample, host, offs, th, args.warmup + args.steps)
+    timed = rates[args.warmup:]
+    v = statistics.mean(timed)
+    line = {
+        "impl": "reference", "metric": "swap-in (restore + verify) throughput, whole job", "value": round(v, 3),
+        "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(payload / (v * GB) * 1e3, 3), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": f"{name}: {desc}", "sample": f"first {len(sample)} regions, {payload} B"},
+        "cpu_baseline": {"value": round(v, 3), "unit": "GB/s", "cores": th, "kind": "oracle",
+                         "sample": f"oracle_restore (memcpy + Sarwate CRC-32C per 1 MiB chunk) over the first "
+                                   f"{len(sample)} regions of workload {name} ({payload} B), {th} OpenMP threads"},
+        "e2e": {"value": round(v, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------------------- our arm
+def run_ours(args):
+    import torch
+    import torch.distributed as tdist
+
+    from paper_conf_sc_stoyanovsracb25_b200 import swap
+    from paper_conf_sc_stoyanovsracb25_b200 import dist as sdist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        print(f"warning: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        tdist.init_process_group("nccl", device_id=dev)
+
+    def barrier():
+        if world > 1:
+            tdist.barrier()
+        torch.cuda.synchronize()
+
+    def allmax(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
+        return float(t.item())
+
+    def allsum(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        tdist.all_reduce(t, op=tdist.ReduceOp.SUM)
+        return float(t.item())
+
+    name, specs, desc = workload(args.config, rank, world)
+    offs, arena_bytes = W.place(specs)
+    payload = sum(r.nbytes for r in specs)
+    t0 = time.perf_counter()
+    arena = torch.empty(arena_bytes, dtype=torch.uint8, device=dev)
+    W.fill_device_arena(arena, specs, offs, seed=rank)
+    torch.cuda.synchronize()
+    t_fill = time.perf_counter() - t0
+    base = arena.data_ptr()
+    regions = [(base + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs, offs))]
+    kind = swap.SWAP_CHECKSUM_CRC32C if args.checksum == "crc32c" else swap.SWAP_CHECKSUM_XXH64
+    t0 = time.perf_counter()
+    sw = swap.Swapper(regions, chunk_bytes=args.chunk, checksum=kind, mechanism=args.mechanism, device=local,
+                      rank=rank, world=world, grid_ctas=args.grid)
+    t_register = time.perf_counter() - t0
+    stream = torch.cuda.Stream(device=dev)
+
+    def poison():
+        with torch.cuda.stream(stream):
+            for r, o in zip(specs, offs):
+                if r.nbytes:
+                    arena[o:o + r.nbytes].fill_(W.POISON_BYTE)
+
+    def step(record: dict | None):
+        """One pass of the hot path; returns per-phase device/host times."""
+        sw.checkpoint(stream, sync=True)  # a3 + a4
+        if world > 1:
+            sdist.gather_manifest(sw, None)  # a5
+        poison()  # a6 (harness)
+        ev0 = torch.cuda.Event(enable_timing=True)
+        ev1 = torch.cuda.Event(enable_timing=True)
+        ev0.record(stream)
+        h0 = time.perf_counter()
+        sw.restore(stream)  # a7
+        res = sw.verify(stream, hbm_pass=True)  # a8 (synchronises the stream)
+        h1 = time.perf_counter()
+        ev1.record(stream)
+        bad = sdist.agree_restore(res, None) if world > 1 else res["n_bad"] + res["hbm_n_bad"]  # a9
+        ev1.synchronize()
+        assert bad == 0 and res["status"] == 0, res
+        if record is not None:
+            t = sw.timings()
+            record.setdefault("swapin_ms", []).append(ev0.elapsed_time(ev1))
+            record.setdefault("host_ms", []).append((h1 - h0) * 1e3)
+            record.setdefault("ckpt_ms", []).append(t["checkpoint_ms"])
+            record.setdefault("restore_ms", []).append(t["restore_ms"])
+            record.setdefault("verify_ms", []).append(t["verify_ms"])
+
+    for _ in range(args.warmup):
+        step(None)
+    clocks = ClockSampler(local)
+    rec: dict = {}
+    launches0 = sw.launch_count()
+    barrier()
+    clocks.start()
+    e_start = torch.cuda.Event(enable_timing=True)
+    e_end = torch.cuda.Event(enable_timing=True)
+    e_start.record(stream)
+    for _ in range(args.steps):
+        step(rec)
+    e_end.record(stream)
+    barrier()
+    clk = clocks.stop()
+    launches = sw.launch_count() - launches0
+    step_ms = allmax(e_start.elapsed_time(e_end) / args.steps)
+
+    swapin_ms = allmax(statistics.mean(rec["swapin_ms"]))
+    host_ms = allmax(statistics.mean(rec["host_ms"]))
+    restore_ms = statistics.mean(rec["restore_ms"])
+    verify_ms = statistics.mean(rec["verify_ms"])
+    ckpt_ms = allmax(statistics.mean(rec["ckpt_ms"]))
+    total_payload = allsum(payload)
+
+    # context: other movers on the same image (outside the timed region)
+    compare = {}
+    if not args.no_compare:
+        mechs = ["sm", "sm_nocheck", "ce_region", "ce_batch"]
+        for m in mechs:
+            sw.set_mechanism(m)
+            r2: dict = {}
+            step(None)
+            for _ in range(2):
+                step(r2)
+            compare[m] = {"restore_GBps": round(payload / (statistics.mean(r2["restore_ms"]) * 1e-3) / GB, 2),
+                          "checkpoint_GBps": round(payload / (statistics.mean(r2["ckpt_ms"]) * 1e-3) / GB, 2),
+                          "swapin_GBps": round(payload / (statistics.mean(r2["swapin_ms"]) * 1e-3) / GB, 2)}
+        sw.set_mechanism(args.mechanism)
+
+    # copy-engine link peaks measured here (torch pinned copies, 2 GiB)
+    ce = {}
+    if rank == 0:
+        n = min(2 << 30, arena_bytes)
+        h = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+        for nm, (dst, src) in {"h2d": (arena[:n], h), "d2h": (h, arena[:n])}.items():
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            with torch.cuda.stream(stream):
+                dst.copy_(src, non_blocking=True)
+                a.record(stream)
+                for _ in range(3):
+                    dst.copy_(src, non_blocking=True)
+                b.record(stream)
+            b.synchronize()
+            ce[nm] = 3 * n / (a.elapsed_time(b) * 1e-3) / GB
+        del h
+
+    cpu = None
+    if rank == 0 and not args.no_cpu_baseline:
+        import oracle
+
+        sample, _ = oracle_sample_specs(specs, args.sample_bytes)
+        s_offs, s_total = W.place(sample)
+        s_host = arena[:s_total].cpu().numpy()  # same placement recipe: the arena prefix holds the sample
+        th = cpu_threads()
+        rates, sbytes = time_oracle_restore(oracle, sample, s_host, s_offs, th, 3)
+        cpu = {"value": round(statistics.mean(rates), 3), "unit": "GB/s", "cores": th, "kind": "oracle",
+               "sample": f"oracle_restore (memcpy + Sarwate CRC-32C per 1 MiB chunk) over the first {len(sample)} "
+                         f"regions of workload {name} ({sbytes} B, contents copied from the GPU arena), "
+                         f"{th} OpenMP threads, mean of 3"}
+
+    if rank == 0:
+        value = total_payload / (swapin_ms * 1e-3) / GB
+        achieved = payload / (restore_ms * 1e-3) / GB
+        peaks = json.load(open(MEASURED_PEAKS)) if os.path.exists(MEASURED_PEAKS) else {}
+        hbm_peak = peaks.get("hbm_gbs", 6650.0)
+        line = {
+            "metric": "swap-in (restore + HBM verify) throughput, whole job", "value": round(value, 3),
+            "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(step_ms, 3), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "u8", "data": "synthetic",
+            "config": {"workload": f"{name}: {desc}", "regions_per_rank": len(specs),
+                       "payload_bytes_per_rank": payload, "chunk_bytes": args.chunk, "checksum": args.checksum,
+                       "mechanism": args.mechanism,
+                       "l2": "no flush: every step moves the whole image (>> 126 MB L2)",
+                       "parallelism": "single GPU" if world == 1 else f"tp{world} shard per rank (no data collective)"},
+            "swap_in_latency_s": round(swapin_ms * 1e-3, 5),
+            "swap_in_latency_s_range": [round(min(rec["swapin_ms"]) * 1e-3, 5), round(max(rec["swapin_ms"]) * 1e-3, 5)],
+            "restore_GBps_per_gpu": round(achieved, 3),
+            "checkpoint_GBps_per_gpu": round(payload / (ckpt_ms * 1e-3) / GB, 3),
+            "roofline": {"bound": "host_link", "kernel": f"{args.mechanism} restore (mover_kernel<SCATTER>)",
+                         "achieved": round(achieved, 3), "peak": PCIE_GEN5_X16_GBPS, "unit": "GB/s",
+                         "frac": round(achieved / PCIE_GEN5_X16_GBPS, 4), "traffic": None,
+                         "peak_source": "PCIe Gen5 x16 nominal per direction after 128b/130b (MEASURED_PEAKS.json has no host-link figure)",
+                         "frac_of_measured_ce_h2d": round(achieved / ce["h2d"], 4) if ce else None},
+            "roofline_verify": {"bound": "hbm", "kernel": "mover_kernel<HASH_CHECK>",
+                                "achieved": round(payload / (verify_ms * 1e-3) / GB, 1), "peak": hbm_peak,
+                                "unit": "GB/s", "frac": round(payload / (verify_ms * 1e-3) / GB / hbm_peak, 4),
+                                "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)"},
+            "measured_ce_GBps": {k: round(v, 2) for k, v in ce.items()},
+            "mechanisms": compare,
+            "setup_s": {"fill": round(t_fill, 2), "register_pin": round(t_register, 2)},
+            "e2e": {"value": round(total_payload / (host_ms * 1e-3) / GB, 3), "unit": "GB/s",
+                    "h2d_bytes_per_step": payload, "d2h_bytes_per_step": 32,
+                    "how": "host wall clock around swap_restore + swap_verify (C ABI via ctypes), image in pinned host DRAM"},
+            "gpu_launches": int(launches),
+            "clocks": clk,
+            "cpu_baseline": cpu,
+        }
+        s = json.dumps(line)
+        print(s, flush=True)
+        if args.out:
+            with open(args.out, "a") as f:
+                f.write(s + "\n")
+    sw.close()
+    if world > 1:
+        tdist.barrier()
+        tdist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    a = parse()
+    if a.impl == "reference":
+        run_reference(a)
+    else:
+        run_ours(a)

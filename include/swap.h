@@ -1,0 +1,207 @@
+/*
+ * swap.h — C ABI of libswap: B200-native checkpoint/restore of an inference engine's
+ * GPU memory state (the data path of SwapServeLLM's model hot-swap).
+ *
+ * Paper: Stoyanov et al., "Engine-Agnostic Model Hot-Swapping for Cost-Effective LLM
+ * Inference", SC Workshops '25 (/root/reference/PAPER.md, "P:Lnnn" = line nnn).
+ *   - preempt = "saves the amount of GPU memory in use. It then creates an in-memory
+ *     snapshot ... thus freeing GPU capacity" (§4.2)      -> swap_checkpoint + swap_sync
+ *   - snapshot taken once after initialisation, restored many times (§3, §3.2)
+ *                                                                  -> REGISTERED -> CHECKPOINTED -> RESTORED*
+ *   - swap-in = reserve memory, restore GPU state, check the engine (§3.3, §3.4);
+ *     its time "primarily depends on the GPU memory utilized" (§5.3)
+ *                                                                  -> swap_restore + swap_verify
+ *   - per-GPU topology fixed at init, per-GPU reservations (§6) -> one ctx per (process, device, rank)
+ * The paper's mechanism is the closed cuda-checkpoint driver path; the image
+ * layout, chunk checksums and manifest below are this library's (DESIGN.md §"Readings",
+ * SURVEY.md §8(c)), identical to the CPU oracle's definition in oracle/oracle.c.
+ *
+ * Conventions (all entry points):
+ *   - Every call returns swap_status: 0 = OK, < 0 = error. Nothing aborts or throws.
+ *   - Argument checks run in a fixed order: null/arg -> config -> alignment -> overlap ->
+ *     duplicate id -> state -> CUDA; the first failing check's code is returned.
+ *   - CUDA failures return SWAP_ECUDA; swap_last_error(ctx) holds the text.
+ *   - Streams are cudaStream_t values passed as swap_stream_t (NULL = legacy default stream).
+ *   - Calls on one ctx are NOT thread-safe; the caller serialises them (the paper's
+ *     per-backend write lock, §3.5). Distinct ctxs are independent.
+ *   - There is no CPU fallback: with no usable sm_100 device, swap_create returns SWAP_ECUDA.
+ */
+#ifndef SWAP_H
+#define SWAP_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(__GNUC__)
+#define SWAP_API __attribute__((visibility("default")))
+#else
+#define SWAP_API
+#endif
+
+typedef int32_t swap_status;
+#define SWAP_OK 0
+#define SWAP_EINVAL (-1)       /* bad argument, config or region table */
+#define SWAP_ENOMEM (-2)       /* host pinning or device allocation failed */
+#define SWAP_ECUDA (-3)        /* CUDA runtime error; see swap_last_error */
+#define SWAP_ESTATE (-4)       /* call not valid in the ctx's current state */
+#define SWAP_ECORRUPT (-5)     /* manifest CRC bad, or >= 1 chunk checksum mismatch */
+#define SWAP_ENCCL (-6)        /* inconsistent global manifest (rank/world mismatch) */
+#define SWAP_EUNSUPPORTED (-7) /* valid but unsupported here (e.g. chunk_bytes > 2 GiB) */
+#define SWAP_EINTERNAL (-8)
+
+/* Chunk checksum H_K (reading 1-3): */
+#define SWAP_CHECKSUM_CRC32C 1u /* CRC-32C/ISCSI (RFC 3720), zero-extended to u64 */
+#define SWAP_CHECKSUM_XXH64 2u  /* XXH64, seed 0 for every chunk */
+
+/* Data mover for checkpoint/restore (the image bytes are identical for all of them): */
+#define SWAP_MECH_SM 0u          /* one SM kernel: 16-B vector loads/stores to mapped pinned host
+                                    memory with the chunk checksum fused from the same registers */
+#define SWAP_MECH_CE_REGION 1u   /* copy engine: cudaMemcpyAsync per region + separate HBM hash pass */
+#define SWAP_MECH_CE_CHUNK 2u    /* copy engine: cudaMemcpyAsync per chunk + HBM hash pass */
+#define SWAP_MECH_CE_BATCH 3u    /* copy engine: one cudaMemcpyBatchAsync per call + HBM hash pass */
+#define SWAP_MECH_SM_NOCHECK 4u  /* diagnostic: the SM kernel with the checksum compiled out. Checkpoint
+                                    writes c_g = 0; restore reports no mismatches. Only for measuring
+                                    the fused-checksum overhead (BASELINE.json north_star: <= 5 %). */
+
+/* Region kinds (manifest only; movement is kind-agnostic) */
+#define SWAP_KIND_WEIGHTS 0u
+#define SWAP_KIND_KV 1u
+#define SWAP_KIND_WORKSPACE 2u
+#define SWAP_KIND_OTHER 3u
+
+/* One registered device allocation. dev_addr must be 16-B aligned; bytes may be any
+ * value (0 allowed: a region record with no chunks). Non-empty regions must not
+ * overlap; ids must be unique. Regions are laid out in the image in the order given. */
+typedef struct {
+  uint64_t dev_addr;
+  uint64_t bytes;
+  uint32_t id;
+  uint32_t kind; /* SWAP_KIND_* (0..3) */
+} swap_region_t;
+
+typedef struct {
+  uint64_t chunk_bytes; /* checksum granule C: power of 2, >= 16, <= 2^31; 0 -> 1 MiB */
+  uint64_t align;       /* image offset alignment A: power of 2, >= 16; 0 -> 4096 */
+  uint32_t checksum;    /* SWAP_CHECKSUM_*; 0 -> CRC32C */
+  uint32_t mechanism;   /* SWAP_MECH_*; default SWAP_MECH_SM */
+  int32_t device;       /* CUDA device ordinal the regions live on */
+  int32_t rank;         /* 0 <= rank < world (tensor-parallel shard index) */
+  int32_t world;        /* >= 1 */
+  uint32_t grid_ctas;   /* SM mover grid; 0 -> auto (2 CTAs per SM) */
+  uint32_t seg_bytes;   /* CRC32C work split inside a chunk: power of 2, >= 4096; 0 -> 256 KiB */
+  uint32_t reserved;    /* must be 0 */
+} swap_config_t;
+
+typedef struct {
+  uint64_t n_bad;           /* chunks whose checksum over the bytes moved by the last restore
+                               differs from the manifest (fused check) */
+  uint64_t first_bad_chunk; /* lowest such global chunk index, or UINT64_MAX */
+  uint64_t hbm_n_bad;       /* same, recomputed from device memory by the HBM pass (if run) */
+  uint64_t hbm_first_bad;   /* lowest such chunk, or UINT64_MAX */
+  uint32_t manifest_ok;     /* 1 if the manifest CRC holds */
+  uint32_t hbm_checked;     /* 1 if the HBM pass ran in this call */
+} swap_verify_result_t;
+
+/* Exactly 64 bytes, little-endian; the unit of the multi-GPU all-gather. */
+typedef struct {
+  uint32_t rank, world, checksum, n_regions;
+  uint64_t n_chunks, payload_bytes, image_bytes;
+  uint64_t manifest_crc; /* the manifest's trailing CRC-32C */
+  uint64_t chunk_digest; /* CRC-32C over the n_chunks little-endian u64 chunk checksums */
+  uint64_t reserved;     /* 0 */
+} swap_shard_summary_t;
+
+/* Opaque per-(process, device, rank) context. */
+typedef struct swap_ctx swap_ctx_t;
+/* A cudaStream_t (struct CUstream_st*) without pulling CUDA headers into this file. */
+typedef struct CUstream_st* swap_stream_t;
+
+/* Fills *cfg with the defaults above (device 0, rank 0, world 1). */
+SWAP_API void swap_config_default(swap_config_t* cfg);
+
+/* Validates cfg and binds the ctx to cfg->device. EINVAL on a bad cfg; ECUDA when the
+ * device is missing or not sm_100. *out receives a ctx the caller frees with swap_destroy. */
+SWAP_API swap_status swap_create(const swap_config_t* cfg, swap_ctx_t** out);
+
+/* Copies the table (caller keeps ownership of `regions` and of the device memory),
+ * validates it, plans the image (offsets, chunks), allocates the library-owned
+ * pinned + mapped host image (zero-filled, so padding is 0), builds and uploads the
+ * work descriptors. Allowed once per ctx. State -> REGISTERED. The caller must keep
+ * every region allocated at the same address until swap_destroy. */
+SWAP_API swap_status swap_register_regions(swap_ctx_t* ctx, const swap_region_t* regions, size_t n);
+
+/* Enqueues the gather of every region into the image plus the chunk checksums (written
+ * into the manifest's chunk records) on `stream`. Needs REGISTERED or RESTORED (or
+ * CHECKPOINTED: re-snapshot). The caller must not write the regions until the stream
+ * reaches this point. State -> CHECKPOINT_PENDING; swap_sync completes it. */
+SWAP_API swap_status swap_checkpoint(swap_ctx_t* ctx, swap_stream_t stream);
+
+/* Synchronises `stream`, then finalises the manifest (header, region records, trailing
+ * CRC-32C). State CHECKPOINT_PENDING -> CHECKPOINTED; a no-op in other states. */
+SWAP_API swap_status swap_sync(swap_ctx_t* ctx, swap_stream_t stream);
+
+/* Needs CHECKPOINTED or RESTORED (restore many times). Checks on the host, before
+ * anything is enqueued, that the manifest CRC holds and that the manifest describes the
+ * registered layout (else ECORRUPT, nothing written). Then enqueues the scatter of the image
+ * to the recorded device addresses with the fused per-chunk compare. Mismatches do not stop
+ * the scatter: every byte is written and the result is reported by swap_verify.
+ * The caller must not read the regions until the stream reaches this point. State -> RESTORED. */
+SWAP_API swap_status swap_restore(swap_ctx_t* ctx, swap_stream_t stream);
+
+/* Needs RESTORED. If hbm_pass != 0, first enqueues the HBM re-read of every region with
+ * checksums recomputed against the manifest. Synchronises `stream` and fills *res.
+ * Returns ECORRUPT iff a mismatch was found or the manifest is bad, else OK. */
+SWAP_API swap_status swap_verify(swap_ctx_t* ctx, swap_stream_t stream, int hbm_pass, swap_verify_result_t* res);
+
+/* Selects the data mover for later calls (SWAP_MECH_*). The image format is unchanged. */
+SWAP_API swap_status swap_set_mechanism(swap_ctx_t* ctx, uint32_t mechanism);
+
+/* Borrowed views, valid until swap_destroy. The manifest is final only after swap_sync.
+ * The image is writable: a caller may load a stored image into it and call swap_import. */
+SWAP_API swap_status swap_get_manifest(const swap_ctx_t* ctx, const void** bytes, size_t* n);
+SWAP_API swap_status swap_get_image(const swap_ctx_t* ctx, void** host, size_t* n);
+SWAP_API swap_status swap_get_summary(const swap_ctx_t* ctx, swap_shard_summary_t* out);
+
+/* Declares that the image buffer now holds a complete image (e.g. loaded from storage):
+ * checks the manifest CRC and that it describes the registered layout (ECORRUPT if not).
+ * Needs REGISTERED, CHECKPOINTED or RESTORED. State -> CHECKPOINTED. */
+SWAP_API swap_status swap_import(swap_ctx_t* ctx);
+
+/* After the all-gather of every rank's summary (rank order): checks world and that entry r
+ * has rank r and this ctx's own entry equals its summary (ENCCL otherwise), stores the
+ * global manifest and writes the global digest (CRC-32C of the world*64 bytes). */
+SWAP_API swap_status swap_set_global(swap_ctx_t* ctx, const swap_shard_summary_t* all, int world, uint64_t* global_digest);
+
+/* Ctx-free half of swap_set_global, usable without a GPU: checks that `all` holds `world`
+ * summaries with all[r].rank == r and all[r].world == world (ENCCL otherwise) and writes
+ * the global digest = CRC-32C of the world*64 summary bytes. */
+SWAP_API swap_status swap_merge_global(const swap_shard_summary_t* all, int world, uint64_t* global_digest);
+
+/* Device time (CUDA events recorded on the caller's stream right before and after the
+ * movers) of the last checkpoint (updated by swap_sync), and of the last restore and HBM
+ * verify pass (updated by swap_verify). 0 if the phase has not run. */
+typedef struct {
+  float checkpoint_ms; /* gather kernel, or hash pass + copy-engine copies */
+  float restore_ms;    /* scatter kernel, or copy-engine copies + hash pass */
+  float verify_ms;     /* HBM verify pass */
+  float reserved;
+} swap_timings_t;
+SWAP_API swap_status swap_get_timings(const swap_ctx_t* ctx, swap_timings_t* out);
+
+/* Number of libswap kernels this ctx has launched in total (for the bench's gpu_launches). */
+SWAP_API swap_status swap_get_launch_count(const swap_ctx_t* ctx, uint64_t* launches);
+
+SWAP_API const char* swap_status_str(swap_status s);
+SWAP_API const char* swap_last_error(const swap_ctx_t* ctx);
+
+/* Frees the pinned image, descriptors and device scratch. NULL is a no-op. */
+SWAP_API void swap_destroy(swap_ctx_t* ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SWAP_H */

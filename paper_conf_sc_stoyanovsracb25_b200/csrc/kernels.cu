@@ -1,0 +1,455 @@
+// kernels.cu — libswap's sm_100a data movers (see kernels.cuh for the mode list).
+//
+// Design:
+//  * Persistent grid (2 CTAs x 512 threads per SM). A CTA takes WARPS consecutive segment
+//    descriptors per round; thread 0 stages them into shared memory with a TMA bulk copy
+//    (cp.async.bulk + mbarrier complete_tx), double-buffered two rounds ahead.
+//  * One warp moves one segment in 512-B steps: lane l owns bytes [16l, 16l+16) of every
+//    512-B block, so each warp-wide ld/st.v4 is one fully coalesced 512-B transaction on
+//    HBM and on the PCIe link to the mapped pinned image. U blocks are loaded before any
+//    store or hash step, keeping U x 512 B in flight per warp.
+//  * CRC-32C from the same registers: lane l keeps T_l = F(0, its strided sub-stream) with
+//    the Horner step T <- F(Z^496(T), piece) (slicing-by-16 + a 4-lookup shift), tables in
+//    shared memory. The warp folds lanes with x^(8*16*(31-l)) and an XOR shuffle reduction;
+//    a ragged tail (< 512 B) is staged in shared memory and finished by lane 0 bytewise.
+//    Segments of one chunk are combined by the last-arriving warp (atomic counter) with
+//    the GF(2) shift crc(A||B) = Z^|B|(crc(A)) ^ crc(B).
+//  * XXH64 (non-combinable): one warp per chunk; stripe words are routed to 4 accumulator
+//    lanes with shuffles, the tail and finalisation run on lane 0.
+#include <cstdio>
+
+#include "kernels.cuh"
+
+namespace swk {
+
+constexpr uint32_t POLY = 0x82F63B78u;  // CRC-32C, reflected
+constexpr int THREADS = 512;
+constexpr int WARPS = THREADS / 32;
+constexpr int U = 8;  // 512-B blocks in flight per warp
+constexpr int TAIL_BYTES = 512;
+
+constexpr uint64_t P1 = 0x9E3779B185EBCA87ull, P2 = 0xC2B2AE3D27D4EB4Full, P3 = 0x165667B19E3779F9ull,
+                   P4 = 0x85EBCA77C2B2AE63ull, P5 = 0x27D4EB2F165667C5ull;
+
+// ------------------------------------------------------------------ host: tables
+static uint32_t step_byte(uint32_t c) {  // one zero byte through the register, bit-serial
+  for (int k = 0; k < 8; ++k) c = (c & 1u) ? (c >> 1) ^ POLY : (c >> 1);
+  return c;
+}
+
+uint32_t host_multmodp(uint32_t a, uint32_t b) {  // a*b mod P, reflected (bit 31 = x^0)
+  uint32_t p = 0;
+  for (int i = 0; i < 32; ++i) {
+    if ((a >> (31 - i)) & 1u) p ^= b;
+    b = (b & 1u) ? (b >> 1) ^ POLY : (b >> 1);
+  }
+  return p;
+}
+
+uint32_t host_x2nmodp(uint64_t n, unsigned k, const uint32_t* x2n) {  // x^(n*2^k) mod P
+  uint32_t p = 1u << 31;
+  while (n) {
+    if (n & 1) p = host_multmodp(x2n[k & 31], p);
+    n >>= 1;
+    ++k;
+  }
+  return p;
+}
+
+void build_tables(uint32_t* tab) {
+  uint32_t* t = tab + TAB_T16;
+  for (uint32_t b = 0; b < 256; ++b) t[b] = step_byte(b);  // T_0 = one byte
+  for (int k = 1; k < 16; ++k)
+    for (uint32_t b = 0; b < 256; ++b) {
+      uint32_t v = t[(k - 1) * 256 + b];
+      t[k * 256 + b] = t[v & 0xFFu] ^ (v >> 8);  // one more zero byte
+    }
+  for (int j = 0; j < 4; ++j)
+    for (uint32_t b = 0; b < 256; ++b) {
+      uint32_t v = b << (8 * j);
+      for (int z = 0; z < 496; ++z) v = t[v & 0xFFu] ^ (v >> 8);
+      tab[TAB_Z496 + j * 256 + b] = v;
+    }
+  uint32_t* x2n = tab + TAB_X2N;
+  x2n[0] = 1u << 30;  // x^1
+  for (int k = 1; k < 32; ++k) x2n[k] = host_multmodp(x2n[k - 1], x2n[k - 1]);
+  for (int l = 0; l < 32; ++l) tab[TAB_LANE + l] = host_x2nmodp(16ull * (31 - l), 3, x2n);
+}
+
+// ------------------------------------------------------------------ device helpers
+__device__ __forceinline__ int4 ld_stream(const void* p) {
+  int4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ void st_stream(void* p, const int4& v) {
+  asm volatile("st.global.L1::no_allocate.v4.s32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z),
+               "r"(v.w)
+               : "memory");
+}
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// a * b mod P (reflected), branch-free.
+__device__ __forceinline__ uint32_t multmodp(uint32_t a, uint32_t b) {
+  uint32_t p = 0;
+#pragma unroll
+  for (int i = 0; i < 32; ++i) {
+    p ^= b & (0u - ((a >> (31 - i)) & 1u));
+    b = (b >> 1) ^ (POLY & (0u - (b & 1u)));
+  }
+  return p;
+}
+__device__ uint32_t x2nmodp(uint64_t n, unsigned k, const uint32_t* __restrict__ x2n) {
+  uint32_t p = 1u << 31;
+  while (n) {
+    if (n & 1) p = multmodp(__ldg(x2n + (k & 31)), p);
+    n >>= 1;
+    ++k;
+  }
+  return p;
+}
+// Z^len(s): the register after `len` zero bytes.
+__device__ __forceinline__ uint32_t crc_shift(uint32_t s, uint64_t len, const uint32_t* x2n) {
+  return multmodp(x2nmodp(len, 3, x2n), s);
+}
+
+// One 16-B piece of a lane's strided sub-stream: T <- F(Z^496(T), piece).
+__device__ __forceinline__ uint32_t crc_piece(uint32_t T, const int4& v, const uint32_t* __restrict__ sT) {
+  const uint32_t* Z = sT + TAB_Z496;
+  uint32_t s = Z[T & 0xFF] ^ Z[256 + ((T >> 8) & 0xFF)] ^ Z[512 + ((T >> 16) & 0xFF)] ^ Z[768 + (T >> 24)];
+  uint32_t a = static_cast<uint32_t>(v.x) ^ s, b = v.y, c = v.z, d = v.w;
+  return sT[15 * 256 + (a & 0xFF)] ^ sT[14 * 256 + ((a >> 8) & 0xFF)] ^ sT[13 * 256 + ((a >> 16) & 0xFF)] ^
+         sT[12 * 256 + (a >> 24)] ^ sT[11 * 256 + (b & 0xFF)] ^ sT[10 * 256 + ((b >> 8) & 0xFF)] ^
+         sT[9 * 256 + ((b >> 16) & 0xFF)] ^ sT[8 * 256 + (b >> 24)] ^ sT[7 * 256 + (c & 0xFF)] ^
+         sT[6 * 256 + ((c >> 8) & 0xFF)] ^ sT[5 * 256 + ((c >> 16) & 0xFF)] ^ sT[4 * 256 + (c >> 24)] ^
+         sT[3 * 256 + (d & 0xFF)] ^ sT[2 * 256 + ((d >> 8) & 0xFF)] ^ sT[1 * 256 + ((d >> 16) & 0xFF)] ^
+         sT[0 * 256 + (d >> 24)];
+}
+
+__device__ __forceinline__ uint64_t rotl64(uint64_t x, int r) { return (x << r) | (x >> (64 - r)); }
+__device__ __forceinline__ uint64_t xround(uint64_t acc, uint64_t in) { return rotl64(acc + in * P2, 31) * P1; }
+__device__ __forceinline__ uint64_t xmerge(uint64_t h, uint64_t v) { return (h ^ xround(0, v)) * P1 + P4; }
+__device__ __forceinline__ uint64_t ld_u64_smem(const uint8_t* p) {  // 8-aligned not guaranteed
+  uint64_t v = 0;
+#pragma unroll
+  for (int i = 7; i >= 0; --i) v = (v << 8) | p[i];
+  return v;
+}
+
+// The result of chunk g: store (checkpoint / hash pass) or compare (restore / verify).
+template <int MODE>
+__device__ __forceinline__ void chunk_result(const Params& p, uint32_t g, uint64_t c) {
+  if (MODE == GATHER || MODE == HASH_STORE) {
+    p.cs_out[4ull * g] = c;
+  } else {
+    uint64_t e = p.cs_exp[4ull * g];
+    if (e != c) {
+      atomicAdd(p.n_bad, 1ull);
+      atomicMin(p.first_bad, static_cast<unsigned long long>(g));
+    }
+  }
+}
+
+// Stage the ragged tail [base, base + r) (r < 512) into smem (and copy it to dst).
+template <int MODE>
+__device__ __forceinline__ void stage_tail(const uint8_t* src, uint8_t* dst, uint32_t r, uint8_t* tail, int lane) {
+  const uint32_t lo = lane * 16u;
+  if (lo + 16 <= r) {
+    int4 v = ld_stream(src + lo);
+    *reinterpret_cast<int4*>(tail + lo) = v;
+    if (MODE == GATHER || MODE == SCATTER) st_stream(dst + lo, v);
+  } else if (lo < r) {
+    for (uint32_t i = lo; i < r; ++i) {
+      uint8_t b = src[i];
+      tail[i] = b;
+      if (MODE == GATHER || MODE == SCATTER) dst[i] = b;
+    }
+  }
+  __syncwarp();
+}
+
+// ------------------------------------------------------------------ segment movers
+template <int MODE, int KIND>
+__device__ __forceinline__ void move_segment(const Params& p, const SegDesc& d, uint32_t idx, const uint32_t* sT,
+                                             uint8_t* tail, int lane) {
+  const uint8_t* src = reinterpret_cast<const uint8_t*>(MODE == SCATTER ? d.host : d.dev);
+  uint8_t* dst = reinterpret_cast<uint8_t*>(MODE == SCATTER ? d.dev : d.host);
+  const uint32_t len = d.bytes;
+  const uint32_t nblk = len / 512u;
+  constexpr bool COPY = (MODE == GATHER || MODE == SCATTER);
+
+  if (KIND == KIND_XXH64) {
+    // acc lanes 0..3 hold v1..v4 (seed 0).
+    uint64_t acc = lane == 0 ? P1 + P2 : lane == 1 ? P2 : lane == 2 ? 0ull : 0ull - P1;
+    const int half = (lane & 3) >> 1;
+    uint32_t b = 0;
+    for (; b < nblk; b += U) {
+      const uint32_t nb = nblk - b < (uint32_t)U ? nblk - b : (uint32_t)U;
+      int4 v[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+        if (u < (int)nb) v[u] = ld_stream(src + (size_t)(b + u) * 512 + lane * 16);
+      if (COPY) {
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+          if (u < (int)nb) st_stream(dst + (size_t)(b + u) * 512 + lane * 16, v[u]);
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (u < (int)nb) {
+          const uint64_t lo = (uint64_t)(uint32_t)v[u].x | ((uint64_t)(uint32_t)v[u].y << 32);
+          const uint64_t hi = (uint64_t)(uint32_t)v[u].z | ((uint64_t)(uint32_t)v[u].w << 32);
+#pragma unroll
+          for (int s = 0; s < 16; ++s) {
+            const int srcl = 2 * s + half;
+            const uint64_t wlo = __shfl_sync(0xffffffffu, lo, srcl);
+            const uint64_t whi = __shfl_sync(0xffffffffu, hi, srcl);
+            const uint64_t w = (lane & 1) ? whi : wlo;
+            if (lane < 4) acc = xround(acc, w);
+          }
+        }
+      }
+    }
+    const uint32_t r = len - nblk * 512u;
+    const uint64_t base = (uint64_t)nblk * 512u;
+    stage_tail<MODE>(src + base, COPY ? dst + base : nullptr, r, tail, lane);
+    const uint64_t v1 = __shfl_sync(0xffffffffu, acc, 0), v2 = __shfl_sync(0xffffffffu, acc, 1);
+    const uint64_t v3 = __shfl_sync(0xffffffffu, acc, 2), v4 = __shfl_sync(0xffffffffu, acc, 3);
+    if (lane == 0) {
+      uint64_t a1 = v1, a2 = v2, a3 = v3, a4 = v4;
+      uint32_t i = 0;
+      for (; i + 32 <= r; i += 32) {
+        a1 = xround(a1, ld_u64_smem(tail + i));
+        a2 = xround(a2, ld_u64_smem(tail + i + 8));
+        a3 = xround(a3, ld_u64_smem(tail + i + 16));
+        a4 = xround(a4, ld_u64_smem(tail + i + 24));
+      }
+      uint64_t h;
+      if (len >= 32) {
+        h = rotl64(a1, 1) + rotl64(a2, 7) + rotl64(a3, 12) + rotl64(a4, 18);
+        h = xmerge(h, a1);
+        h = xmerge(h, a2);
+        h = xmerge(h, a3);
+        h = xmerge(h, a4);
+      } else {
+        h = P5;
+      }
+      h += len;
+      for (; i + 8 <= r; i += 8) {
+        h ^= xround(0, ld_u64_smem(tail + i));
+        h = rotl64(h, 27) * P1 + P4;
+      }
+      if (i + 4 <= r) {
+        uint32_t w = (uint32_t)tail[i] | ((uint32_t)tail[i + 1] << 8) | ((uint32_t)tail[i + 2] << 16) |
+                     ((uint32_t)tail[i + 3] << 24);
+        h ^= (uint64_t)w * P1;
+        h = rotl64(h, 23) * P2 + P3;
+        i += 4;
+      }
+      for (; i < r; ++i) {
+        h ^= (uint64_t)tail[i] * P5;
+        h = rotl64(h, 11) * P1;
+      }
+      h ^= h >> 33;
+      h *= P2;
+      h ^= h >> 29;
+      h *= P3;
+      h ^= h >> 32;
+      chunk_result<MODE>(p, d.chunk, h);
+    }
+    return;
+  }
+
+  // CRC-32C or no checksum.
+  uint32_t T = 0;
+  uint32_t b = 0;
+  for (; b + U <= nblk; b += U) {
+    int4 v[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) v[u] = ld_stream(src + (size_t)(b + u) * 512 + lane * 16);
+    if (COPY) {
+#pragma unroll
+      for (int u = 0; u < U; ++u) st_stream(dst + (size_t)(b + u) * 512 + lane * 16, v[u]);
+    }
+    if (KIND == KIND_CRC32C) {
+#pragma unroll
+      for (int u = 0; u < U; ++u) T = crc_piece(T, v[u], sT);
+    }
+  }
+  for (; b < nblk; ++b) {
+    int4 v = ld_stream(src + (size_t)b * 512 + lane * 16);
+    if (COPY) st_stream(dst + (size_t)b * 512 + lane * 16, v);
+    if (KIND == KIND_CRC32C) T = crc_piece(T, v, sT);
+  }
+  const uint32_t r = len - nblk * 512u;
+  const uint64_t base = (uint64_t)nblk * 512u;
+  if (KIND != KIND_CRC32C) {
+    if (r) stage_tail<MODE>(src + base, COPY ? dst + base : nullptr, r, tail, lane);
+    return;
+  }
+  // Fold lanes: X = XOR_l Z^(16*(31-l))(T_l) = F(0, full blocks).
+  uint32_t X = nblk ? multmodp(sT[TAB_LANE + lane], T) : 0u;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) X ^= __shfl_xor_sync(0xffffffffu, X, o);
+  if (r) stage_tail<MODE>(src + base, COPY ? dst + base : nullptr, r, tail, lane);
+  if (lane == 0) {
+    uint32_t S = X;  // continue the register through the tail: F(X, tail) = F(0, full || tail)
+    for (uint32_t i = 0; i < r; ++i) S = sT[(S ^ tail[i]) & 0xFFu] ^ (S >> 8);
+    const uint32_t* x2n = p.tables + TAB_X2N;
+    if (d.nseg == 1) {
+      const uint32_t zi = (len == p.chunk_bytes) ? p.zinit_c : crc_shift(0xFFFFFFFFu, len, x2n);
+      chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ S)));
+      return;
+    }
+    p.partial[idx] = S;
+    __threadfence();
+    const uint32_t prev = atomicAdd(p.arrive + d.chunk, 1u);
+    if (prev == d.nseg - 1) {  // last arriver combines the chunk's segments in order
+      __threadfence();
+      const uint32_t first = idx - d.seg;
+      const uint32_t last_len = __ldcg(&p.desc[first + d.nseg - 1].bytes);
+      uint32_t acc = 0;
+      for (uint32_t s = 0; s < d.nseg; ++s) {
+        const uint32_t f = __ldcg(p.partial + first + s);
+        if (s == 0) {
+          acc = f;
+        } else if (s + 1 < d.nseg || last_len == p.seg_bytes) {
+          acc = multmodp(p.xseg, acc) ^ f;
+        } else {
+          acc = crc_shift(acc, last_len, x2n) ^ f;
+        }
+      }
+      p.arrive[d.chunk] = 0;
+      const uint64_t L = (uint64_t)(d.nseg - 1) * p.seg_bytes + last_len;
+      const uint32_t zi = (L == p.chunk_bytes) ? p.zinit_c : crc_shift(0xFFFFFFFFu, L, x2n);
+      chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ acc)));
+    }
+  }
+}
+
+// ------------------------------------------------------------------ the persistent kernel
+template <int KIND>
+struct SmemLayout {
+  static constexpr int tab_words = (KIND == KIND_CRC32C) ? TAB_SMEM_WORDS : 0;
+  static constexpr size_t off_desc = ((size_t)tab_words * 4 + 127) / 128 * 128;
+  static constexpr size_t off_bar = off_desc + 2 * WARPS * sizeof(SegDesc);
+  static constexpr size_t off_tail = (off_bar + 16 + 127) / 128 * 128;
+  static constexpr size_t bytes = off_tail + (size_t)WARPS * TAIL_BYTES;
+};
+
+template <int MODE, int KIND>
+__global__ void __launch_bounds__(THREADS, 2) mover_kernel(const Params p) {
+  using L = SmemLayout<KIND>;
+  extern __shared__ __align__(128) uint8_t smem[];
+  uint32_t* sT = reinterpret_cast<uint32_t*>(smem);
+  SegDesc* sDesc = reinterpret_cast<SegDesc*>(smem + L::off_desc);
+  uint64_t* sBar = reinterpret_cast<uint64_t*>(smem + L::off_bar);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  uint8_t* tail = smem + L::off_tail + warp * TAIL_BYTES;
+
+  if (KIND == KIND_CRC32C)
+    for (int i = tid; i < L::tab_words; i += THREADS) sT[i] = __ldg(p.tables + i);
+
+  const uint32_t per_round = gridDim.x * WARPS;
+  const uint32_t first0 = blockIdx.x * WARPS;
+  const uint32_t rounds = p.n_desc > first0 ? (p.n_desc - first0 + per_round - 1) / per_round : 0u;
+  auto issue = [&](uint32_t r) {
+    const uint32_t first = r * per_round + first0;
+    const uint32_t cnt = min((uint32_t)WARPS, p.n_desc - first);
+    uint64_t* bar = sBar + (r & 1);
+    mbar_expect_tx(bar, cnt * (uint32_t)sizeof(SegDesc));
+    bulk_g2s(sDesc + (r & 1) * WARPS, p.desc + first, cnt * (uint32_t)sizeof(SegDesc), bar);
+  };
+  if (tid == 0) {
+    mbar_init(sBar, 1);
+    mbar_init(sBar + 1, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    if (rounds > 0) issue(0);
+    if (rounds > 1) issue(1);
+  }
+  __syncthreads();
+
+  for (uint32_t r = 0; r < rounds; ++r) {
+    mbar_wait(sBar + (r & 1), (r >> 1) & 1u);
+    const uint32_t idx = r * per_round + first0 + warp;
+    if (idx < p.n_desc) {
+      const SegDesc d = sDesc[(r & 1) * WARPS + warp];
+      move_segment<MODE, KIND>(p, d, idx, sT, tail, lane);
+    }
+    __syncthreads();
+    if (tid == 0 && r + 2 < rounds) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      issue(r + 2);
+    }
+  }
+}
+
+int mover_threads() { return THREADS; }
+size_t mover_smem_bytes(int kind) {
+  return kind == KIND_CRC32C ? SmemLayout<KIND_CRC32C>::bytes : SmemLayout<KIND_NONE>::bytes;
+}
+
+template <int MODE, int KIND>
+static cudaError_t launch_t(const Params& p, int grid, cudaStream_t s) {
+  const size_t smem = SmemLayout<KIND>::bytes;
+  static unsigned long long attr_set = 0;  // bit per device: the attribute is per function, per device
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (!((attr_set >> (dev & 63)) & 1ull)) {
+    e = cudaFuncSetAttribute(mover_kernel<MODE, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr_set |= 1ull << (dev & 63);
+  }
+  mover_kernel<MODE, KIND><<<grid, THREADS, smem, s>>>(p);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_mover(int mode, int kind, const Params& p, int grid, cudaStream_t s) {
+  if (p.n_desc == 0) return cudaSuccess;
+#define SWK_CASE(M, K) \
+  if (mode == M && kind == K) return launch_t<M, K>(p, grid, s);
+  SWK_CASE(GATHER, KIND_NONE)
+  SWK_CASE(GATHER, KIND_CRC32C)
+  SWK_CASE(GATHER, KIND_XXH64)
+  SWK_CASE(SCATTER, KIND_NONE)
+  SWK_CASE(SCATTER, KIND_CRC32C)
+  SWK_CASE(SCATTER, KIND_XXH64)
+  SWK_CASE(HASH_STORE, KIND_CRC32C)
+  SWK_CASE(HASH_STORE, KIND_XXH64)
+  SWK_CASE(HASH_CHECK, KIND_CRC32C)
+  SWK_CASE(HASH_CHECK, KIND_XXH64)
+#undef SWK_CASE
+  return cudaErrorInvalidValue;
+}
+
+}  // namespace swk

@@ -1,0 +1,70 @@
+// kernels.cuh — device-side data movers of libswap (sm_100a). Internal header.
+//
+// One persistent kernel family moves bytes between HBM and the mapped pinned host image
+// and computes the per-chunk checksum from the same registers (BASELINE.json north_star
+// (a)+(b); SURVEY.md §2d K1 gather_ckpt, K2 scatter_restore, K3 verify_hbm):
+//   GATHER      HBM -> host image, c_g stored into the manifest chunk record   (checkpoint)
+//   SCATTER     host image -> HBM, c_g compared with the manifest               (restore)
+//   HASH_STORE  HBM only, c_g stored      (copy-engine checkpoint's hash pass, K4)
+//   HASH_CHECK  HBM only, c_g compared    (HBM verify pass K3; copy-engine restore's check)
+// Work unit: a "segment" descriptor (32 B). CRC-32C chunks are split into segments of
+// seg_bytes whose partial CRCs are combined by the last-arriving warp; XXH64 is not
+// combinable, so an XXH64 segment is a whole chunk.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace swk {
+
+struct SegDesc {
+  uint64_t dev;    // device address of the segment's first byte
+  uint64_t host;   // host (mapped, UVA) address of the segment's first byte in the image
+  uint32_t bytes;  // segment length
+  uint32_t chunk;  // global chunk index g
+  uint32_t seg;    // index of this segment inside chunk g
+  uint32_t nseg;   // number of segments of chunk g
+};
+static_assert(sizeof(SegDesc) == 32, "descriptor is 32 B");
+
+struct DevStatus {
+  unsigned long long n_bad, first_bad;          // fused check of the last restore
+  unsigned long long hbm_n_bad, hbm_first_bad;  // HBM verify pass
+};
+
+enum Mode : int { GATHER = 0, SCATTER = 1, HASH_STORE = 2, HASH_CHECK = 3 };
+enum Kind : int { KIND_NONE = 0, KIND_CRC32C = 1, KIND_XXH64 = 2 };
+
+// CRC tables blob, built on the host by build_tables() and uploaded once per ctx.
+constexpr int TAB_T16 = 0;          // [16][256] slicing-by-16: T_k[b] = F(0, b . 0^k)
+constexpr int TAB_Z496 = 16 * 256;  // [4][256]  Z^496 applied to byte j of a register
+constexpr int TAB_LANE = TAB_Z496 + 4 * 256;  // [32] x^(8*16*(31-l)) mod P
+constexpr int TAB_X2N = TAB_LANE + 32;        // [32] x^(2^k) mod P
+constexpr int TAB_WORDS = TAB_X2N + 32;
+constexpr int TAB_SMEM_WORDS = TAB_LANE + 32;  // the part staged in shared memory
+
+struct Params {
+  const SegDesc* desc;
+  uint32_t n_desc;
+  uint32_t seg_bytes;            // CRC split size (all segments but a chunk's last)
+  uint32_t* partial;             // [n_desc] partial F(0, segment)
+  uint32_t* arrive;              // [n_chunks] arrival counters (kept at 0 between launches)
+  uint64_t* cs_out;              // &chunk_record[0].c_g in the mapped manifest; stride 4 u64
+  const uint64_t* cs_exp;        // same field, read for compares
+  unsigned long long* n_bad;     // mismatch counter
+  unsigned long long* first_bad; // atomicMin target
+  const uint32_t* tables;        // TAB_WORDS words in device memory
+  uint64_t chunk_bytes;          // C
+  uint32_t zinit_c;              // Z^C(0xFFFFFFFF): the init term of a full chunk
+  uint32_t xseg;                 // x^(8*seg_bytes) mod P
+};
+
+void build_tables(uint32_t* tab /* TAB_WORDS */);
+uint32_t host_x2nmodp(uint64_t n, unsigned k, const uint32_t* x2n);
+uint32_t host_multmodp(uint32_t a, uint32_t b);
+
+// Launch mover kernel <mode, kind> with `grid` CTAs on `stream`.
+cudaError_t launch_mover(int mode, int kind, const Params& p, int grid, cudaStream_t stream);
+int mover_threads();
+size_t mover_smem_bytes(int kind);
+
+}  // namespace swk

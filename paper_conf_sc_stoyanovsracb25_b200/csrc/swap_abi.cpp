@@ -1,0 +1,542 @@
+// swap_abi.cpp — the extern "C" boundary of libswap (declared and documented in include/swap.h).
+//
+// Context state machine (include/swap.h; the paper's snapshot-once / restore-many model,
+// P:L115):
+//   CREATED --register--> REGISTERED --checkpoint--> CKPT_PENDING --sync--> CHECKPOINTED
+//   CHECKPOINTED|RESTORED --restore--> RESTORED;   REGISTERED|CHECKPOINTED|RESTORED --checkpoint--> CKPT_PENDING
+#include <sys/mman.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "kernels.cuh"
+#include "plan.h"
+
+namespace {
+
+enum class St { CREATED, REGISTERED, CKPT_PENDING, CHECKPOINTED, RESTORED };
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+}  // namespace
+
+struct swap_ctx {
+  swap_config_t cfg{};
+  St st = St::CREATED;
+  int sm_count = 0;
+  swp::Plan plan;
+  // host image: mmap'd, pinned + mapped with cudaHostRegister (library-owned)
+  uint8_t* image = nullptr;
+  size_t map_bytes = 0;
+  bool host_registered = false;
+  uint8_t* image_dev = nullptr;  // device (UVA) view of the image
+  // device-side work state
+  swk::SegDesc* d_desc = nullptr;
+  uint32_t n_desc = 0;
+  uint32_t* d_partial = nullptr;
+  uint32_t* d_arrive = nullptr;
+  swk::DevStatus* d_status = nullptr;
+  swk::DevStatus* h_status = nullptr;  // pinned
+  uint32_t* d_tables = nullptr;
+  uint32_t zinit_c = 0, xseg = 0;
+  // copy-engine lists (per chunk and per region)
+  std::vector<void*> ce_dev, ce_host;
+  std::vector<size_t> ce_bytes;
+  cudaEvent_t ev[6] = {};  // checkpoint, restore, verify: begin/end pairs
+  bool pending[3] = {false, false, false};
+  float ms[3] = {0.f, 0.f, 0.f};
+  uint64_t launches = 0;
+  std::string err;
+  std::vector<swap_shard_summary_t> global;
+};
+
+namespace {
+
+swap_status cuda_fail(swap_ctx* c, cudaError_t e, const char* what) {
+  c->err = std::string(what) + ": " + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ")";
+  return SWAP_ECUDA;
+}
+#define CUDA_TRY(ctx, expr)                                    \
+  do {                                                         \
+    cudaError_t e_ = (expr);                                   \
+    if (e_ != cudaSuccess) return cuda_fail((ctx), e_, #expr); \
+  } while (0)
+
+uint8_t* manifest_ptr(swap_ctx* c) { return c->image + c->plan.manifest_off; }
+
+swk::Params base_params(swap_ctx* c) {
+  swk::Params p{};
+  p.desc = c->d_desc;
+  p.n_desc = c->n_desc;
+  p.seg_bytes = c->cfg.seg_bytes;
+  p.partial = c->d_partial;
+  p.arrive = c->d_arrive;
+  const uint64_t cs_off = c->plan.manifest_off + swp::kHeaderBytes + swp::kRegionRecBytes * c->plan.regions.size() + 24;
+  p.cs_out = reinterpret_cast<uint64_t*>(c->image_dev + cs_off);
+  p.cs_exp = p.cs_out;
+  p.n_bad = &c->d_status->n_bad;
+  p.first_bad = &c->d_status->first_bad;
+  p.tables = c->d_tables;
+  p.chunk_bytes = c->plan.C;
+  p.zinit_c = c->zinit_c;
+  p.xseg = c->xseg;
+  return p;
+}
+
+int grid_of(swap_ctx* c) { return c->cfg.grid_ctas ? (int)c->cfg.grid_ctas : 2 * c->sm_count; }
+int kind_of(swap_ctx* c) {
+  if (c->cfg.mechanism == SWAP_MECH_SM_NOCHECK) return swk::KIND_NONE;
+  return c->plan.kind == SWAP_CHECKSUM_XXH64 ? swk::KIND_XXH64 : swk::KIND_CRC32C;
+}
+int hash_kind(swap_ctx* c) { return c->plan.kind == SWAP_CHECKSUM_XXH64 ? swk::KIND_XXH64 : swk::KIND_CRC32C; }
+
+swap_status launch(swap_ctx* c, int mode, int kind, const swk::Params& p, cudaStream_t s) {
+  if (p.n_desc == 0) return SWAP_OK;
+  cudaError_t e = swk::launch_mover(mode, kind, p, grid_of(c), s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "mover kernel launch");
+  ++c->launches;
+  return SWAP_OK;
+}
+
+// Copy-engine data movement for mechanisms CE_*: dir 0 = device -> image, 1 = image -> device.
+swap_status ce_copy(swap_ctx* c, int dir, cudaStream_t s) {
+  const auto kind = dir == 0 ? cudaMemcpyDeviceToHost : cudaMemcpyHostToDevice;
+  if (c->cfg.mechanism == SWAP_MECH_CE_REGION) {
+    for (const auto& r : c->plan.regions) {
+      if (!r.r.bytes) continue;
+      void* dev = reinterpret_cast<void*>(r.r.dev_addr);
+      void* host = c->image + r.off;
+      CUDA_TRY(c, dir == 0 ? cudaMemcpyAsync(host, dev, r.r.bytes, kind, s)
+                           : cudaMemcpyAsync(dev, host, r.r.bytes, kind, s));
+    }
+    return SWAP_OK;
+  }
+  if (c->cfg.mechanism == SWAP_MECH_CE_CHUNK) {
+    for (size_t i = 0; i < c->ce_bytes.size(); ++i)
+      CUDA_TRY(c, dir == 0 ? cudaMemcpyAsync(c->ce_host[i], c->ce_dev[i], c->ce_bytes[i], kind, s)
+                           : cudaMemcpyAsync(c->ce_dev[i], c->ce_host[i], c->ce_bytes[i], kind, s));
+    return SWAP_OK;
+  }
+  // CE_BATCH: one cudaMemcpyBatchAsync over every chunk.
+  if (s == nullptr) {
+    c->err = "SWAP_MECH_CE_BATCH needs a non-default stream (cudaMemcpyBatchAsync restriction)";
+    return SWAP_EUNSUPPORTED;
+  }
+  if (c->ce_bytes.empty()) return SWAP_OK;
+  cudaMemcpyAttributes attr;
+  std::memset(&attr, 0, sizeof(attr));
+  attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
+  attr.srcLocHint.type = dir == 0 ? cudaMemLocationTypeDevice : cudaMemLocationTypeHost;
+  attr.srcLocHint.id = dir == 0 ? c->cfg.device : 0;
+  attr.dstLocHint.type = dir == 0 ? cudaMemLocationTypeHost : cudaMemLocationTypeDevice;
+  attr.dstLocHint.id = dir == 0 ? 0 : c->cfg.device;
+  size_t attr_idx = 0, fail_idx = 0;
+  std::vector<void*>& dst = dir == 0 ? c->ce_host : c->ce_dev;
+  std::vector<void*>& src = dir == 0 ? c->ce_dev : c->ce_host;
+  CUDA_TRY(c, cudaMemcpyBatchAsync(dst.data(), src.data(), c->ce_bytes.data(), c->ce_bytes.size(), &attr, &attr_idx, 1,
+                                   &fail_idx, s));
+  return SWAP_OK;
+}
+
+// Phase p: 0 checkpoint, 1 restore, 2 verify. Call after the stream has been synchronised.
+swap_status collect_timing(swap_ctx* c, int p) {
+  if (!c->pending[p]) return SWAP_OK;
+  CUDA_TRY(c, cudaEventElapsedTime(&c->ms[p], c->ev[2 * p], c->ev[2 * p + 1]));
+  c->pending[p] = false;
+  return SWAP_OK;
+}
+
+bool is_ce(uint32_t m) { return m == SWAP_MECH_CE_REGION || m == SWAP_MECH_CE_CHUNK || m == SWAP_MECH_CE_BATCH; }
+
+void release(swap_ctx* c) {
+  if (c->d_desc) cudaFree(c->d_desc);
+  if (c->d_partial) cudaFree(c->d_partial);
+  if (c->d_arrive) cudaFree(c->d_arrive);
+  if (c->d_status) cudaFree(c->d_status);
+  if (c->h_status) cudaFreeHost(c->h_status);
+  if (c->d_tables) cudaFree(c->d_tables);
+  for (auto& e : c->ev)
+    if (e) cudaEventDestroy(e);
+  if (c->host_registered) cudaHostUnregister(c->image);
+  if (c->image) munmap(c->image, c->map_bytes);
+  c->d_desc = nullptr;
+  c->image = nullptr;
+}
+
+}  // namespace
+
+extern "C" {
+
+void swap_config_default(swap_config_t* cfg) {
+  if (!cfg) return;
+  std::memset(cfg, 0, sizeof(*cfg));
+  cfg->chunk_bytes = 1ull << 20;
+  cfg->align = 4096;
+  cfg->checksum = SWAP_CHECKSUM_CRC32C;
+  cfg->mechanism = SWAP_MECH_SM;
+  cfg->world = 1;
+  cfg->seg_bytes = 256u << 10;
+}
+
+swap_status swap_create(const swap_config_t* cfg_in, swap_ctx_t** out) {
+  if (!cfg_in || !out) return SWAP_EINVAL;
+  *out = nullptr;
+  auto* c = new (std::nothrow) swap_ctx();
+  if (!c) return SWAP_ENOMEM;
+  c->cfg = *cfg_in;
+  swap_status st = swp::normalize_config(&c->cfg, &c->err);
+  if (st != SWAP_OK) {
+    fprintf(stderr, "libswap: swap_create: %s\n", c->err.c_str());
+    delete c;
+    return st;
+  }
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || c->cfg.device >= ndev) {
+    fprintf(stderr, "libswap: swap_create: no CUDA device %d (%s)\n", c->cfg.device,
+            e != cudaSuccess ? cudaGetErrorString(e) : "ordinal out of range");
+    delete c;
+    return SWAP_ECUDA;
+  }
+  cudaDeviceProp prop;
+  if (cudaGetDeviceProperties(&prop, c->cfg.device) != cudaSuccess || prop.major != 10 || !prop.canMapHostMemory) {
+    fprintf(stderr, "libswap: swap_create: device %d is not an sm_100 GPU with mapped host memory\n",
+            c->cfg.device);
+    delete c;
+    return SWAP_ECUDA;
+  }
+  c->sm_count = prop.multiProcessorCount;
+  DeviceGuard g(c->cfg.device);
+  std::vector<uint32_t> tab(swk::TAB_WORDS);
+  swk::build_tables(tab.data());
+  if ((e = cudaMalloc(&c->d_tables, tab.size() * 4)) != cudaSuccess ||
+      (e = cudaMemcpy(c->d_tables, tab.data(), tab.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess ||
+      (e = cudaMalloc(&c->d_status, sizeof(swk::DevStatus))) != cudaSuccess ||
+      (e = cudaMemset(c->d_status, 0, sizeof(swk::DevStatus))) != cudaSuccess ||
+      (e = cudaHostAlloc(&c->h_status, sizeof(swk::DevStatus), cudaHostAllocDefault)) != cudaSuccess ||
+      (e = cudaEventCreate(&c->ev[0])) != cudaSuccess || (e = cudaEventCreate(&c->ev[1])) != cudaSuccess ||
+      (e = cudaEventCreate(&c->ev[2])) != cudaSuccess || (e = cudaEventCreate(&c->ev[3])) != cudaSuccess ||
+      (e = cudaEventCreate(&c->ev[4])) != cudaSuccess || (e = cudaEventCreate(&c->ev[5])) != cudaSuccess) {
+    cuda_fail(c, e, "swap_create");
+    fprintf(stderr, "libswap: %s\n", c->err.c_str());
+    release(c);
+    delete c;
+    return SWAP_ECUDA;
+  }
+  const uint32_t* x2n = tab.data() + swk::TAB_X2N;
+  c->zinit_c = swk::host_multmodp(swk::host_x2nmodp(c->cfg.chunk_bytes, 3, x2n), 0xFFFFFFFFu);
+  c->xseg = swk::host_x2nmodp(c->cfg.seg_bytes, 3, x2n);
+  *out = c;
+  return SWAP_OK;
+}
+
+swap_status swap_register_regions(swap_ctx_t* c, const swap_region_t* regions, size_t n) {
+  if (!c) return SWAP_EINVAL;
+  swp::Plan plan;
+  swap_status st = swp::build_plan(regions, n, c->cfg, &plan, &c->err);
+  if (st != SWAP_OK) return st;
+  if (c->st != St::CREATED) {
+    c->err = "regions already registered";
+    return SWAP_ESTATE;
+  }
+  DeviceGuard g(c->cfg.device);
+  c->plan = std::move(plan);
+  const swp::Plan& P = c->plan;
+
+  // Library-owned image: anonymous mapping (zero-filled, so padding is 0), huge pages when
+  // available, pinned and mapped into the device address space.
+  const size_t page = 2u << 20;
+  c->map_bytes = (P.image_bytes + page - 1) / page * page;
+  void* m = mmap(nullptr, c->map_bytes, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+  if (m == MAP_FAILED) {
+    c->err = "mmap of " + std::to_string(c->map_bytes) + " B failed";
+    c->map_bytes = 0;
+    return SWAP_ENOMEM;
+  }
+  c->image = static_cast<uint8_t*>(m);
+  madvise(m, c->map_bytes, MADV_HUGEPAGE);
+  cudaError_t e = cudaHostRegister(m, c->map_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    munmap(m, c->map_bytes);
+    c->image = nullptr;
+    c->map_bytes = 0;
+    c->err = std::string("cudaHostRegister (pinning the image) failed: ") + cudaGetErrorString(e);
+    return SWAP_ENOMEM;
+  }
+  c->host_registered = true;
+  void* dview = nullptr;
+  CUDA_TRY(c, cudaHostGetDevicePointer(&dview, m, 0));
+  c->image_dev = static_cast<uint8_t*>(dview);
+  swp::write_manifest_skeleton(P, manifest_ptr(c));
+
+  // Segment descriptors: CRC-32C chunks split at seg_bytes; XXH64 segments are whole chunks.
+  const uint64_t seg = P.kind == SWAP_CHECKSUM_XXH64 ? P.C : std::min<uint64_t>(P.C, c->cfg.seg_bytes);
+  std::vector<swk::SegDesc> desc;
+  c->ce_dev.clear();
+  c->ce_host.clear();
+  c->ce_bytes.clear();
+  for (const auto& r : P.regions) {
+    for (uint64_t j = 0; j < r.nchunks; ++j) {
+      const uint64_t lo = j * P.C, len = std::min<uint64_t>(P.C, r.r.bytes - lo);
+      const uint32_t nseg = (uint32_t)((len + seg - 1) / seg);
+      for (uint32_t s = 0; s < nseg; ++s) {
+        swk::SegDesc d;
+        d.dev = r.r.dev_addr + lo + s * seg;
+        d.host = reinterpret_cast<uint64_t>(c->image_dev + r.off + lo + s * seg);
+        d.bytes = (uint32_t)std::min<uint64_t>(seg, len - s * seg);
+        d.chunk = (uint32_t)(r.first + j);
+        d.seg = s;
+        d.nseg = nseg;
+        desc.push_back(d);
+      }
+      c->ce_dev.push_back(reinterpret_cast<void*>(r.r.dev_addr + lo));
+      c->ce_host.push_back(c->image + r.off + lo);
+      c->ce_bytes.push_back(len);
+    }
+  }
+  if (desc.size() > 0xFFFFFFFFull) {
+    c->err = "too many segments";
+    return SWAP_EUNSUPPORTED;
+  }
+  c->n_desc = (uint32_t)desc.size();
+  const size_t nd = std::max<size_t>(1, desc.size());
+  CUDA_TRY(c, cudaMalloc(&c->d_desc, nd * sizeof(swk::SegDesc)));
+  if (!desc.empty())
+    CUDA_TRY(c, cudaMemcpy(c->d_desc, desc.data(), desc.size() * sizeof(swk::SegDesc), cudaMemcpyHostToDevice));
+  CUDA_TRY(c, cudaMalloc(&c->d_partial, nd * 4));
+  CUDA_TRY(c, cudaMalloc(&c->d_arrive, std::max<uint64_t>(1, P.n_chunks) * 4));
+  CUDA_TRY(c, cudaMemset(c->d_arrive, 0, std::max<uint64_t>(1, P.n_chunks) * 4));
+  c->st = St::REGISTERED;
+  return SWAP_OK;
+}
+
+swap_status swap_checkpoint(swap_ctx_t* c, swap_stream_t stream) {
+  if (!c) return SWAP_EINVAL;
+  if (c->st == St::CREATED || c->st == St::CKPT_PENDING) {
+    c->err = c->st == St::CREATED ? "checkpoint before swap_register_regions" : "previous checkpoint not synced";
+    return SWAP_ESTATE;
+  }
+  DeviceGuard g(c->cfg.device);
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  swk::Params p = base_params(c);
+  CUDA_TRY(c, cudaEventRecord(c->ev[0], s));
+  swap_status st;
+  if (is_ce(c->cfg.mechanism)) {
+    if ((st = launch(c, swk::HASH_STORE, hash_kind(c), p, s)) != SWAP_OK) return st;
+    if ((st = ce_copy(c, 0, s)) != SWAP_OK) return st;
+  } else {
+    if ((st = launch(c, swk::GATHER, kind_of(c), p, s)) != SWAP_OK) return st;
+  }
+  CUDA_TRY(c, cudaEventRecord(c->ev[1], s));
+  c->pending[0] = true;
+  c->st = St::CKPT_PENDING;
+  return SWAP_OK;
+}
+
+swap_status swap_sync(swap_ctx_t* c, swap_stream_t stream) {
+  if (!c) return SWAP_EINVAL;
+  DeviceGuard g(c->cfg.device);
+  CUDA_TRY(c, cudaStreamSynchronize(reinterpret_cast<cudaStream_t>(stream)));
+  if (c->pending[0]) {
+    CUDA_TRY(c, cudaEventSynchronize(c->ev[1]));
+    swap_status ts = collect_timing(c, 0);
+    if (ts != SWAP_OK) return ts;
+  }
+  if (c->st == St::CKPT_PENDING) {
+    swp::seal_manifest(c->plan, manifest_ptr(c));
+    c->st = St::CHECKPOINTED;
+  }
+  return SWAP_OK;
+}
+
+swap_status swap_restore(swap_ctx_t* c, swap_stream_t stream) {
+  if (!c) return SWAP_EINVAL;
+  if (c->st != St::CHECKPOINTED && c->st != St::RESTORED) {
+    c->err = "restore needs a completed checkpoint (swap_sync) or an imported image";
+    return SWAP_ESTATE;
+  }
+  swap_status st = swp::check_manifest(c->plan, manifest_ptr(c), &c->err);
+  if (st != SWAP_OK) return st;
+  DeviceGuard g(c->cfg.device);
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  swk::Params p = base_params(c);
+  CUDA_TRY(c, cudaMemsetAsync(&c->d_status->n_bad, 0, 8, s));
+  CUDA_TRY(c, cudaMemsetAsync(&c->d_status->first_bad, 0xFF, 8, s));
+  CUDA_TRY(c, cudaEventRecord(c->ev[2], s));
+  if (is_ce(c->cfg.mechanism)) {
+    if ((st = ce_copy(c, 1, s)) != SWAP_OK) return st;
+    if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, s)) != SWAP_OK) return st;
+  } else {
+    if ((st = launch(c, swk::SCATTER, kind_of(c), p, s)) != SWAP_OK) return st;
+  }
+  CUDA_TRY(c, cudaEventRecord(c->ev[3], s));
+  c->pending[1] = true;
+  c->st = St::RESTORED;
+  return SWAP_OK;
+}
+
+swap_status swap_verify(swap_ctx_t* c, swap_stream_t stream, int hbm_pass, swap_verify_result_t* res) {
+  if (!c || !res) return SWAP_EINVAL;
+  if (c->st != St::RESTORED) {
+    c->err = "verify needs a restore";
+    return SWAP_ESTATE;
+  }
+  DeviceGuard g(c->cfg.device);
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  if (hbm_pass) {
+    swk::Params p = base_params(c);
+    p.n_bad = &c->d_status->hbm_n_bad;
+    p.first_bad = &c->d_status->hbm_first_bad;
+    CUDA_TRY(c, cudaMemsetAsync(&c->d_status->hbm_n_bad, 0, 8, s));
+    CUDA_TRY(c, cudaMemsetAsync(&c->d_status->hbm_first_bad, 0xFF, 8, s));
+    CUDA_TRY(c, cudaEventRecord(c->ev[4], s));
+    swap_status st = launch(c, swk::HASH_CHECK, hash_kind(c), p, s);
+    if (st != SWAP_OK) return st;
+    CUDA_TRY(c, cudaEventRecord(c->ev[5], s));
+    c->pending[2] = true;
+  }
+  CUDA_TRY(c, cudaMemcpyAsync(c->h_status, c->d_status, sizeof(swk::DevStatus), cudaMemcpyDeviceToHost, s));
+  CUDA_TRY(c, cudaStreamSynchronize(s));
+  for (int ph = 1; ph < 3; ++ph) {
+    swap_status ts = collect_timing(c, ph);
+    if (ts != SWAP_OK) return ts;
+  }
+  res->n_bad = c->h_status->n_bad;
+  res->first_bad_chunk = c->h_status->first_bad;
+  res->hbm_checked = hbm_pass ? 1u : 0u;
+  res->hbm_n_bad = hbm_pass ? c->h_status->hbm_n_bad : 0;
+  res->hbm_first_bad = hbm_pass ? c->h_status->hbm_first_bad : UINT64_MAX;
+  res->manifest_ok = swp::manifest_crc_ok(c->plan, manifest_ptr(c)) ? 1u : 0u;
+  if (res->n_bad || res->hbm_n_bad || !res->manifest_ok) {
+    c->err = "verification failed: " + std::to_string(res->n_bad) + " bad chunk(s) in restore, " +
+             std::to_string(res->hbm_n_bad) + " in HBM pass, manifest_ok=" + std::to_string(res->manifest_ok);
+    return SWAP_ECORRUPT;
+  }
+  return SWAP_OK;
+}
+
+swap_status swap_set_mechanism(swap_ctx_t* c, uint32_t mechanism) {
+  if (!c || mechanism > SWAP_MECH_SM_NOCHECK) return SWAP_EINVAL;
+  c->cfg.mechanism = mechanism;
+  return SWAP_OK;
+}
+
+swap_status swap_get_manifest(const swap_ctx_t* c, const void** bytes, size_t* n) {
+  if (!c || !bytes || !n) return SWAP_EINVAL;
+  if (!c->image) return SWAP_ESTATE;
+  *bytes = c->image + c->plan.manifest_off;
+  *n = c->plan.manifest_bytes;
+  return SWAP_OK;
+}
+
+swap_status swap_get_image(const swap_ctx_t* c, void** host, size_t* n) {
+  if (!c || !host || !n) return SWAP_EINVAL;
+  if (!c->image) return SWAP_ESTATE;
+  *host = c->image;
+  *n = c->plan.image_bytes;
+  return SWAP_OK;
+}
+
+swap_status swap_get_summary(const swap_ctx_t* c, swap_shard_summary_t* out) {
+  if (!c || !out) return SWAP_EINVAL;
+  if (c->st != St::CHECKPOINTED && c->st != St::RESTORED) return SWAP_ESTATE;
+  swp::make_summary(c->plan, c->image + c->plan.manifest_off, out);
+  return SWAP_OK;
+}
+
+swap_status swap_import(swap_ctx_t* c) {
+  if (!c) return SWAP_EINVAL;
+  if (c->st == St::CREATED || c->st == St::CKPT_PENDING) return SWAP_ESTATE;
+  swap_status st = swp::check_manifest(c->plan, manifest_ptr(c), &c->err);
+  if (st != SWAP_OK) return st;
+  c->st = St::CHECKPOINTED;
+  return SWAP_OK;
+}
+
+swap_status swap_merge_global(const swap_shard_summary_t* all, int world, uint64_t* digest) {
+  if (!all || world < 1) return SWAP_EINVAL;
+  for (int r = 0; r < world; ++r)
+    if ((int)all[r].rank != r || (int)all[r].world != world || all[r].reserved != 0) return SWAP_ENCCL;
+  if (digest) *digest = swp::crc32c_host(all, sizeof(swap_shard_summary_t) * (size_t)world);
+  return SWAP_OK;
+}
+
+swap_status swap_set_global(swap_ctx_t* c, const swap_shard_summary_t* all, int world, uint64_t* digest) {
+  if (!c || !all || world < 1) return SWAP_EINVAL;
+  if (c->st != St::CHECKPOINTED && c->st != St::RESTORED) return SWAP_ESTATE;
+  if (world != c->cfg.world) {
+    c->err = "world mismatch in global manifest";
+    return SWAP_ENCCL;
+  }
+  if (swap_merge_global(all, world, nullptr) != SWAP_OK) {
+    c->err = "global manifest entries are not rank-ordered summaries of this world";
+    return SWAP_ENCCL;
+  }
+  swap_shard_summary_t mine;
+  swp::make_summary(c->plan, c->image + c->plan.manifest_off, &mine);
+  if (std::memcmp(&mine, &all[c->cfg.rank], sizeof(mine)) != 0) {
+    c->err = "own entry of the global manifest differs from the local summary";
+    return SWAP_ENCCL;
+  }
+  c->global.assign(all, all + world);
+  if (digest) *digest = swp::crc32c_host(all, sizeof(swap_shard_summary_t) * (size_t)world);
+  return SWAP_OK;
+}
+
+swap_status swap_get_timings(const swap_ctx_t* c, swap_timings_t* out) {
+  if (!c || !out) return SWAP_EINVAL;
+  out->checkpoint_ms = c->ms[0];
+  out->restore_ms = c->ms[1];
+  out->verify_ms = c->ms[2];
+  out->reserved = 0.f;
+  return SWAP_OK;
+}
+
+swap_status swap_get_launch_count(const swap_ctx_t* c, uint64_t* n) {
+  if (!c || !n) return SWAP_EINVAL;
+  *n = c->launches;
+  return SWAP_OK;
+}
+
+const char* swap_status_str(swap_status s) {
+  switch (s) {
+    case SWAP_OK: return "SWAP_OK";
+    case SWAP_EINVAL: return "SWAP_EINVAL";
+    case SWAP_ENOMEM: return "SWAP_ENOMEM";
+    case SWAP_ECUDA: return "SWAP_ECUDA";
+    case SWAP_ESTATE: return "SWAP_ESTATE";
+    case SWAP_ECORRUPT: return "SWAP_ECORRUPT";
+    case SWAP_ENCCL: return "SWAP_ENCCL";
+    case SWAP_EUNSUPPORTED: return "SWAP_EUNSUPPORTED";
+    case SWAP_EINTERNAL: return "SWAP_EINTERNAL";
+    default: return "SWAP_UNKNOWN";
+  }
+}
+
+const char* swap_last_error(const swap_ctx_t* c) { return c ? c->err.c_str() : "null ctx"; }
+
+void swap_destroy(swap_ctx_t* c) {
+  if (!c) return;
+  {
+    DeviceGuard g(c->cfg.device);
+    release(c);
+  }
+  delete c;
+}
+
+}  // extern "C"

@@ -1,0 +1,59 @@
+"""Multi-GPU shard coordinator (§6 "Multi-GPU Orchestration").
+
+A tensor-parallel engine's device memory is already per rank: rank r checkpoints and
+restores its own shard on its own device and stream with no data-path collective. The
+only exchanges are
+  K5  all-gather of the 64-B shard summaries -> one rank-ordered global manifest + digest,
+  K6  all-reduce(SUM) of the mismatch counts after restore/verify, so every rank agrees
+      the engine is whole before serving resumes ("verifies that the inference
+      engine API is active").
+Both go through torch.distributed (NCCL over NVLink on the GPU box; gloo in CPU tests).
+Validation and the digest run in libswap (swap_set_global / swap_merge_global).
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+from .swap import SWAP_OK, SwapError, Swapper, swap_merge_global
+
+
+def _comm_device(group=None) -> torch.device:
+    backend = dist.get_backend(group)
+    if backend == "nccl":
+        return torch.device("cuda", torch.cuda.current_device())
+    return torch.device("cpu")
+
+
+def all_gather_summaries(summary: bytes, group=None) -> bytes:
+    """K5: every rank contributes its 64-B summary; returns the world*64 bytes in rank order."""
+    assert len(summary) == 64
+    world = dist.get_world_size(group)
+    dev = _comm_device(group)
+    mine = torch.frombuffer(bytearray(summary), dtype=torch.uint8).to(dev)
+    out = torch.empty(world * 64, dtype=torch.uint8, device=dev)
+    dist.all_gather_into_tensor(out, mine, group=group)
+    return out.cpu().numpy().tobytes()
+
+
+def merge_global(summaries: bytes) -> int:
+    """Validates rank order and returns the global digest (libswap swap_merge_global)."""
+    st, digest = swap_merge_global(summaries, len(summaries) // 64)
+    if st != SWAP_OK:
+        raise SwapError(st, "global manifest is not a rank-ordered set of summaries")
+    return digest
+
+
+def gather_manifest(sw: Swapper, group=None) -> tuple[bytes, int]:
+    """After a checkpoint on every rank: all-gather summaries, install them in the ctx."""
+    allb = all_gather_summaries(sw.summary(), group)
+    return allb, sw.set_global(allb)
+
+
+def agree_restore(verify_result: dict, group=None) -> int:
+    """K6: global number of bad chunks (fused restore check + HBM pass) over all ranks."""
+    dev = _comm_device(group)
+    t = torch.tensor([verify_result["n_bad"] + verify_result["hbm_n_bad"] + (0 if verify_result["manifest_ok"] else 1)],
+                     dtype=torch.int64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+    return int(t.item())

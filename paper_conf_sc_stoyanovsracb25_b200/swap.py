@@ -1,0 +1,306 @@
+"""ctypes binding of libswap (include/swap.h) — argument marshalling only.
+
+Every step of the checkpoint/restore path runs in libswap's CUDA kernels or copy-engine
+calls; this module only converts Python values to the C ABI and back. There is no CPU
+fallback: if libswap.so is missing or no sm_100 GPU is present, calls fail loudly.
+
+The low-level functions keep the C names (``swap_create``, ``swap_register_regions``,
+``swap_checkpoint``, ``swap_restore``, ``swap_verify``, ...) and return the raw status;
+``Swapper`` is the convenience wrapper tests and bench.py use (it raises ``SwapError``).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+from . import build as _build
+
+SWAP_OK, SWAP_EINVAL, SWAP_ENOMEM, SWAP_ECUDA, SWAP_ESTATE = 0, -1, -2, -3, -4
+SWAP_ECORRUPT, SWAP_ENCCL, SWAP_EUNSUPPORTED, SWAP_EINTERNAL = -5, -6, -7, -8
+SWAP_CHECKSUM_CRC32C, SWAP_CHECKSUM_XXH64 = 1, 2
+SWAP_MECH_SM, SWAP_MECH_CE_REGION, SWAP_MECH_CE_CHUNK, SWAP_MECH_CE_BATCH, SWAP_MECH_SM_NOCHECK = 0, 1, 2, 3, 4
+MECHANISMS = {"sm": 0, "ce_region": 1, "ce_chunk": 2, "ce_batch": 3, "sm_nocheck": 4}
+SWAP_KIND_WEIGHTS, SWAP_KIND_KV, SWAP_KIND_WORKSPACE, SWAP_KIND_OTHER = 0, 1, 2, 3
+U64_MAX = (1 << 64) - 1
+
+EXPORTS = [
+    "swap_config_default", "swap_create", "swap_register_regions", "swap_checkpoint", "swap_sync",
+    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_manifest", "swap_get_image",
+    "swap_get_summary", "swap_import", "swap_set_global", "swap_merge_global", "swap_get_timings",
+    "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
+]
+
+
+class swap_region_t(ctypes.Structure):
+    _fields_ = [("dev_addr", ctypes.c_uint64), ("bytes", ctypes.c_uint64), ("id", ctypes.c_uint32),
+                ("kind", ctypes.c_uint32)]
+
+
+class swap_config_t(ctypes.Structure):
+    _fields_ = [("chunk_bytes", ctypes.c_uint64), ("align", ctypes.c_uint64), ("checksum", ctypes.c_uint32),
+                ("mechanism", ctypes.c_uint32), ("device", ctypes.c_int32), ("rank", ctypes.c_int32),
+                ("world", ctypes.c_int32), ("grid_ctas", ctypes.c_uint32), ("seg_bytes", ctypes.c_uint32),
+                ("reserved", ctypes.c_uint32)]
+
+
+class swap_verify_result_t(ctypes.Structure):
+    _fields_ = [("n_bad", ctypes.c_uint64), ("first_bad_chunk", ctypes.c_uint64), ("hbm_n_bad", ctypes.c_uint64),
+                ("hbm_first_bad", ctypes.c_uint64), ("manifest_ok", ctypes.c_uint32),
+                ("hbm_checked", ctypes.c_uint32)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class swap_shard_summary_t(ctypes.Structure):
+    _fields_ = [("rank", ctypes.c_uint32), ("world", ctypes.c_uint32), ("checksum", ctypes.c_uint32),
+                ("n_regions", ctypes.c_uint32), ("n_chunks", ctypes.c_uint64), ("payload_bytes", ctypes.c_uint64),
+                ("image_bytes", ctypes.c_uint64), ("manifest_crc", ctypes.c_uint64),
+                ("chunk_digest", ctypes.c_uint64), ("reserved", ctypes.c_uint64)]
+
+
+class swap_timings_t(ctypes.Structure):
+    _fields_ = [("checkpoint_ms", ctypes.c_float), ("restore_ms", ctypes.c_float), ("verify_ms", ctypes.c_float),
+                ("reserved", ctypes.c_float)]
+
+
+assert ctypes.sizeof(swap_shard_summary_t) == 64 and ctypes.sizeof(swap_config_t) == 48
+
+_lib = None
+
+
+def lib_path() -> str:
+    return _build.LIB
+
+
+def load(build_if_missing: bool = True) -> ctypes.CDLL:
+    """Loads the in-tree libswap.so (building it with nvcc if absent). Raises if unavailable."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not _build.up_to_date():
+        if not build_if_missing:
+            raise RuntimeError(f"libswap.so missing or stale at {_build.LIB}; run paper_conf_sc_stoyanovsracb25_b200.build")
+        _build.build()
+    L = ctypes.CDLL(_build.LIB)
+    vp, st, u32, sz = ctypes.c_void_p, ctypes.c_int32, ctypes.c_uint32, ctypes.c_size_t
+    P = ctypes.POINTER
+    sig = {
+        "swap_config_default": (None, [P(swap_config_t)]),
+        "swap_create": (st, [P(swap_config_t), P(vp)]),
+        "swap_register_regions": (st, [vp, P(swap_region_t), sz]),
+        "swap_checkpoint": (st, [vp, vp]),
+        "swap_sync": (st, [vp, vp]),
+        "swap_restore": (st, [vp, vp]),
+        "swap_verify": (st, [vp, vp, ctypes.c_int, P(swap_verify_result_t)]),
+        "swap_set_mechanism": (st, [vp, u32]),
+        "swap_get_manifest": (st, [vp, P(vp), P(sz)]),
+        "swap_get_image": (st, [vp, P(vp), P(sz)]),
+        "swap_get_summary": (st, [vp, P(swap_shard_summary_t)]),
+        "swap_import": (st, [vp]),
+        "swap_set_global": (st, [vp, P(swap_shard_summary_t), ctypes.c_int, P(ctypes.c_uint64)]),
+        "swap_merge_global": (st, [P(swap_shard_summary_t), ctypes.c_int, P(ctypes.c_uint64)]),
+        "swap_get_timings": (st, [vp, P(swap_timings_t)]),
+        "swap_get_launch_count": (st, [vp, P(ctypes.c_uint64)]),
+        "swap_status_str": (ctypes.c_char_p, [st]),
+        "swap_last_error": (ctypes.c_char_p, [vp]),
+        "swap_destroy": (None, [vp]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(L, name)
+        f.restype, f.argtypes = res, args
+    _lib = L
+    return L
+
+
+class SwapError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        self.status = status
+        super().__init__(f"{load().swap_status_str(status).decode()} ({status}): {msg}")
+
+
+# ------------------------------------------------------------------ thin C-named wrappers
+def swap_config_default() -> swap_config_t:
+    cfg = swap_config_t()
+    load().swap_config_default(ctypes.byref(cfg))
+    return cfg
+
+
+def swap_create(cfg: swap_config_t):
+    h = ctypes.c_void_p()
+    st = load().swap_create(ctypes.byref(cfg), ctypes.byref(h))
+    return st, h
+
+
+def swap_register_regions(ctx, regions) -> int:
+    """regions: sequence of (dev_addr, nbytes, id, kind)."""
+    arr = (swap_region_t * max(1, len(regions)))()
+    for i, (addr, nb, rid, kind) in enumerate(regions):
+        arr[i].dev_addr, arr[i].bytes, arr[i].id, arr[i].kind = addr, nb, rid, kind
+    return load().swap_register_regions(ctx, arr, len(regions))
+
+
+def swap_checkpoint(ctx, stream: int = 0) -> int:
+    return load().swap_checkpoint(ctx, ctypes.c_void_p(stream))
+
+
+def swap_sync(ctx, stream: int = 0) -> int:
+    return load().swap_sync(ctx, ctypes.c_void_p(stream))
+
+
+def swap_restore(ctx, stream: int = 0) -> int:
+    return load().swap_restore(ctx, ctypes.c_void_p(stream))
+
+
+def swap_verify(ctx, stream: int = 0, hbm_pass: bool = True):
+    res = swap_verify_result_t()
+    st = load().swap_verify(ctx, ctypes.c_void_p(stream), 1 if hbm_pass else 0, ctypes.byref(res))
+    return st, res
+
+
+def swap_merge_global(summaries: bytes, world: int):
+    arr = (swap_shard_summary_t * world).from_buffer_copy(summaries)
+    d = ctypes.c_uint64()
+    st = load().swap_merge_global(arr, world, ctypes.byref(d))
+    return st, d.value
+
+
+def _torch_stream(stream) -> int:
+    if stream is None:
+        import torch
+
+        return torch.cuda.current_stream().cuda_stream
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+# ------------------------------------------------------------------ Swapper
+class Swapper:
+    """One registered engine shard on one device.
+
+    regions: sequence of torch CUDA tensors (whole storages are registered), or of
+    (dev_addr, nbytes, kind) / (dev_addr, nbytes, kind, id) tuples.
+    """
+
+    def __init__(self, regions, chunk_bytes: int = 1 << 20, checksum: int = SWAP_CHECKSUM_CRC32C,
+                 mechanism: int | str = SWAP_MECH_SM, device: int | None = None, rank: int = 0, world: int = 1,
+                 align: int = 4096, grid_ctas: int = 0, seg_bytes: int = 0):
+        L = load()
+        table = []
+        for i, r in enumerate(regions):
+            if hasattr(r, "data_ptr"):
+                if device is None:
+                    device = r.device.index
+                table.append((r.untyped_storage().data_ptr(), r.untyped_storage().nbytes(), i, SWAP_KIND_OTHER))
+            else:
+                addr, nb, kind = r[0], r[1], r[2]
+                table.append((addr, nb, r[3] if len(r) > 3 else i, kind))
+        if isinstance(mechanism, str):
+            mechanism = MECHANISMS[mechanism]
+        cfg = swap_config_default()
+        cfg.chunk_bytes, cfg.checksum, cfg.mechanism, cfg.align = chunk_bytes, checksum, mechanism, align
+        cfg.device, cfg.rank, cfg.world = device or 0, rank, world
+        cfg.grid_ctas, cfg.seg_bytes = grid_ctas, seg_bytes
+        st, h = swap_create(cfg)
+        if st:
+            raise SwapError(st, "swap_create failed (no sm_100 GPU / bad config)")
+        self._ctx = h
+        self.device = cfg.device
+        self.rank, self.world = rank, world
+        st = swap_register_regions(h, table)
+        if st:
+            msg = L.swap_last_error(h).decode()
+            self.close()
+            raise SwapError(st, msg)
+        self.regions = table
+
+    # -- helpers
+    def _check(self, st: int):
+        if st:
+            raise SwapError(st, load().swap_last_error(self._ctx).decode())
+
+    @property
+    def ctx(self):
+        return self._ctx
+
+    def checkpoint(self, stream=None, sync: bool = True):
+        s = _torch_stream(stream)
+        self._check(swap_checkpoint(self._ctx, s))
+        if sync:
+            self._check(swap_sync(self._ctx, s))
+
+    def sync(self, stream=None):
+        self._check(swap_sync(self._ctx, _torch_stream(stream)))
+
+    def restore(self, stream=None):
+        self._check(swap_restore(self._ctx, _torch_stream(stream)))
+
+    def verify(self, stream=None, hbm_pass: bool = True, raise_on_corrupt: bool = True) -> dict:
+        st, res = swap_verify(self._ctx, _torch_stream(stream), hbm_pass)
+        if st and (raise_on_corrupt or st != SWAP_ECORRUPT):
+            self._check(st)
+        d = res.as_dict()
+        d["status"] = st
+        return d
+
+    def set_mechanism(self, mechanism: int | str):
+        if isinstance(mechanism, str):
+            mechanism = MECHANISMS[mechanism]
+        self._check(load().swap_set_mechanism(self._ctx, mechanism))
+
+    def import_image(self):
+        self._check(load().swap_import(self._ctx))
+
+    def image(self) -> np.ndarray:
+        """Borrowed, writable uint8 view of the library's pinned image (valid until close)."""
+        p, n = ctypes.c_void_p(), ctypes.c_size_t()
+        self._check(load().swap_get_image(self._ctx, ctypes.byref(p), ctypes.byref(n)))
+        return np.ctypeslib.as_array(ctypes.cast(p, ctypes.POINTER(ctypes.c_uint8)), shape=(n.value,))
+
+    def manifest(self) -> np.ndarray:
+        p, n = ctypes.c_void_p(), ctypes.c_size_t()
+        self._check(load().swap_get_manifest(self._ctx, ctypes.byref(p), ctypes.byref(n)))
+        return np.ctypeslib.as_array(ctypes.cast(p, ctypes.POINTER(ctypes.c_uint8)), shape=(n.value,))
+
+    def summary(self) -> bytes:
+        s = swap_shard_summary_t()
+        self._check(load().swap_get_summary(self._ctx, ctypes.byref(s)))
+        return bytes(s)
+
+    def set_global(self, summaries: bytes) -> int:
+        world = len(summaries) // 64
+        arr = (swap_shard_summary_t * world).from_buffer_copy(summaries)
+        d = ctypes.c_uint64()
+        self._check(load().swap_set_global(self._ctx, arr, world, ctypes.byref(d)))
+        return d.value
+
+    def timings(self) -> dict:
+        """Device ms of the last checkpoint / restore / HBM verify movers (CUDA events)."""
+        t = swap_timings_t()
+        self._check(load().swap_get_timings(self._ctx, ctypes.byref(t)))
+        return {"checkpoint_ms": t.checkpoint_ms, "restore_ms": t.restore_ms, "verify_ms": t.verify_ms}
+
+    def launch_count(self) -> int:
+        n = ctypes.c_uint64()
+        self._check(load().swap_get_launch_count(self._ctx, ctypes.byref(n)))
+        return n.value
+
+    def close(self):
+        if getattr(self, "_ctx", None):
+            load().swap_destroy(self._ctx)
+            self._ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
