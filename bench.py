@@ -33,6 +33,7 @@ sys.path.insert(0, ROOT)
 import workloads as W  # noqa: E402
 
 GB = 1e9
+METRIC = "swap-in (restore + HBM verify) throughput, whole job"
 PCIE_GEN5_X16_GBPS = 63.015  # 64 GB/s x 128/130 (nominal, per direction)
 MEASURED_PEAKS = os.path.join(ROOT, "MEASURED_PEAKS.json")
 
@@ -44,7 +45,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="auto", choices=["auto", "A", "B", "C", "D"])
-    ap.add_argument("--mechanism", default="sm", choices=["sm", "ce_region", "ce_chunk", "ce_batch", "sm_nocheck"])
+    ap.add_argument("--mechanism", default="auto",
+                    choices=["auto", "sm", "ce_region", "ce_chunk", "ce_batch", "ce_pipe", "sm_nocheck"])
     ap.add_argument("--checksum", default="crc32c", choices=["crc32c", "xxh64"])
     ap.add_argument("--chunk", type=int, default=1 << 20)
     ap.add_argument("--grid", type=int, default=0)
@@ -160,11 +162,14 @@ def run_reference(args):
     timed = rates[args.warmup:]
     v = statistics.mean(timed)
     line = {
-        "impl": "reference", "metric": "swap-in (restore + verify) throughput, whole job", "value": round(v, 3),
+        "impl": "reference", "metric": METRIC, "value": round(v, 3),
         "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(payload / (v * GB) * 1e3, 3), "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-        "config": {"workload": f"{name}: {desc}", "sample": f"first {len(sample)} regions, {payload} B"},
+        "config": {"workload": f"{name}: {desc}", "regions_per_rank": len(specs),
+                   "payload_bytes_per_rank": sum(r.nbytes for r in specs), "chunk_bytes": 1 << 20,
+                   "checksum": "crc32c", "mechanism": "cpu oracle",
+                   "sample": f"each step restores the first {len(sample)} regions ({payload} B) on the host"},
         "cpu_baseline": {"value": round(v, 3), "unit": "GB/s", "cores": th, "kind": "oracle",
                          "sample": f"oracle_restore (memcpy + Sarwate CRC-32C per 1 MiB chunk) over the first "
                                    f"{len(sample)} regions of workload {name} ({payload} B), {th} OpenMP threads"},
@@ -286,7 +291,7 @@ def run_ours(args):
     # context: other movers on the same image (outside the timed region)
     compare = {}
     if not args.no_compare:
-        mechs = ["sm", "sm_nocheck", "ce_region", "ce_batch"]
+        mechs = ["sm", "sm_nocheck", "ce_region", "ce_batch", "ce_pipe"]
         for m in mechs:
             sw.set_mechanism(m)
             r2: dict = {}
@@ -335,7 +340,7 @@ def run_ours(args):
         peaks = json.load(open(MEASURED_PEAKS)) if os.path.exists(MEASURED_PEAKS) else {}
         hbm_peak = peaks.get("hbm_gbs", 6650.0)
         line = {
-            "metric": "swap-in (restore + HBM verify) throughput, whole job", "value": round(value, 3),
+            "metric": METRIC, "value": round(value, 3),
             "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": round(step_ms, 3), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "u8", "data": "synthetic",

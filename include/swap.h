@@ -58,14 +58,19 @@ typedef int32_t swap_status;
 #define SWAP_CHECKSUM_XXH64 2u  /* XXH64, seed 0 for every chunk */
 
 /* Data mover for checkpoint/restore (the image bytes are identical for all of them): */
-#define SWAP_MECH_SM 0u          /* one SM kernel: 16-B vector loads/stores to mapped pinned host
-                                    memory with the chunk checksum fused from the same registers */
-#define SWAP_MECH_CE_REGION 1u   /* copy engine: cudaMemcpyAsync per region + separate HBM hash pass */
-#define SWAP_MECH_CE_CHUNK 2u    /* copy engine: cudaMemcpyAsync per chunk + HBM hash pass */
-#define SWAP_MECH_CE_BATCH 3u    /* copy engine: one cudaMemcpyBatchAsync per call + HBM hash pass */
-#define SWAP_MECH_SM_NOCHECK 4u  /* diagnostic: the SM kernel with the checksum compiled out. Checkpoint
-                                    writes c_g = 0; restore reports no mismatches. Only for measuring
-                                    the fused-checksum overhead (BASELINE.json north_star: <= 5 %). */
+#define SWAP_MECH_AUTO 0u        /* default: SWAP_MECH_CE_PIPE when the payload is >= 512 MiB, else SWAP_MECH_SM */
+#define SWAP_MECH_SM 1u          /* one SM kernel: 16-B vector loads/stores to mapped pinned host memory with the
+                                    chunk checksum fused from the same registers (one pass, bytes checked in flight) */
+#define SWAP_MECH_CE_REGION 2u   /* copy engine: cudaMemcpyAsync per region + separate HBM hash pass */
+#define SWAP_MECH_CE_CHUNK 3u    /* copy engine: cudaMemcpyAsync per chunk + HBM hash pass */
+#define SWAP_MECH_CE_BATCH 4u    /* copy engine: one cudaMemcpyBatchAsync per call + HBM hash pass */
+#define SWAP_MECH_CE_PIPE 5u     /* copy engine moves the image in groups of ~pipe_mib MiB on the caller's stream
+                                    while the hash kernel checks (restore) / hashes (checkpoint) each group from
+                                    HBM on a second, library-owned stream; the caller's stream joins at the end */
+#define SWAP_MECH_SM_NOCHECK 6u  /* diagnostic: the SM kernel with the checksum compiled out. Checkpoint leaves
+                                    c_g unspecified; restore reports no mismatches. Only for measuring the
+                                    fused-checksum overhead (BASELINE.json north_star: <= 5 %). */
+#define SWAP_MECH_COUNT 7u
 
 /* Region kinds (manifest only; movement is kind-agnostic) */
 #define SWAP_KIND_WEIGHTS 0u
@@ -87,13 +92,13 @@ typedef struct {
   uint64_t chunk_bytes; /* checksum granule C: power of 2, >= 16, <= 2^31; 0 -> 1 MiB */
   uint64_t align;       /* image offset alignment A: power of 2, >= 16; 0 -> 4096 */
   uint32_t checksum;    /* SWAP_CHECKSUM_*; 0 -> CRC32C */
-  uint32_t mechanism;   /* SWAP_MECH_*; default SWAP_MECH_SM */
+  uint32_t mechanism;   /* SWAP_MECH_*; default SWAP_MECH_AUTO */
   int32_t device;       /* CUDA device ordinal the regions live on */
   int32_t rank;         /* 0 <= rank < world (tensor-parallel shard index) */
   int32_t world;        /* >= 1 */
   uint32_t grid_ctas;   /* SM mover grid; 0 -> auto (2 CTAs per SM) */
   uint32_t seg_bytes;   /* CRC32C work split inside a chunk: power of 2, >= 4096; 0 -> 256 KiB */
-  uint32_t reserved;    /* must be 0 */
+  uint32_t pipe_mib;    /* SWAP_MECH_CE_PIPE group size in MiB (rounded to whole chunks); 0 -> 256 */
 } swap_config_t;
 
 typedef struct {

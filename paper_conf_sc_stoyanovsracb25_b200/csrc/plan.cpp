@@ -74,7 +74,8 @@ swap_status normalize_config(swap_config_t* c, std::string* err) {
     *err = "checksum must be SWAP_CHECKSUM_CRC32C or SWAP_CHECKSUM_XXH64";
     return SWAP_EINVAL;
   }
-  if (c->mechanism > SWAP_MECH_SM_NOCHECK) {
+  if (c->pipe_mib == 0) c->pipe_mib = 256;
+  if (c->mechanism >= SWAP_MECH_COUNT) {
     *err = "unknown mechanism";
     return SWAP_EINVAL;
   }
@@ -82,8 +83,8 @@ swap_status normalize_config(swap_config_t* c, std::string* err) {
     *err = "need world >= 1, 0 <= rank < world, device >= 0";
     return SWAP_EINVAL;
   }
-  if (!pow2_ge(c->seg_bytes, 4096) || c->reserved != 0) {
-    *err = "seg_bytes must be a power of 2 >= 4096; reserved must be 0";
+  if (!pow2_ge(c->seg_bytes, 4096)) {
+    *err = "seg_bytes must be a power of 2 >= 4096";
     return SWAP_EINVAL;
   }
   if (c->chunk_bytes > (1ull << 31)) {

@@ -34,6 +34,16 @@ struct DeviceGuard {
 
 }  // namespace
 
+struct Span {  // one copy-engine transfer: contiguous on the device and in the image
+  uint64_t dev;
+  uint8_t* host;
+  uint64_t bytes;
+};
+struct Group {  // CE_PIPE unit: whole chunks, descriptor range [d0, d1)
+  uint32_t d0, d1;
+  std::vector<Span> spans;
+};
+
 struct swap_ctx {
   swap_config_t cfg{};
   St st = St::CREATED;
@@ -62,6 +72,11 @@ struct swap_ctx {
   uint64_t launches = 0;
   std::string err;
   std::vector<swap_shard_summary_t> global;
+  // CE_PIPE
+  std::vector<Group> groups;
+  std::vector<cudaEvent_t> group_ev;
+  cudaStream_t side = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };
 
 namespace {
@@ -98,37 +113,54 @@ swk::Params base_params(swap_ctx* c) {
 }
 
 int grid_of(swap_ctx* c) { return c->cfg.grid_ctas ? (int)c->cfg.grid_ctas : 2 * c->sm_count; }
+
+// The mechanism actually used: AUTO picks the copy-engine pipeline for large images (the copy
+// engines reach a higher link rate than SM-issued accesses) and the single fused
+// SM pass for small ones (no per-copy launch overhead).
+constexpr uint64_t kAutoPipeBytes = 512ull << 20;
+uint32_t mech(const swap_ctx* c) {
+  if (c->cfg.mechanism != SWAP_MECH_AUTO) return c->cfg.mechanism;
+  return c->plan.payload_bytes >= kAutoPipeBytes ? SWAP_MECH_CE_PIPE : SWAP_MECH_SM;
+}
 int kind_of(swap_ctx* c) {
-  if (c->cfg.mechanism == SWAP_MECH_SM_NOCHECK) return swk::KIND_NONE;
+  if (mech(c) == SWAP_MECH_SM_NOCHECK) return swk::KIND_NONE;
   return c->plan.kind == SWAP_CHECKSUM_XXH64 ? swk::KIND_XXH64 : swk::KIND_CRC32C;
 }
 int hash_kind(swap_ctx* c) { return c->plan.kind == SWAP_CHECKSUM_XXH64 ? swk::KIND_XXH64 : swk::KIND_CRC32C; }
 
 swap_status launch(swap_ctx* c, int mode, int kind, const swk::Params& p, cudaStream_t s) {
   if (p.n_desc == 0) return SWAP_OK;
-  cudaError_t e = swk::launch_mover(mode, kind, p, grid_of(c), s);
+  // never more CTAs than descriptor batches (idle CTAs would only load tables)
+  const int want = (int)std::min<uint64_t>((uint64_t)grid_of(c), (p.n_desc + 15) / 16);
+  cudaError_t e = swk::launch_mover(mode, kind, p, std::max(1, want), s);
   if (e != cudaSuccess) return cuda_fail(c, e, "mover kernel launch");
   ++c->launches;
   return SWAP_OK;
 }
 
-// Copy-engine data movement for mechanisms CE_*: dir 0 = device -> image, 1 = image -> device.
+swap_status memcpy_dir(swap_ctx* c, const Span& sp, int dir, cudaStream_t s) {
+  void* dev = reinterpret_cast<void*>(sp.dev);
+  CUDA_TRY(c, dir == 0 ? cudaMemcpyAsync(sp.host, dev, sp.bytes, cudaMemcpyDeviceToHost, s)
+                       : cudaMemcpyAsync(dev, sp.host, sp.bytes, cudaMemcpyHostToDevice, s));
+  return SWAP_OK;
+}
+
+// Copy-engine data movement for CE_REGION / CE_CHUNK / CE_BATCH: dir 0 = device -> image, 1 = image -> device.
 swap_status ce_copy(swap_ctx* c, int dir, cudaStream_t s) {
-  const auto kind = dir == 0 ? cudaMemcpyDeviceToHost : cudaMemcpyHostToDevice;
-  if (c->cfg.mechanism == SWAP_MECH_CE_REGION) {
+  const uint32_t m = mech(c);
+  if (m == SWAP_MECH_CE_REGION) {
     for (const auto& r : c->plan.regions) {
       if (!r.r.bytes) continue;
-      void* dev = reinterpret_cast<void*>(r.r.dev_addr);
-      void* host = c->image + r.off;
-      CUDA_TRY(c, dir == 0 ? cudaMemcpyAsync(host, dev, r.r.bytes, kind, s)
-                           : cudaMemcpyAsync(dev, host, r.r.bytes, kind, s));
+      swap_status st = memcpy_dir(c, Span{r.r.dev_addr, c->image + r.off, r.r.bytes}, dir, s);
+      if (st != SWAP_OK) return st;
     }
     return SWAP_OK;
   }
-  if (c->cfg.mechanism == SWAP_MECH_CE_CHUNK) {
-    for (size_t i = 0; i < c->ce_bytes.size(); ++i)
-      CUDA_TRY(c, dir == 0 ? cudaMemcpyAsync(c->ce_host[i], c->ce_dev[i], c->ce_bytes[i], kind, s)
-                           : cudaMemcpyAsync(c->ce_dev[i], c->ce_host[i], c->ce_bytes[i], kind, s));
+  if (m == SWAP_MECH_CE_CHUNK) {
+    for (size_t i = 0; i < c->ce_bytes.size(); ++i) {
+      swap_status st = memcpy_dir(c, Span{(uint64_t)c->ce_dev[i], (uint8_t*)c->ce_host[i], c->ce_bytes[i]}, dir, s);
+      if (st != SWAP_OK) return st;
+    }
     return SWAP_OK;
   }
   // CE_BATCH: one cudaMemcpyBatchAsync over every chunk.
@@ -152,6 +184,33 @@ swap_status ce_copy(swap_ctx* c, int dir, cudaStream_t s) {
   return SWAP_OK;
 }
 
+// CE_PIPE. Checkpoint (dir 0): the hash pass over HBM runs on the side stream concurrently with the
+// D2H copies (both only read HBM). Restore (dir 1): group g's H2D copies are followed by an event;
+// the side stream waits for it and checks group g from HBM while the copy engine moves group g+1.
+swap_status ce_pipe(swap_ctx* c, int dir, const swk::Params& base, cudaStream_t s) {
+  CUDA_TRY(c, cudaEventRecord(c->ev_fork, s));
+  CUDA_TRY(c, cudaStreamWaitEvent(c->side, c->ev_fork, 0));
+  swap_status st;
+  if (dir == 0 && (st = launch(c, swk::HASH_STORE, hash_kind(c), base, c->side)) != SWAP_OK) return st;
+  for (size_t g = 0; g < c->groups.size(); ++g) {
+    const Group& G = c->groups[g];
+    for (const Span& sp : G.spans)
+      if ((st = memcpy_dir(c, sp, dir, s)) != SWAP_OK) return st;
+    if (dir == 1) {
+      CUDA_TRY(c, cudaEventRecord(c->group_ev[g], s));
+      CUDA_TRY(c, cudaStreamWaitEvent(c->side, c->group_ev[g], 0));
+      swk::Params p = base;
+      p.desc = base.desc + G.d0;
+      p.partial = base.partial + G.d0;
+      p.n_desc = G.d1 - G.d0;
+      if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, c->side)) != SWAP_OK) return st;
+    }
+  }
+  CUDA_TRY(c, cudaEventRecord(c->ev_join, c->side));
+  CUDA_TRY(c, cudaStreamWaitEvent(s, c->ev_join, 0));
+  return SWAP_OK;
+}
+
 // Phase p: 0 checkpoint, 1 restore, 2 verify. Call after the stream has been synchronised.
 swap_status collect_timing(swap_ctx* c, int p) {
   if (!c->pending[p]) return SWAP_OK;
@@ -171,6 +230,12 @@ void release(swap_ctx* c) {
   if (c->d_tables) cudaFree(c->d_tables);
   for (auto& e : c->ev)
     if (e) cudaEventDestroy(e);
+  for (auto& e : c->group_ev)
+    if (e) cudaEventDestroy(e);
+  c->group_ev.clear();
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_join) cudaEventDestroy(c->ev_join);
+  if (c->side) cudaStreamDestroy(c->side);
   if (c->host_registered) cudaHostUnregister(c->image);
   if (c->image) munmap(c->image, c->map_bytes);
   c->d_desc = nullptr;
@@ -187,9 +252,10 @@ void swap_config_default(swap_config_t* cfg) {
   cfg->chunk_bytes = 1ull << 20;
   cfg->align = 4096;
   cfg->checksum = SWAP_CHECKSUM_CRC32C;
-  cfg->mechanism = SWAP_MECH_SM;
+  cfg->mechanism = SWAP_MECH_AUTO;
   cfg->world = 1;
   cfg->seg_bytes = 256u << 10;
+  cfg->pipe_mib = 256;
 }
 
 swap_status swap_create(const swap_config_t* cfg_in, swap_ctx_t** out) {
@@ -309,6 +375,38 @@ swap_status swap_register_regions(swap_ctx_t* c, const swap_region_t* regions, s
       c->ce_bytes.push_back(len);
     }
   }
+  // CE_PIPE groups: consecutive whole chunks up to ~pipe_mib MiB; spans merge chunks of one region.
+  {
+    const uint64_t target = (uint64_t)c->cfg.pipe_mib << 20;
+    Group cur{0, 0, {}};
+    uint64_t cur_bytes = 0;
+    size_t di = 0;
+    for (const auto& r : P.regions) {
+      for (uint64_t j = 0; j < r.nchunks; ++j) {
+        const uint64_t lo = j * P.C, len = std::min<uint64_t>(P.C, r.r.bytes - lo);
+        Span sp{r.r.dev_addr + lo, c->image + r.off + lo, len};
+        if (!cur.spans.empty() && cur.spans.back().dev + cur.spans.back().bytes == sp.dev &&
+            cur.spans.back().host + cur.spans.back().bytes == sp.host)
+          cur.spans.back().bytes += len;
+        else
+          cur.spans.push_back(sp);
+        while (di < desc.size() && desc[di].chunk == r.first + j) ++di;
+        cur.d1 = (uint32_t)di;
+        cur_bytes += len;
+        if (cur_bytes >= target) {
+          c->groups.push_back(std::move(cur));
+          cur = Group{(uint32_t)di, (uint32_t)di, {}};
+          cur_bytes = 0;
+        }
+      }
+    }
+    if (!cur.spans.empty()) c->groups.push_back(std::move(cur));
+    c->group_ev.assign(c->groups.size(), nullptr);
+    for (auto& e : c->group_ev) CUDA_TRY(c, cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+    CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
+    CUDA_TRY(c, cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
+  }
   if (desc.size() > 0xFFFFFFFFull) {
     c->err = "too many segments";
     return SWAP_EUNSUPPORTED;
@@ -336,7 +434,9 @@ swap_status swap_checkpoint(swap_ctx_t* c, swap_stream_t stream) {
   swk::Params p = base_params(c);
   CUDA_TRY(c, cudaEventRecord(c->ev[0], s));
   swap_status st;
-  if (is_ce(c->cfg.mechanism)) {
+  if (mech(c) == SWAP_MECH_CE_PIPE) {
+    if ((st = ce_pipe(c, 0, p, s)) != SWAP_OK) return st;
+  } else if (is_ce(mech(c))) {
     if ((st = launch(c, swk::HASH_STORE, hash_kind(c), p, s)) != SWAP_OK) return st;
     if ((st = ce_copy(c, 0, s)) != SWAP_OK) return st;
   } else {
@@ -378,7 +478,9 @@ swap_status swap_restore(swap_ctx_t* c, swap_stream_t stream) {
   CUDA_TRY(c, cudaMemsetAsync(&c->d_status->n_bad, 0, 8, s));
   CUDA_TRY(c, cudaMemsetAsync(&c->d_status->first_bad, 0xFF, 8, s));
   CUDA_TRY(c, cudaEventRecord(c->ev[2], s));
-  if (is_ce(c->cfg.mechanism)) {
+  if (mech(c) == SWAP_MECH_CE_PIPE) {
+    if ((st = ce_pipe(c, 1, p, s)) != SWAP_OK) return st;
+  } else if (is_ce(mech(c))) {
     if ((st = ce_copy(c, 1, s)) != SWAP_OK) return st;
     if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, s)) != SWAP_OK) return st;
   } else {
@@ -431,7 +533,7 @@ swap_status swap_verify(swap_ctx_t* c, swap_stream_t stream, int hbm_pass, swap_
 }
 
 swap_status swap_set_mechanism(swap_ctx_t* c, uint32_t mechanism) {
-  if (!c || mechanism > SWAP_MECH_SM_NOCHECK) return SWAP_EINVAL;
+  if (!c || mechanism >= SWAP_MECH_COUNT) return SWAP_EINVAL;
   c->cfg.mechanism = mechanism;
   return SWAP_OK;
 }

@@ -20,8 +20,9 @@ from . import build as _build
 SWAP_OK, SWAP_EINVAL, SWAP_ENOMEM, SWAP_ECUDA, SWAP_ESTATE = 0, -1, -2, -3, -4
 SWAP_ECORRUPT, SWAP_ENCCL, SWAP_EUNSUPPORTED, SWAP_EINTERNAL = -5, -6, -7, -8
 SWAP_CHECKSUM_CRC32C, SWAP_CHECKSUM_XXH64 = 1, 2
-SWAP_MECH_SM, SWAP_MECH_CE_REGION, SWAP_MECH_CE_CHUNK, SWAP_MECH_CE_BATCH, SWAP_MECH_SM_NOCHECK = 0, 1, 2, 3, 4
-MECHANISMS = {"sm": 0, "ce_region": 1, "ce_chunk": 2, "ce_batch": 3, "sm_nocheck": 4}
+SWAP_MECH_AUTO, SWAP_MECH_SM, SWAP_MECH_CE_REGION, SWAP_MECH_CE_CHUNK = 0, 1, 2, 3
+SWAP_MECH_CE_BATCH, SWAP_MECH_CE_PIPE, SWAP_MECH_SM_NOCHECK = 4, 5, 6
+MECHANISMS = {"auto": 0, "sm": 1, "ce_region": 2, "ce_chunk": 3, "ce_batch": 4, "ce_pipe": 5, "sm_nocheck": 6}
 SWAP_KIND_WEIGHTS, SWAP_KIND_KV, SWAP_KIND_WORKSPACE, SWAP_KIND_OTHER = 0, 1, 2, 3
 U64_MAX = (1 << 64) - 1
 
@@ -42,7 +43,7 @@ class swap_config_t(ctypes.Structure):
     _fields_ = [("chunk_bytes", ctypes.c_uint64), ("align", ctypes.c_uint64), ("checksum", ctypes.c_uint32),
                 ("mechanism", ctypes.c_uint32), ("device", ctypes.c_int32), ("rank", ctypes.c_int32),
                 ("world", ctypes.c_int32), ("grid_ctas", ctypes.c_uint32), ("seg_bytes", ctypes.c_uint32),
-                ("reserved", ctypes.c_uint32)]
+                ("pipe_mib", ctypes.c_uint32)]
 
 
 class swap_verify_result_t(ctypes.Structure):
@@ -186,8 +187,8 @@ class Swapper:
     """
 
     def __init__(self, regions, chunk_bytes: int = 1 << 20, checksum: int = SWAP_CHECKSUM_CRC32C,
-                 mechanism: int | str = SWAP_MECH_SM, device: int | None = None, rank: int = 0, world: int = 1,
-                 align: int = 4096, grid_ctas: int = 0, seg_bytes: int = 0):
+                 mechanism: int | str = SWAP_MECH_AUTO, device: int | None = None, rank: int = 0, world: int = 1,
+                 align: int = 4096, grid_ctas: int = 0, seg_bytes: int = 0, pipe_mib: int = 0):
         L = load()
         table = []
         for i, r in enumerate(regions):
@@ -203,7 +204,7 @@ class Swapper:
         cfg = swap_config_default()
         cfg.chunk_bytes, cfg.checksum, cfg.mechanism, cfg.align = chunk_bytes, checksum, mechanism, align
         cfg.device, cfg.rank, cfg.world = device or 0, rank, world
-        cfg.grid_ctas, cfg.seg_bytes = grid_ctas, seg_bytes
+        cfg.grid_ctas, cfg.seg_bytes, cfg.pipe_mib = grid_ctas, seg_bytes, pipe_mib
         st, h = swap_create(cfg)
         if st:
             raise SwapError(st, "swap_create failed (no sm_100 GPU / bad config)")

@@ -14,7 +14,7 @@ from gpu_util import chunk_records, device_case, poison
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
 
-MECHS = ["sm", "ce_region", "ce_chunk", "ce_batch"]
+MECHS = ["sm", "ce_region", "ce_chunk", "ce_batch", "ce_pipe", "auto"]
 U64_MAX = (1 << 64) - 1
 
 
@@ -102,6 +102,14 @@ def test_launch_shapes(swp, orc, stream, grid, seg):
     """Odd grids (rounds with partial descriptor batches) and segment splits of a chunk."""
     specs = W.config_a(4)
     roundtrip(swp, orc, stream, specs, 4, 1 << 20, 1, "sm", key=("A", 4, 1 << 20, 1), grid_ctas=grid, seg_bytes=seg)
+
+
+@pytest.mark.parametrize("pipe_mib", [1, 3, 16])
+@pytest.mark.parametrize("kind", [1, 2], ids=["crc32c", "xxh64"])
+def test_ce_pipe_groups(swp, orc, stream, pipe_mib, kind):
+    """CE_PIPE with many groups: group boundaries cut regions; hash launches see descriptor offsets."""
+    roundtrip(swp, orc, stream, W.config_a(2), 2, 1 << 16, kind, "ce_pipe", key=("A", 2, 1 << 16, kind),
+              pipe_mib=pipe_mib, seg_bytes=16384)
 
 
 @pytest.mark.parametrize("name", list(W.edge_tables(4096)))
