@@ -16,6 +16,7 @@
 //    the GF(2) shift crc(A||B) = Z^|B|(crc(A)) ^ crc(B).
 //  * XXH64 (non-combinable): one warp per chunk; stripe words are routed to 4 accumulator
 //    lanes with shuffles, the tail and finalisation run on lane 0.
+#include <algorithm>
 #include <cstdio>
 
 #include "kernels.cuh"
@@ -56,7 +57,7 @@ uint32_t host_x2nmodp(uint64_t n, unsigned k, const uint32_t* x2n) {  // x^(n*2^
   return p;
 }
 
-void build_tables(uint32_t* tab) {
+void build_tables(uint32_t* tab, uint64_t L1) {
   uint32_t* t = tab + TAB_T16;
   for (uint32_t b = 0; b < 256; ++b) t[b] = step_byte(b);  // T_0 = one byte
   for (int k = 1; k < 16; ++k)
@@ -74,6 +75,12 @@ void build_tables(uint32_t* tab) {
   x2n[0] = 1u << 30;  // x^1
   for (int k = 1; k < 32; ++k) x2n[k] = host_multmodp(x2n[k - 1], x2n[k - 1]);
   for (int l = 0; l < 32; ++l) tab[TAB_LANE + l] = host_x2nmodp(16ull * (31 - l), 3, x2n);
+  // hash kernel: lane l hashes [l*q, min((l+1)*q, L1)); its register is shifted by the bytes after it.
+  const uint64_t q = hash_lane_run(L1);
+  for (int l = 0; l < 32; ++l) {
+    const uint64_t end = std::min<uint64_t>((uint64_t)(l + 1) * q, L1);
+    tab[TAB_HLANE + l] = (uint64_t)l * q < L1 ? host_x2nmodp(L1 - end, 3, x2n) : 0u;
+  }
 }
 
 // ------------------------------------------------------------------ device helpers
@@ -413,6 +420,305 @@ __global__ void __launch_bounds__(THREADS, 2) mover_kernel(const Params p) {
   }
 }
 
+
+// ------------------------------------------------------------------ HBM hash kernel (CRC-32C)
+// HASH_STORE / HASH_CHECK read device memory only, so lanes need not own 512-B-coalesced slices:
+// lane l hashes the contiguous run [l*q, min((l+1)*q, len)) of its warp's segment with 256-bit
+// loads (one 32-B sector per lane per load) and slicing-by-4 tables replicated once per lane in
+// shared memory (entry (k, e) of lane l at word ((k*256 + e) * 32 + l): bank = lane, conflict-free).
+// The 32 lane registers are folded with x^(8 * bytes-after-run) and an XOR shuffle tree.
+constexpr int HT_THREADS = 1024;
+constexpr int HT_WARPS = HT_THREADS / 32;
+constexpr int HT_U = 4;  // 32-B loads in flight per lane
+constexpr size_t HT_TAB_WORDS = 4 * 256 * 32;
+constexpr size_t HT_OFF_DESC = HT_TAB_WORDS * 4;
+constexpr size_t HT_OFF_BAR = HT_OFF_DESC + 2 * HT_WARPS * sizeof(SegDesc);
+constexpr size_t HT_SMEM = HT_OFF_BAR + 16;
+
+__device__ __forceinline__ void ld32(const uint8_t* p, uint32_t (&w)[8]) {
+  asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7])
+               : "l"(p));
+}
+__device__ __forceinline__ void ld32_v4x2(const uint8_t* p, uint32_t (&w)[8]) {  // 16-B aligned fallback
+  int4 a = __ldg(reinterpret_cast<const int4*>(p)), b = __ldg(reinterpret_cast<const int4*>(p + 16));
+  w[0] = a.x; w[1] = a.y; w[2] = a.z; w[3] = a.w; w[4] = b.x; w[5] = b.y; w[6] = b.z; w[7] = b.w;
+}
+
+// slicing-by-4 word step on the lane's replicated tables (sT already offset by the lane)
+__device__ __forceinline__ uint32_t crc_word4(uint32_t c, uint32_t w, const uint32_t* __restrict__ sT) {
+  c ^= w;
+  return sT[(3 * 256 + (c & 0xFF)) * 32] ^ sT[(2 * 256 + ((c >> 8) & 0xFF)) * 32] ^
+         sT[(1 * 256 + ((c >> 16) & 0xFF)) * 32] ^ sT[(0 * 256 + (c >> 24)) * 32];
+}
+
+template <bool AL32>
+__device__ __forceinline__ void ld32a(const uint8_t* p, uint32_t (&w)[8]) {
+  if (AL32) ld32(p, w); else ld32_v4x2(p, w);
+}
+
+// CRC register of one lane's contiguous run [lo, hi) (hi - lo < 2^32), from 0.
+template <bool AL32>
+__device__ __forceinline__ uint32_t lane_run_crc(const uint8_t* src, uint64_t lo, uint64_t hi, const uint32_t* myT) {
+  uint32_t c = 0;
+  uint64_t o = lo;
+  const uint64_t full_end = lo + (hi - lo) / 32 * 32;
+  for (; o + 32 * HT_U <= full_end; o += 32 * HT_U) {
+    uint32_t w[HT_U][8];
+#pragma unroll
+    for (int u = 0; u < HT_U; ++u) ld32a<AL32>(src + o + 32 * u, w[u]);
+#pragma unroll
+    for (int u = 0; u < HT_U; ++u)
+#pragma unroll
+      for (int j = 0; j < 8; ++j) c = crc_word4(c, w[u][j], myT);
+  }
+  for (; o < full_end; o += 32) {
+    uint32_t w[8];
+    ld32a<AL32>(src + o, w);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) c = crc_word4(c, w[j], myT);
+  }
+  for (; o < hi; ++o) c = myT[((c ^ src[o]) & 0xFFu) * 32] ^ (c >> 8);  // ragged tail, T0 = one byte
+  return c;
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  uint32_t* sT = reinterpret_cast<uint32_t*>(smem);
+  SegDesc* sDesc = reinterpret_cast<SegDesc*>(smem + HT_OFF_DESC);
+  uint64_t* sBar = reinterpret_cast<uint64_t*>(smem + HT_OFF_BAR);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+
+  // replicate T0..T3 (the first four slicing tables) once per lane
+  for (int i = tid; i < 4 * 256; i += HT_THREADS) {
+    const uint32_t v = __ldg(p.tables + TAB_T16 + i);
+    uint4* dst = reinterpret_cast<uint4*>(sT + (size_t)i * 32);
+#pragma unroll
+    for (int r = 0; r < 8; ++r) dst[r] = make_uint4(v, v, v, v);
+  }
+  const uint32_t per_round = gridDim.x * HT_WARPS;
+  const uint32_t first0 = blockIdx.x * HT_WARPS;
+  const uint32_t rounds = p.n_desc > first0 ? (p.n_desc - first0 + per_round - 1) / per_round : 0u;
+  auto issue = [&](uint32_t r) {
+    const uint32_t first = r * per_round + first0;
+    const uint32_t cnt = min((uint32_t)HT_WARPS, p.n_desc - first);
+    uint64_t* bar = sBar + (r & 1);
+    mbar_expect_tx(bar, cnt * (uint32_t)sizeof(SegDesc));
+    bulk_g2s(sDesc + (r & 1) * HT_WARPS, p.desc + first, cnt * (uint32_t)sizeof(SegDesc), bar);
+  };
+  if (tid == 0) {
+    mbar_init(sBar, 1);
+    mbar_init(sBar + 1, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    if (rounds > 0) issue(0);
+    if (rounds > 1) issue(1);
+  }
+  __syncthreads();
+  const uint32_t* myT = sT + lane;
+  const uint32_t* x2n = p.tables + TAB_X2N;
+
+  for (uint32_t r = 0; r < rounds; ++r) {
+    mbar_wait(sBar + (r & 1), (r >> 1) & 1u);
+    const uint32_t idx = r * per_round + first0 + warp;
+    if (idx < p.n_desc) {
+      const SegDesc d = sDesc[(r & 1) * HT_WARPS + warp];
+      const uint64_t len = d.bytes;
+      const uint64_t q = hash_lane_run(len);
+      const uint64_t lo = (uint64_t)lane * q;
+      const uint64_t hi = lo + q < len ? lo + q : len;
+      const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
+      const bool al32 = ((d.dev & 31) == 0);
+      uint32_t c = 0;
+      if (lo < hi) c = al32 ? lane_run_crc<true>(src, lo, hi, myT) : lane_run_crc<false>(src, lo, hi, myT);
+      // fold: X = XOR_l Z^(len - hi_l)(c_l)
+      uint32_t X = 0;
+      if (lo < hi) {
+        const uint32_t k = (len == p.hlane_len) ? __ldg(p.tables + TAB_HLANE + lane) : x2nmodp(len - hi, 3, x2n);
+        X = multmodp(k, c);
+      }
+#pragma unroll
+      for (int s = 16; s > 0; s >>= 1) X ^= __shfl_xor_sync(0xffffffffu, X, s);
+      if (lane == 0) {
+        if (d.nseg == 1) {
+          const uint32_t zi = (len == p.chunk_bytes) ? p.zinit_c : crc_shift(0xFFFFFFFFu, len, x2n);
+          chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ X)));
+        } else {
+          p.partial[idx] = X;
+          __threadfence();
+          const uint32_t prev = atomicAdd(p.arrive + d.chunk, 1u);
+          if (prev == d.nseg - 1) {
+            __threadfence();
+            const uint32_t first = idx - d.seg;
+            const uint32_t last_len = __ldcg(&p.desc[first + d.nseg - 1].bytes);
+            uint32_t acc = 0;
+            for (uint32_t s = 0; s < d.nseg; ++s) {
+              const uint32_t f = __ldcg(p.partial + first + s);
+              if (s == 0) acc = f;
+              else if (s + 1 < d.nseg || last_len == p.seg_bytes) acc = multmodp(p.xseg, acc) ^ f;
+              else acc = crc_shift(acc, last_len, x2n) ^ f;
+            }
+            p.arrive[d.chunk] = 0;
+            const uint64_t L = (uint64_t)(d.nseg - 1) * p.seg_bytes + last_len;
+            const uint32_t zi = (L == p.chunk_bytes) ? p.zinit_c : crc_shift(0xFFFFFFFFu, L, x2n);
+            chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ acc)));
+          }
+        }
+      }
+    }
+    __syncthreads();
+    if (tid == 0 && r + 2 < rounds) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      issue(r + 2);
+    }
+  }
+}
+
+template <int MODE>
+static cudaError_t launch_hash(const Params& p, int grid, cudaStream_t s) {
+  static unsigned long long attr_set = 0;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (!((attr_set >> (dev & 63)) & 1ull)) {
+    e = cudaFuncSetAttribute(hash_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)HT_SMEM);
+    if (e != cudaSuccess) return e;
+    attr_set |= 1ull << (dev & 63);
+  }
+  hash_kernel<MODE><<<grid, HT_THREADS, HT_SMEM, s>>>(p);
+  return cudaGetLastError();
+}
+
+int hash_grid(int sm_count, uint32_t n_desc) {
+  const uint32_t batches = (n_desc + HT_WARPS - 1) / HT_WARPS;
+  return (int)std::max<uint32_t>(1, std::min<uint32_t>((uint32_t)sm_count, batches));
+}
+
+
+// ------------------------------------------------------------------ HBM hash kernel (XXH64)
+// XXH64 consumes a chunk's 32-B stripes strictly in order, so parallelism comes from chunks:
+// one LANE per chunk, its four accumulators in registers, one 256-bit load per stripe (a full
+// sector), XK_U stripes in flight. Used for HASH_STORE / HASH_CHECK when there are enough chunks
+// to occupy the GPU (hash_xxh_lane_ok); otherwise the warp-per-chunk mover handles it.
+constexpr int XK_THREADS = 256;
+constexpr int XK_U = 4;
+constexpr size_t XK_OFF_BAR = 2 * XK_THREADS * sizeof(SegDesc);
+constexpr size_t XK_SMEM = XK_OFF_BAR + 16;
+
+__device__ __forceinline__ uint64_t w64(const uint32_t (&w)[8], int i) {
+  return (uint64_t)w[2 * i] | ((uint64_t)w[2 * i + 1] << 32);
+}
+
+template <bool AL32>
+__device__ __forceinline__ void xxh_stripes(const uint8_t* src, uint64_t end, uint64_t (&v)[4]) {
+  uint64_t o = 0;
+  for (; o + 32 * XK_U <= end; o += 32 * XK_U) {
+    uint32_t w[XK_U][8];
+#pragma unroll
+    for (int u = 0; u < XK_U; ++u) ld32a<AL32>(src + o + 32 * u, w[u]);
+#pragma unroll
+    for (int u = 0; u < XK_U; ++u)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) v[i] = xround(v[i], w64(w[u], i));
+  }
+  for (; o < end; o += 32) {
+    uint32_t w[8];
+    ld32a<AL32>(src + o, w);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) v[i] = xround(v[i], w64(w, i));
+  }
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(XK_THREADS) xxh_lane_kernel(const Params p) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  SegDesc* sDesc = reinterpret_cast<SegDesc*>(smem);
+  uint64_t* sBar = reinterpret_cast<uint64_t*>(smem + XK_OFF_BAR);
+  const int tid = threadIdx.x;
+  const uint32_t per_round = gridDim.x * XK_THREADS;
+  const uint32_t first0 = blockIdx.x * XK_THREADS;
+  const uint32_t rounds = p.n_desc > first0 ? (p.n_desc - first0 + per_round - 1) / per_round : 0u;
+  auto issue = [&](uint32_t r) {
+    const uint32_t first = r * per_round + first0;
+    const uint32_t cnt = min((uint32_t)XK_THREADS, p.n_desc - first);
+    uint64_t* bar = sBar + (r & 1);
+    mbar_expect_tx(bar, cnt * (uint32_t)sizeof(SegDesc));
+    bulk_g2s(sDesc + (r & 1) * XK_THREADS, p.desc + first, cnt * (uint32_t)sizeof(SegDesc), bar);
+  };
+  if (tid == 0) {
+    mbar_init(sBar, 1);
+    mbar_init(sBar + 1, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    if (rounds > 0) issue(0);
+    if (rounds > 1) issue(1);
+  }
+  __syncthreads();
+  for (uint32_t r = 0; r < rounds; ++r) {
+    mbar_wait(sBar + (r & 1), (r >> 1) & 1u);
+    const uint32_t idx = r * per_round + first0 + tid;
+    if (idx < p.n_desc) {
+      const SegDesc d = sDesc[(r & 1) * XK_THREADS + tid];
+      const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
+      const uint64_t len = d.bytes;
+      const bool al32 = ((d.dev & 31) == 0);
+      uint64_t v[4] = {P1 + P2, P2, 0, 0ull - P1};
+      const uint64_t stripes_end = len / 32 * 32;
+      if (al32) xxh_stripes<true>(src, stripes_end, v); else xxh_stripes<false>(src, stripes_end, v);
+      const uint64_t v1 = v[0], v2 = v[1], v3 = v[2], v4 = v[3];
+      uint64_t o = stripes_end;
+      uint64_t h;
+      if (len >= 32) {
+        h = rotl64(v1, 1) + rotl64(v2, 7) + rotl64(v3, 12) + rotl64(v4, 18);
+        h = xmerge(h, v1);
+        h = xmerge(h, v2);
+        h = xmerge(h, v3);
+        h = xmerge(h, v4);
+      } else {
+        h = P5;
+      }
+      h += len;
+      for (; o + 8 <= len; o += 8) {
+        h ^= xround(0, ld_u64_smem(src + o));  // bytewise little-endian read (tail is unaligned)
+        h = rotl64(h, 27) * P1 + P4;
+      }
+      if (o + 4 <= len) {
+        const uint32_t w = (uint32_t)src[o] | ((uint32_t)src[o + 1] << 8) | ((uint32_t)src[o + 2] << 16) |
+                           ((uint32_t)src[o + 3] << 24);
+        h ^= (uint64_t)w * P1;
+        h = rotl64(h, 23) * P2 + P3;
+        o += 4;
+      }
+      for (; o < len; ++o) {
+        h ^= (uint64_t)src[o] * P5;
+        h = rotl64(h, 11) * P1;
+      }
+      h ^= h >> 33;
+      h *= P2;
+      h ^= h >> 29;
+      h *= P3;
+      h ^= h >> 32;
+      chunk_result<MODE>(p, d.chunk, h);
+    }
+    __syncthreads();
+    if (tid == 0 && r + 2 < rounds) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      issue(r + 2);
+    }
+  }
+}
+
+template <int MODE>
+static cudaError_t launch_xxh_lane(const Params& p, int sm_count, cudaStream_t s) {
+  const uint32_t blocks = (p.n_desc + XK_THREADS - 1) / XK_THREADS;
+  const int grid = (int)std::max<uint32_t>(1, std::min<uint32_t>(blocks, (uint32_t)sm_count * 4));
+  xxh_lane_kernel<MODE><<<grid, XK_THREADS, XK_SMEM, s>>>(p);
+  return cudaGetLastError();
+}
+
+bool hash_xxh_lane_ok(int sm_count, uint32_t n_desc) { return n_desc >= (uint32_t)sm_count * 192u; }
+
 int mover_threads() { return THREADS; }
 size_t mover_smem_bytes(int kind) {
   return kind == KIND_CRC32C ? SmemLayout<KIND_CRC32C>::bytes : SmemLayout<KIND_NONE>::bytes;
@@ -434,6 +740,11 @@ static cudaError_t launch_t(const Params& p, int grid, cudaStream_t s) {
   return cudaGetLastError();
 }
 
+cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_t s) {
+  if (p.n_desc == 0) return cudaSuccess;
+  return mode == HASH_STORE ? launch_xxh_lane<HASH_STORE>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK>(p, sm_count, s);
+}
+
 cudaError_t launch_mover(int mode, int kind, const Params& p, int grid, cudaStream_t s) {
   if (p.n_desc == 0) return cudaSuccess;
 #define SWK_CASE(M, K) \
@@ -444,10 +755,10 @@ cudaError_t launch_mover(int mode, int kind, const Params& p, int grid, cudaStre
   SWK_CASE(SCATTER, KIND_NONE)
   SWK_CASE(SCATTER, KIND_CRC32C)
   SWK_CASE(SCATTER, KIND_XXH64)
-  SWK_CASE(HASH_STORE, KIND_CRC32C)
   SWK_CASE(HASH_STORE, KIND_XXH64)
-  SWK_CASE(HASH_CHECK, KIND_CRC32C)
   SWK_CASE(HASH_CHECK, KIND_XXH64)
+  if (mode == HASH_STORE && kind == KIND_CRC32C) return launch_hash<HASH_STORE>(p, grid, s);
+  if (mode == HASH_CHECK && kind == KIND_CRC32C) return launch_hash<HASH_CHECK>(p, grid, s);
 #undef SWK_CASE
   return cudaErrorInvalidValue;
 }

@@ -39,7 +39,8 @@ constexpr int TAB_T16 = 0;          // [16][256] slicing-by-16: T_k[b] = F(0, b 
 constexpr int TAB_Z496 = 16 * 256;  // [4][256]  Z^496 applied to byte j of a register
 constexpr int TAB_LANE = TAB_Z496 + 4 * 256;  // [32] x^(8*16*(31-l)) mod P
 constexpr int TAB_X2N = TAB_LANE + 32;        // [32] x^(2^k) mod P
-constexpr int TAB_WORDS = TAB_X2N + 32;
+constexpr int TAB_HLANE = TAB_X2N + 32;       // [32] hash kernel: Z^(L1 - end_l) for the common segment length L1
+constexpr int TAB_WORDS = TAB_HLANE + 32;
 constexpr int TAB_SMEM_WORDS = TAB_LANE + 32;  // the part staged in shared memory
 
 struct Params {
@@ -56,15 +57,23 @@ struct Params {
   uint64_t chunk_bytes;          // C
   uint32_t zinit_c;              // Z^C(0xFFFFFFFF): the init term of a full chunk
   uint32_t xseg;                 // x^(8*seg_bytes) mod P
+  uint32_t hlane_len;            // L1: the segment length TAB_HLANE was built for
 };
 
-void build_tables(uint32_t* tab /* TAB_WORDS */);
+void build_tables(uint32_t* tab /* TAB_WORDS */, uint64_t common_seg_len);
+// Per-lane run length of the HBM hash kernel for a segment of `len` bytes (multiple of 32).
+__host__ __device__ inline uint64_t hash_lane_run(uint64_t len) { return ((len + 31) / 32 + 31) / 32 * 32; }
 uint32_t host_x2nmodp(uint64_t n, unsigned k, const uint32_t* x2n);
 uint32_t host_multmodp(uint32_t a, uint32_t b);
 
 // Launch mover kernel <mode, kind> with `grid` CTAs on `stream`.
 cudaError_t launch_mover(int mode, int kind, const Params& p, int grid, cudaStream_t stream);
 int mover_threads();
+// Grid for the CRC HBM hash kernel (1 CTA of 1024 threads per SM, 128 KB tables).
+int hash_grid(int sm_count, uint32_t n_desc);
 size_t mover_smem_bytes(int kind);
+// XXH64 HBM hash with one lane per chunk (needs many chunks to fill the GPU).
+bool hash_xxh_lane_ok(int sm_count, uint32_t n_desc);
+cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_t stream);
 
 }  // namespace swk

@@ -109,6 +109,7 @@ swk::Params base_params(swap_ctx* c) {
   p.chunk_bytes = c->plan.C;
   p.zinit_c = c->zinit_c;
   p.xseg = c->xseg;
+  p.hlane_len = (uint32_t)std::min<uint64_t>(c->plan.C, c->cfg.seg_bytes);
   return p;
 }
 
@@ -131,8 +132,15 @@ int hash_kind(swap_ctx* c) { return c->plan.kind == SWAP_CHECKSUM_XXH64 ? swk::K
 swap_status launch(swap_ctx* c, int mode, int kind, const swk::Params& p, cudaStream_t s) {
   if (p.n_desc == 0) return SWAP_OK;
   // never more CTAs than descriptor batches (idle CTAs would only load tables)
-  const int want = (int)std::min<uint64_t>((uint64_t)grid_of(c), (p.n_desc + 15) / 16);
-  cudaError_t e = swk::launch_mover(mode, kind, p, std::max(1, want), s);
+  int want = (int)std::min<uint64_t>((uint64_t)grid_of(c), (p.n_desc + 15) / 16);
+  if ((mode == swk::HASH_STORE || mode == swk::HASH_CHECK) && kind == swk::KIND_CRC32C)
+    want = c->cfg.grid_ctas ? std::min<int>(want, (int)c->cfg.grid_ctas) : swk::hash_grid(c->sm_count, p.n_desc);
+  cudaError_t e;
+  if ((mode == swk::HASH_STORE || mode == swk::HASH_CHECK) && kind == swk::KIND_XXH64 && !c->cfg.grid_ctas &&
+      swk::hash_xxh_lane_ok(c->sm_count, p.n_desc))
+    e = swk::launch_xxh_hash(mode, p, c->sm_count, s);
+  else
+    e = swk::launch_mover(mode, kind, p, std::max(1, want), s);
   if (e != cudaSuccess) return cuda_fail(c, e, "mover kernel launch");
   ++c->launches;
   return SWAP_OK;
@@ -288,7 +296,7 @@ swap_status swap_create(const swap_config_t* cfg_in, swap_ctx_t** out) {
   c->sm_count = prop.multiProcessorCount;
   DeviceGuard g(c->cfg.device);
   std::vector<uint32_t> tab(swk::TAB_WORDS);
-  swk::build_tables(tab.data());
+  swk::build_tables(tab.data(), std::min<uint64_t>(c->cfg.chunk_bytes, c->cfg.seg_bytes));
   if ((e = cudaMalloc(&c->d_tables, tab.size() * 4)) != cudaSuccess ||
       (e = cudaMemcpy(c->d_tables, tab.data(), tab.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess ||
       (e = cudaMalloc(&c->d_status, sizeof(swk::DevStatus))) != cudaSuccess ||
