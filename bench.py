@@ -34,6 +34,16 @@ import workloads as W  # noqa: E402
 
 GB = 1e9
 METRIC = "swap-in (restore + HBM verify) throughput, whole job"
+RESTORE_KERNEL = {
+    "sm": "mover_kernel<SCATTER,CRC|XXH> (SM loads from mapped pinned image + fused checksum)",
+    "sm_nocheck": "mover_kernel<SCATTER,NONE>",
+    "ce_pipe": "restore phase: cudaMemcpyAsync H2D groups (copy engine) + hash_kernel<HASH_CHECK> per group on a side stream",
+    "ce_region": "restore phase: cudaMemcpyAsync per region + HBM hash pass",
+    "ce_chunk": "restore phase: cudaMemcpyAsync per chunk + HBM hash pass",
+    "ce_batch": "restore phase: cudaMemcpyBatchAsync + HBM hash pass",
+}
+VERIFY_KERNEL = {"crc32c": "hash_kernel<HASH_CHECK> (CRC-32C, per-lane runs, replicated slice-by-4 tables)",
+                 "xxh64": "xxh_lane_kernel<HASH_CHECK> (XXH64, one lane per chunk)"}
 PCIE_GEN5_X16_GBPS = 63.015  # 64 GB/s x 128/130 (nominal, per direction)
 MEASURED_PEAKS = os.path.join(ROOT, "MEASURED_PEAKS.json")
 
@@ -54,6 +64,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--sample-bytes", type=int, default=1 << 30, help="oracle sample size per step")
     ap.add_argument("--out", default=None, help="also append the JSON line to this file")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo: test mode, several ranks may share one GPU (collectives on CPU)")
     return ap.parse_args()
 
 
@@ -191,10 +203,16 @@ def run_ours(args):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         print(f"warning: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    ndev = torch.cuda.device_count()
+    local_dev = local % ndev if args.dist_backend == "gloo" else local
+    torch.cuda.set_device(local_dev)
+    dev = torch.device("cuda", local_dev)
     if world > 1:
-        tdist.init_process_group("nccl", device_id=dev)
+        if args.dist_backend == "nccl":
+            tdist.init_process_group("nccl", device_id=dev)
+        else:
+            tdist.init_process_group("gloo")
+    cdev = dev if args.dist_backend == "nccl" else torch.device("cpu")  # where collective tensors live
 
     def barrier():
         if world > 1:
@@ -204,14 +222,14 @@ def run_ours(args):
     def allmax(x: float) -> float:
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        t = torch.tensor([x], dtype=torch.float64, device=cdev)
         tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
         return float(t.item())
 
     def allsum(x: float) -> float:
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        t = torch.tensor([x], dtype=torch.float64, device=cdev)
         tdist.all_reduce(t, op=tdist.ReduceOp.SUM)
         return float(t.item())
 
@@ -227,9 +245,10 @@ def run_ours(args):
     regions = [(base + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs, offs))]
     kind = swap.SWAP_CHECKSUM_CRC32C if args.checksum == "crc32c" else swap.SWAP_CHECKSUM_XXH64
     t0 = time.perf_counter()
-    sw = swap.Swapper(regions, chunk_bytes=args.chunk, checksum=kind, mechanism=args.mechanism, device=local,
+    sw = swap.Swapper(regions, chunk_bytes=args.chunk, checksum=kind, mechanism=args.mechanism, device=local_dev,
                       rank=rank, world=world, grid_ctas=args.grid)
     t_register = time.perf_counter() - t0
+    eff_mech = sw.mechanism()
     stream = torch.cuda.Stream(device=dev)
 
     def poison():
@@ -265,7 +284,7 @@ def run_ours(args):
 
     for _ in range(args.warmup):
         step(None)
-    clocks = ClockSampler(local)
+    clocks = ClockSampler(local_dev)
     rec: dict = {}
     launches0 = sw.launch_count()
     barrier()
@@ -346,19 +365,19 @@ def run_ours(args):
             "dtype": "u8", "data": "synthetic",
             "config": {"workload": f"{name}: {desc}", "regions_per_rank": len(specs),
                        "payload_bytes_per_rank": payload, "chunk_bytes": args.chunk, "checksum": args.checksum,
-                       "mechanism": args.mechanism,
+                       "mechanism": f"{args.mechanism} -> {eff_mech}",
                        "l2": "no flush: every step moves the whole image (>> 126 MB L2)",
                        "parallelism": "single GPU" if world == 1 else f"tp{world} shard per rank (no data collective)"},
             "swap_in_latency_s": round(swapin_ms * 1e-3, 5),
             "swap_in_latency_s_range": [round(min(rec["swapin_ms"]) * 1e-3, 5), round(max(rec["swapin_ms"]) * 1e-3, 5)],
             "restore_GBps_per_gpu": round(achieved, 3),
             "checkpoint_GBps_per_gpu": round(payload / (ckpt_ms * 1e-3) / GB, 3),
-            "roofline": {"bound": "host_link", "kernel": f"{args.mechanism} restore (mover_kernel<SCATTER>)",
+            "roofline": {"bound": "host_link", "kernel": RESTORE_KERNEL[eff_mech],
                          "achieved": round(achieved, 3), "peak": PCIE_GEN5_X16_GBPS, "unit": "GB/s",
                          "frac": round(achieved / PCIE_GEN5_X16_GBPS, 4), "traffic": None,
                          "peak_source": "PCIe Gen5 x16 nominal per direction after 128b/130b (MEASURED_PEAKS.json has no host-link figure)",
                          "frac_of_measured_ce_h2d": round(achieved / ce["h2d"], 4) if ce else None},
-            "roofline_verify": {"bound": "hbm", "kernel": "mover_kernel<HASH_CHECK>",
+            "roofline_verify": {"bound": "hbm", "kernel": VERIFY_KERNEL[args.checksum],
                                 "achieved": round(payload / (verify_ms * 1e-3) / GB, 1), "peak": hbm_peak,
                                 "unit": "GB/s", "frac": round(payload / (verify_ms * 1e-3) / GB / hbm_peak, 4),
                                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)"},

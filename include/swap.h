@@ -164,6 +164,8 @@ SWAP_API swap_status swap_verify(swap_ctx_t* ctx, swap_stream_t stream, int hbm_
 
 /* Selects the data mover for later calls (SWAP_MECH_*). The image format is unchanged. */
 SWAP_API swap_status swap_set_mechanism(swap_ctx_t* ctx, uint32_t mechanism);
+/* The mechanism the next checkpoint/restore will use (SWAP_MECH_AUTO resolved; needs REGISTERED+). */
+SWAP_API swap_status swap_get_mechanism(const swap_ctx_t* ctx, uint32_t* effective);
 
 /* Borrowed views, valid until swap_destroy. The manifest is final only after swap_sync.
  * The image is writable: a caller may load a stored image into it and call swap_import. */

@@ -546,6 +546,13 @@ swap_status swap_set_mechanism(swap_ctx_t* c, uint32_t mechanism) {
   return SWAP_OK;
 }
 
+swap_status swap_get_mechanism(const swap_ctx_t* c, uint32_t* effective) {
+  if (!c || !effective) return SWAP_EINVAL;
+  if (c->st == St::CREATED) return SWAP_ESTATE;
+  *effective = mech(c);
+  return SWAP_OK;
+}
+
 swap_status swap_get_manifest(const swap_ctx_t* c, const void** bytes, size_t* n) {
   if (!c || !bytes || !n) return SWAP_EINVAL;
   if (!c->image) return SWAP_ESTATE;

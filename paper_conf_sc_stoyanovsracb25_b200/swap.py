@@ -28,7 +28,7 @@ U64_MAX = (1 << 64) - 1
 
 EXPORTS = [
     "swap_config_default", "swap_create", "swap_register_regions", "swap_checkpoint", "swap_sync",
-    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_manifest", "swap_get_image",
+    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_get_manifest", "swap_get_image",
     "swap_get_summary", "swap_import", "swap_set_global", "swap_merge_global", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
 ]
@@ -97,6 +97,7 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_restore": (st, [vp, vp]),
         "swap_verify": (st, [vp, vp, ctypes.c_int, P(swap_verify_result_t)]),
         "swap_set_mechanism": (st, [vp, u32]),
+        "swap_get_mechanism": (st, [vp, P(u32)]),
         "swap_get_manifest": (st, [vp, P(vp), P(sz)]),
         "swap_get_image": (st, [vp, P(vp), P(sz)]),
         "swap_get_summary": (st, [vp, P(swap_shard_summary_t)]),
@@ -251,6 +252,12 @@ class Swapper:
         if isinstance(mechanism, str):
             mechanism = MECHANISMS[mechanism]
         self._check(load().swap_set_mechanism(self._ctx, mechanism))
+
+    def mechanism(self) -> str:
+        """Name of the mover the next call uses (AUTO resolved)."""
+        m = ctypes.c_uint32()
+        self._check(load().swap_get_mechanism(self._ctx, ctypes.byref(m)))
+        return {v: k for k, v in MECHANISMS.items()}[m.value]
 
     def import_image(self):
         self._check(load().swap_import(self._ctx))

@@ -1,0 +1,29 @@
+"""N>1 path of bench.py (torchrun, one process per rank) on a single GPU: ranks share cuda:0
+and the collectives (K5 summary all-gather, K6 mismatch all-reduce, max-over-ranks timing)
+run over gloo. The NCCL variant differs only in where the 64-B / 8-B tensors live."""
+import json
+import os
+import subprocess
+import sys
+
+import pytest
+
+from conftest import ROOT
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.timeout(600)
+def test_bench_two_ranks_gloo():
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr=127.0.0.1", "--master-port=29533", os.path.join(ROOT, "bench.py"), "--gpus", "2",
+           "--config", "A", "--steps", "2", "--warmup", "1", "--no-compare", "--no-cpu-baseline",
+           "--dist-backend", "gloo"]
+    out = subprocess.run(cmd, capture_output=True, text=True, timeout=540, cwd=ROOT)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, out.stdout  # rank 0 alone prints
+    rec = json.loads(lines[0])
+    assert rec["n_gpus"] == 2 and rec["scaling"] == "weak" and rec["value"] > 0
+    assert rec["config"]["payload_bytes_per_rank"] == 1 << 26
+    assert rec["gpu_launches"] > 0
