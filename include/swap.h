@@ -58,7 +58,8 @@ typedef int32_t swap_status;
 #define SWAP_CHECKSUM_XXH64 2u  /* XXH64, seed 0 for every chunk */
 
 /* Data mover for checkpoint/restore (the image bytes are identical for all of them): */
-#define SWAP_MECH_AUTO 0u        /* default: SWAP_MECH_CE_PIPE when the payload is >= 512 MiB, else SWAP_MECH_SM */
+#define SWAP_MECH_AUTO 0u        /* default: SWAP_MECH_CE_PIPE when the payload is >= 512 MiB (and, for XXH64,
+                                    chunk_bytes <= 1 MiB), else SWAP_MECH_SM (DESIGN.md §6 mechanism sweep) */
 #define SWAP_MECH_SM 1u          /* one SM kernel: 16-B vector loads/stores to mapped pinned host memory with the
                                     chunk checksum fused from the same registers (one pass, bytes checked in flight) */
 #define SWAP_MECH_CE_REGION 2u   /* copy engine: cudaMemcpyAsync per region + separate HBM hash pass */
@@ -201,6 +202,62 @@ SWAP_API swap_status swap_get_timings(const swap_ctx_t* ctx, swap_timings_t* out
 
 /* Number of libswap kernels this ctx has launched in total (for the bench's gpu_launches). */
 SWAP_API swap_status swap_get_launch_count(const swap_ctx_t* ctx, uint64_t* launches);
+
+/* ---------------------------------------------------------------------------------------------
+ * Device arena with releasable HBM (NEXT-1; "freeing GPU capacity for other workloads",
+ * P:L142 swap-in "requesting the required GPU memory"). An engine allocates the state it wants
+ * swappable inside an arena; after swap_checkpoint + swap_sync, swap_arena_release returns the
+ * arena's physical HBM to the device while its virtual addresses stay reserved; before
+ * swap_restore, swap_arena_reacquire maps fresh HBM at the same addresses (contents undefined
+ * until the restore). Built on CUDA virtual memory management (reserve VA once; 1-GiB physical
+ * slabs created, mapped and released). One arena belongs to one device; calls are not
+ * thread-safe per arena.
+ * ------------------------------------------------------------------------------------------- */
+typedef struct swap_arena swap_arena_t;
+/* Reserves VA for `bytes` (rounded up to the allocation granularity) and maps physical memory.
+ * ENOMEM if the device cannot back it; EUNSUPPORTED if the driver lacks VMM entry points. */
+SWAP_API swap_status swap_arena_create(int device, uint64_t bytes, swap_arena_t** out);
+SWAP_API swap_status swap_arena_info(const swap_arena_t* a, uint64_t* dev_addr, uint64_t* bytes, int* resident);
+/* Synchronises the device, unmaps and frees all physical memory. ESTATE if already released. */
+SWAP_API swap_status swap_arena_release(swap_arena_t* a);
+/* Maps new physical memory at the original addresses. ESTATE if resident; ENOMEM if HBM is short. */
+SWAP_API swap_status swap_arena_reacquire(swap_arena_t* a);
+SWAP_API const char* swap_arena_last_error(const swap_arena_t* a);
+SWAP_API void swap_arena_destroy(swap_arena_t* a);
+
+/* ---------------------------------------------------------------------------------------------
+ * Task manager (NEXT-1): memory reservations and demand-aware preemption, host-only.
+ * PAPER.md §3.3-3.5 (L136-148) and §6 (L230): swap-in requests are reservations served from a
+ * priority queue (several granted at once when memory suffices); when memory is short, running
+ * backends are evicted one at a time in the order (shorter request queue, older last access),
+ * re-checking after each; a write-locked backend is not a candidate; a backend's per-GPU needs are
+ * fixed at init and acquired/released together. All sizes are bytes; GPUs are indices
+ * 0..n_gpus-1. Not thread-safe: the caller serialises calls (the paper's task manager is one actor).
+ * ------------------------------------------------------------------------------------------- */
+typedef struct swap_sched swap_sched_t;
+SWAP_API swap_status swap_sched_create(uint32_t n_gpus, const uint64_t* capacity, swap_sched_t** out);
+/* need[n_gpus]: bytes on each GPU (0 = not placed there). EINVAL: duplicate id, no GPU, or a need
+ * above capacity; ENOMEM: `resident` but it does not fit next to the current residents. */
+SWAP_API swap_status swap_sched_add_backend(swap_sched_t* s, uint32_t id, const uint64_t* need, int resident);
+/* Request-handler bookkeeping: current queue length and last-accessed time. */
+SWAP_API swap_status swap_sched_touch(swap_sched_t* s, uint32_t id, uint32_t queue_len, double last_access);
+SWAP_API swap_status swap_sched_lock(swap_sched_t* s, uint32_t id, int locked);
+/* Victims (eviction order) that would let `id` become resident now; *n = 0 if none needed.
+ * ENOMEM if infeasible; EINVAL if more than `cap` victims (then *n holds the count). */
+SWAP_API swap_status swap_sched_plan(const swap_sched_t* s, uint32_t id, uint32_t* victims, uint32_t cap, uint32_t* n);
+/* Queues a reservation (lower priority value = served first; ties in arrival order). ESTATE if
+ * `id` is resident or already queued. */
+SWAP_API swap_status swap_sched_reserve(swap_sched_t* s, uint32_t id, double priority);
+SWAP_API swap_status swap_sched_cancel(swap_sched_t* s, uint32_t id);
+/* Serves the head reservation: *id = the granted backend (UINT32_MAX if the queue is empty) and its
+ * victims, which are marked swapped out while `id` is marked resident. ENOMEM: the head cannot be
+ * satisfied now (it stays queued; *id names it). The caller then swaps the victims out and `id` in. */
+SWAP_API swap_status swap_sched_grant(swap_sched_t* s, uint32_t* id, uint32_t* victims, uint32_t cap, uint32_t* n);
+/* Voluntary swap-out: releases the backend's reservations on all its GPUs. */
+SWAP_API swap_status swap_sched_release(swap_sched_t* s, uint32_t id);
+SWAP_API swap_status swap_sched_query(const swap_sched_t* s, uint32_t id, int* resident, int* queued);
+SWAP_API swap_status swap_sched_free(const swap_sched_t* s, uint32_t gpu, uint64_t* free_bytes);
+SWAP_API void swap_sched_destroy(swap_sched_t* s);
 
 SWAP_API const char* swap_status_str(swap_status s);
 SWAP_API const char* swap_last_error(const swap_ctx_t* ctx);

@@ -12,7 +12,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libswap.so")
-SOURCES = ["kernels.cu", "plan.cpp", "swap_abi.cpp"]
+SOURCES = ["kernels.cu", "plan.cpp", "swap_abi.cpp", "arena.cpp", "sched.cpp"]
 HEADERS = ["kernels.cuh", "plan.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -34,7 +34,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
     cmd = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC,-fvisibility=hidden",
-           "-Xcompiler", "-Wall", "-I", os.path.join(ROOT, "include"),
+           "-Xcompiler", "-Wall", "-I", os.path.join(ROOT, "include"), "-I", "/usr/local/cuda/include",
            "-o", tmp, *[os.path.join(CSRC, f) for f in SOURCES], "-lcudart_static", "-lrt", "-ldl", "-lpthread"]
     if verbose:
         print(" ".join(cmd), flush=True)

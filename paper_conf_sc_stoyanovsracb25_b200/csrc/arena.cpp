@@ -1,0 +1,214 @@
+// arena.cpp — VMM-backed device arena: the "freeing GPU capacity" half of preemption (§4.2)
+// and the "reserve memory" half of swap-in (§3.4), with virtual addresses that survive
+// both so a restore can scatter to the recorded addresses (SURVEY.md §7 hard part 6, NEXT-1).
+//
+// The VA range is reserved once (cuMemAddressReserve). Physical memory is one cuMemCreate
+// allocation per slab (1 GiB, the last one smaller) mapped into the range with read/write access
+// for the owning device. swap_arena_release unmaps and releases every slab (the HBM returns to the
+// device's free pool; the VA stays reserved); swap_arena_reacquire creates and maps fresh slabs at
+// the same addresses. Driver entry points are resolved at run time through cudart
+// (cudaGetDriverEntryPoint), so libswap.so does not link libcuda and still loads on CPU-only hosts.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/swap.h"
+
+namespace {
+
+struct Drv {
+  decltype(&cuMemGetAllocationGranularity) granularity = nullptr;
+  decltype(&cuMemAddressReserve) reserve = nullptr;
+  decltype(&cuMemAddressFree) addr_free = nullptr;
+  decltype(&cuMemCreate) create = nullptr;
+  decltype(&cuMemRelease) release = nullptr;
+  decltype(&cuMemMap) map = nullptr;
+  decltype(&cuMemUnmap) unmap = nullptr;
+  decltype(&cuMemSetAccess) set_access = nullptr;
+  bool ok = false;
+};
+
+template <class F>
+bool resolve(const char* name, F* fn) {
+  void* p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q) != cudaSuccess || q != cudaDriverEntryPointSuccess ||
+      !p)
+    return false;
+  *fn = reinterpret_cast<F>(p);
+  return true;
+}
+
+const Drv& drv() {
+  static Drv d = [] {
+    Drv x;
+    x.ok = resolve("cuMemGetAllocationGranularity", &x.granularity) && resolve("cuMemAddressReserve", &x.reserve) &&
+           resolve("cuMemAddressFree", &x.addr_free) && resolve("cuMemCreate", &x.create) &&
+           resolve("cuMemRelease", &x.release) && resolve("cuMemMap", &x.map) && resolve("cuMemUnmap", &x.unmap) &&
+           resolve("cuMemSetAccess", &x.set_access);
+    return x;
+  }();
+  return d;
+}
+
+constexpr uint64_t kSlab = 1ull << 30;
+
+}  // namespace
+
+struct swap_arena {
+  int device = 0;
+  CUdeviceptr base = 0;
+  uint64_t bytes = 0;  // rounded to the allocation granularity
+  uint64_t gran = 0;
+  std::vector<CUmemGenericAllocationHandle> slabs;
+  bool resident = false;
+  std::string err;
+};
+
+namespace {
+
+swap_status map_all(swap_arena* a) {
+  const Drv& D = drv();
+  CUmemAllocationProp prop;
+  std::memset(&prop, 0, sizeof(prop));
+  prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+  prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  prop.location.id = a->device;
+  CUmemAccessDesc acc;
+  std::memset(&acc, 0, sizeof(acc));
+  acc.location = prop.location;
+  acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+  for (uint64_t off = 0; off < a->bytes; off += kSlab) {
+    const uint64_t sz = a->bytes - off < kSlab ? a->bytes - off : kSlab;
+    CUmemGenericAllocationHandle h;
+    CUresult r = D.create(&h, sz, &prop, 0);
+    if (r != CUDA_SUCCESS) {
+      a->err = "cuMemCreate failed (" + std::to_string((int)r) + ") at offset " + std::to_string(off);
+      return r == CUDA_ERROR_OUT_OF_MEMORY ? SWAP_ENOMEM : SWAP_ECUDA;
+    }
+    if ((r = D.map(a->base + off, sz, 0, h, 0)) != CUDA_SUCCESS) {
+      D.release(h);
+      a->err = "cuMemMap failed (" + std::to_string((int)r) + ")";
+      return SWAP_ECUDA;
+    }
+    a->slabs.push_back(h);
+    if ((r = D.set_access(a->base + off, sz, &acc, 1)) != CUDA_SUCCESS) {
+      a->err = "cuMemSetAccess failed (" + std::to_string((int)r) + ")";
+      return SWAP_ECUDA;
+    }
+  }
+  a->resident = true;
+  return SWAP_OK;
+}
+
+swap_status unmap_all(swap_arena* a) {
+  const Drv& D = drv();
+  swap_status st = SWAP_OK;
+  for (size_t i = 0; i < a->slabs.size(); ++i) {
+    const uint64_t off = i * kSlab;
+    const uint64_t sz = a->bytes - off < kSlab ? a->bytes - off : kSlab;
+    if (D.unmap(a->base + off, sz) != CUDA_SUCCESS) st = SWAP_ECUDA;
+    if (D.release(a->slabs[i]) != CUDA_SUCCESS) st = SWAP_ECUDA;
+  }
+  a->slabs.clear();
+  a->resident = false;
+  if (st != SWAP_OK) a->err = "cuMemUnmap/cuMemRelease failed";
+  return st;
+}
+
+struct CtxGuard {  // run driver calls with the device's primary context current
+  int prev = -1;
+  explicit CtxGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    cudaSetDevice(dev);
+    cudaFree(nullptr);  // make the primary context current on this thread
+  }
+  ~CtxGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+}  // namespace
+
+extern "C" {
+
+swap_status swap_arena_create(int device, uint64_t bytes, swap_arena_t** out) {
+  if (!out || bytes == 0 || device < 0) return SWAP_EINVAL;
+  *out = nullptr;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device >= ndev) return SWAP_ECUDA;
+  CtxGuard g(device);
+  const Drv& D = drv();
+  if (!D.ok) return SWAP_EUNSUPPORTED;
+  auto* a = new (std::nothrow) swap_arena();
+  if (!a) return SWAP_ENOMEM;
+  a->device = device;
+  CUmemAllocationProp prop;
+  std::memset(&prop, 0, sizeof(prop));
+  prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+  prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  prop.location.id = device;
+  size_t gran = 0;
+  if (D.granularity(&gran, &prop, CU_MEM_ALLOC_GRANULARITY_RECOMMENDED) != CUDA_SUCCESS || gran == 0) {
+    delete a;
+    return SWAP_ECUDA;
+  }
+  a->gran = gran;
+  a->bytes = (bytes + gran - 1) / gran * gran;
+  if (D.reserve(&a->base, a->bytes, kSlab, 0, 0) != CUDA_SUCCESS) {
+    delete a;
+    return SWAP_ENOMEM;
+  }
+  swap_status st = map_all(a);
+  if (st != SWAP_OK) {
+    unmap_all(a);
+    D.addr_free(a->base, a->bytes);
+    delete a;
+    return st;
+  }
+  *out = a;
+  return SWAP_OK;
+}
+
+swap_status swap_arena_info(const swap_arena_t* a, uint64_t* dev_addr, uint64_t* bytes, int* resident) {
+  if (!a) return SWAP_EINVAL;
+  if (dev_addr) *dev_addr = (uint64_t)a->base;
+  if (bytes) *bytes = a->bytes;
+  if (resident) *resident = a->resident ? 1 : 0;
+  return SWAP_OK;
+}
+
+swap_status swap_arena_release(swap_arena_t* a) {
+  if (!a) return SWAP_EINVAL;
+  if (!a->resident) return SWAP_ESTATE;
+  CtxGuard g(a->device);
+  if (cudaDeviceSynchronize() != cudaSuccess) return SWAP_ECUDA;  // no kernel may still touch it
+  return unmap_all(a);
+}
+
+swap_status swap_arena_reacquire(swap_arena_t* a) {
+  if (!a) return SWAP_EINVAL;
+  if (a->resident) return SWAP_ESTATE;
+  CtxGuard g(a->device);
+  swap_status st = map_all(a);
+  if (st != SWAP_OK) unmap_all(a);
+  return st;
+}
+
+const char* swap_arena_last_error(const swap_arena_t* a) { return a ? a->err.c_str() : "null arena"; }
+
+void swap_arena_destroy(swap_arena_t* a) {
+  if (!a) return;
+  {
+    CtxGuard g(a->device);
+    cudaDeviceSynchronize();
+    if (a->resident) unmap_all(a);
+    drv().addr_free(a->base, a->bytes);
+  }
+  delete a;
+}
+
+}  // extern "C"

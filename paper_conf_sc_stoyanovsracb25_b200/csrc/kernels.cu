@@ -596,7 +596,135 @@ int hash_grid(int sm_count, uint32_t n_desc) {
 }
 
 
-// ------------------------------------------------------------------ HBM hash kernel (XXH64)
+// ------------------------------------------------------------------ HBM hash kernel (XXH64, TMA ring)
+// XXH64 consumes a chunk's 32-B stripes strictly in order through four accumulator chains, so a
+// chunk's hashing rate is bounded by the round latency, and parallelism must come from chunks.
+// One warp owns one chunk at a time; lane 0 streams the chunk into a per-warp shared-memory ring
+// with TMA bulk copies (cp.async.bulk + mbarrier complete_tx, XR_STAGES x 4 KiB in flight per
+// warp), and lanes 0..3 run the four accumulators out of shared memory (conflict-free: 4 lanes
+// read 32 contiguous bytes). This keeps the memory pipe full even with few, huge chunks.
+constexpr int XR_WARPS = 4;
+constexpr int XR_STAGES = 3;
+constexpr uint32_t XR_STAGE = 4096;
+constexpr size_t XR_RING = (size_t)XR_STAGES * XR_STAGE;
+constexpr size_t XR_SMEM = XR_WARPS * XR_RING + XR_WARPS * XR_STAGES * 8;
+
+__device__ __forceinline__ uint64_t lds_u64(const uint8_t* p) {
+  return *reinterpret_cast<const uint64_t*>(p);  // 8-B aligned by construction
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(XR_WARPS * 32) xxh_ring_kernel(const Params p) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  uint8_t* ring = smem + (size_t)warp * XR_RING;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + XR_WARPS * XR_RING) + warp * XR_STAGES;
+  if (lane == 0) {
+    for (int s = 0; s < XR_STAGES; ++s) mbar_init(bars + s, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncwarp();
+  uint32_t seq = 0;  // stages issued by this warp so far (buffer = seq % STAGES, parity = seq / STAGES & 1)
+  for (uint32_t idx = blockIdx.x * XR_WARPS + warp; idx < p.n_desc; idx += gridDim.x * XR_WARPS) {
+    const SegDesc d = p.desc[idx];
+    const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
+    const uint64_t len = d.bytes, len16 = len & ~15ull;
+    const uint32_t nst = (uint32_t)((len16 + XR_STAGE - 1) / XR_STAGE);
+    auto issue = [&](uint32_t k) {  // lane 0: stage k of this chunk
+      const uint32_t b = (seq + k) % XR_STAGES;
+      const uint32_t sz = (uint32_t)(len16 - (uint64_t)k * XR_STAGE < XR_STAGE ? len16 - (uint64_t)k * XR_STAGE : XR_STAGE);
+      mbar_expect_tx(bars + b, sz);
+      bulk_g2s(ring + (size_t)b * XR_STAGE, src + (size_t)k * XR_STAGE, sz, bars + b);
+    };
+    if (lane == 0) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      for (uint32_t k = 0; k < nst && k < (uint32_t)XR_STAGES; ++k) issue(k);
+    }
+    uint64_t v = lane == 0 ? P1 + P2 : lane == 1 ? P2 : lane == 2 ? 0ull : 0ull - P1;
+    uint32_t last_b = 0;
+    for (uint32_t k = 0; k < nst; ++k) {
+      const uint32_t b = (seq + k) % XR_STAGES;
+      mbar_wait(bars + b, ((seq + k) / XR_STAGES) & 1u);
+      const uint32_t sz = (uint32_t)(len16 - (uint64_t)k * XR_STAGE < XR_STAGE ? len16 - (uint64_t)k * XR_STAGE : XR_STAGE);
+      if (lane < 4) {
+        const uint8_t* q = ring + (size_t)b * XR_STAGE + 8 * lane;
+        const uint32_t ns = sz / 32;
+#pragma unroll 8
+        for (uint32_t s = 0; s < ns; ++s) v = xround(v, lds_u64(q + 32 * s));
+      }
+      last_b = b;
+      __syncwarp();
+      if (lane == 0 && k + XR_STAGES < nst) {
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        issue(k + XR_STAGES);
+      }
+    }
+    const uint64_t v1 = __shfl_sync(0xffffffffu, v, 0), v2 = __shfl_sync(0xffffffffu, v, 1);
+    const uint64_t v3 = __shfl_sync(0xffffffffu, v, 2), v4 = __shfl_sync(0xffffffffu, v, 3);
+    if (lane == 0) {
+      // bytes after the last whole stripe: in the last stage buffer below len16, in HBM above
+      const uint8_t* lastbuf = ring + (size_t)last_b * XR_STAGE;
+      const uint64_t last_off = nst ? (uint64_t)(nst - 1) * XR_STAGE : 0;
+      auto byte_at = [&](uint64_t o) -> uint64_t { return o < len16 ? lastbuf[o - last_off] : src[o]; };
+      uint64_t h;
+      if (len >= 32) {
+        h = rotl64(v1, 1) + rotl64(v2, 7) + rotl64(v3, 12) + rotl64(v4, 18);
+        h = xmerge(h, v1);
+        h = xmerge(h, v2);
+        h = xmerge(h, v3);
+        h = xmerge(h, v4);
+      } else {
+        h = P5;
+      }
+      h += len;
+      uint64_t o = len / 32 * 32;
+      for (; o + 8 <= len; o += 8) {
+        uint64_t w = 0;
+        for (int i = 7; i >= 0; --i) w = (w << 8) | byte_at(o + i);
+        h ^= xround(0, w);
+        h = rotl64(h, 27) * P1 + P4;
+      }
+      if (o + 4 <= len) {
+        uint64_t w = byte_at(o) | (byte_at(o + 1) << 8) | (byte_at(o + 2) << 16) | (byte_at(o + 3) << 24);
+        h ^= w * P1;
+        h = rotl64(h, 23) * P2 + P3;
+        o += 4;
+      }
+      for (; o < len; ++o) {
+        h ^= byte_at(o) * P5;
+        h = rotl64(h, 11) * P1;
+      }
+      h ^= h >> 33;
+      h *= P2;
+      h ^= h >> 29;
+      h *= P3;
+      h ^= h >> 32;
+      chunk_result<MODE>(p, d.chunk, h);
+    }
+    seq += nst;
+    __syncwarp();
+  }
+}
+
+template <int MODE>
+static cudaError_t launch_xxh_ring(const Params& p, int sm_count, cudaStream_t s) {
+  static unsigned long long attr_set = 0;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (!((attr_set >> (dev & 63)) & 1ull)) {
+    e = cudaFuncSetAttribute(xxh_ring_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)XR_SMEM);
+    if (e != cudaSuccess) return e;
+    attr_set |= 1ull << (dev & 63);
+  }
+  const uint32_t ctas = (p.n_desc + XR_WARPS - 1) / XR_WARPS;
+  const int per_sm = (int)(200 * 1024 / XR_SMEM);  // resident CTAs per SM by shared memory
+  const int grid = (int)std::max<uint32_t>(1, std::min<uint32_t>(ctas, (uint32_t)(sm_count * per_sm)));
+  xxh_ring_kernel<MODE><<<grid, XR_WARPS * 32, XR_SMEM, s>>>(p);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------ HBM hash kernel (XXH64, lane per chunk)
 // XXH64 consumes a chunk's 32-B stripes strictly in order, so parallelism comes from chunks:
 // one LANE per chunk, its four accumulators in registers, one 256-bit load per stripe (a full
 // sector), XK_U stripes in flight. Used for HASH_STORE / HASH_CHECK when there are enough chunks
@@ -717,6 +845,8 @@ static cudaError_t launch_xxh_lane(const Params& p, int sm_count, cudaStream_t s
   return cudaGetLastError();
 }
 
+// Many chunks: one lane per chunk keeps all 32 lanes issuing rounds (5+ TB/s measured); few
+// (large) chunks: the TMA ring keeps the memory pipe full with one warp per chunk.
 bool hash_xxh_lane_ok(int sm_count, uint32_t n_desc) { return n_desc >= (uint32_t)sm_count * 192u; }
 
 int mover_threads() { return THREADS; }
@@ -742,7 +872,9 @@ static cudaError_t launch_t(const Params& p, int grid, cudaStream_t s) {
 
 cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_t s) {
   if (p.n_desc == 0) return cudaSuccess;
-  return mode == HASH_STORE ? launch_xxh_lane<HASH_STORE>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK>(p, sm_count, s);
+  if (hash_xxh_lane_ok(sm_count, p.n_desc))
+    return mode == HASH_STORE ? launch_xxh_lane<HASH_STORE>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK>(p, sm_count, s);
+  return mode == HASH_STORE ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
 }
 
 cudaError_t launch_mover(int mode, int kind, const Params& p, int grid, cudaStream_t s) {

@@ -72,7 +72,7 @@ int mover_threads();
 // Grid for the CRC HBM hash kernel (1 CTA of 1024 threads per SM, 128 KB tables).
 int hash_grid(int sm_count, uint32_t n_desc);
 size_t mover_smem_bytes(int kind);
-// XXH64 HBM hash with one lane per chunk (needs many chunks to fill the GPU).
+// XXH64 HBM hash: one warp per chunk, chunk bytes TMA-streamed through a shared-memory ring.
 bool hash_xxh_lane_ok(int sm_count, uint32_t n_desc);
 cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_t stream);
 

@@ -119,9 +119,13 @@ int grid_of(swap_ctx* c) { return c->cfg.grid_ctas ? (int)c->cfg.grid_ctas : 2 *
 // engines reach a higher link rate than SM-issued accesses) and the single fused
 // SM pass for small ones (no per-copy launch overhead).
 constexpr uint64_t kAutoPipeBytes = 512ull << 20;
+// XXH64 is not combinable: with chunks > 1 MiB a pipeline group holds too few chunks for the
+// side-stream hash to keep up with the link, while the fused SM pass hashes every chunk in flight.
 uint32_t mech(const swap_ctx* c) {
   if (c->cfg.mechanism != SWAP_MECH_AUTO) return c->cfg.mechanism;
-  return c->plan.payload_bytes >= kAutoPipeBytes ? SWAP_MECH_CE_PIPE : SWAP_MECH_SM;
+  if (c->plan.payload_bytes < kAutoPipeBytes) return SWAP_MECH_SM;
+  if (c->plan.kind == SWAP_CHECKSUM_XXH64 && c->plan.C > (1ull << 20)) return SWAP_MECH_SM;
+  return SWAP_MECH_CE_PIPE;
 }
 int kind_of(swap_ctx* c) {
   if (mech(c) == SWAP_MECH_SM_NOCHECK) return swk::KIND_NONE;
@@ -136,8 +140,7 @@ swap_status launch(swap_ctx* c, int mode, int kind, const swk::Params& p, cudaSt
   if ((mode == swk::HASH_STORE || mode == swk::HASH_CHECK) && kind == swk::KIND_CRC32C)
     want = c->cfg.grid_ctas ? std::min<int>(want, (int)c->cfg.grid_ctas) : swk::hash_grid(c->sm_count, p.n_desc);
   cudaError_t e;
-  if ((mode == swk::HASH_STORE || mode == swk::HASH_CHECK) && kind == swk::KIND_XXH64 && !c->cfg.grid_ctas &&
-      swk::hash_xxh_lane_ok(c->sm_count, p.n_desc))
+  if ((mode == swk::HASH_STORE || mode == swk::HASH_CHECK) && kind == swk::KIND_XXH64 && !c->cfg.grid_ctas)
     e = swk::launch_xxh_hash(mode, p, c->sm_count, s);
   else
     e = swk::launch_mover(mode, kind, p, std::max(1, want), s);

@@ -31,6 +31,10 @@ EXPORTS = [
     "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_get_manifest", "swap_get_image",
     "swap_get_summary", "swap_import", "swap_set_global", "swap_merge_global", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
+    "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
+    "swap_arena_destroy", "swap_sched_create", "swap_sched_add_backend", "swap_sched_touch", "swap_sched_lock",
+    "swap_sched_plan", "swap_sched_reserve", "swap_sched_cancel", "swap_sched_grant", "swap_sched_release",
+    "swap_sched_query", "swap_sched_free", "swap_sched_destroy",
 ]
 
 
@@ -109,6 +113,24 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_status_str": (ctypes.c_char_p, [st]),
         "swap_last_error": (ctypes.c_char_p, [vp]),
         "swap_destroy": (None, [vp]),
+        "swap_arena_create": (st, [ctypes.c_int, ctypes.c_uint64, P(vp)]),
+        "swap_arena_info": (st, [vp, P(ctypes.c_uint64), P(ctypes.c_uint64), P(ctypes.c_int)]),
+        "swap_arena_release": (st, [vp]),
+        "swap_arena_reacquire": (st, [vp]),
+        "swap_arena_last_error": (ctypes.c_char_p, [vp]),
+        "swap_arena_destroy": (None, [vp]),
+        "swap_sched_create": (st, [u32, P(ctypes.c_uint64), P(vp)]),
+        "swap_sched_add_backend": (st, [vp, u32, P(ctypes.c_uint64), ctypes.c_int]),
+        "swap_sched_touch": (st, [vp, u32, u32, ctypes.c_double]),
+        "swap_sched_lock": (st, [vp, u32, ctypes.c_int]),
+        "swap_sched_plan": (st, [vp, u32, P(u32), u32, P(u32)]),
+        "swap_sched_reserve": (st, [vp, u32, ctypes.c_double]),
+        "swap_sched_cancel": (st, [vp, u32]),
+        "swap_sched_grant": (st, [vp, P(u32), P(u32), u32, P(u32)]),
+        "swap_sched_release": (st, [vp, u32]),
+        "swap_sched_query": (st, [vp, u32, P(ctypes.c_int), P(ctypes.c_int)]),
+        "swap_sched_free": (st, [vp, u32, P(ctypes.c_uint64)]),
+        "swap_sched_destroy": (None, [vp]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)
@@ -248,6 +270,19 @@ class Swapper:
         d["status"] = st
         return d
 
+    def swap_out(self, arena: "Arena | None" = None, stream=None):
+        """Preempt: checkpoint + seal the manifest, then free the arena's HBM."""
+        self.checkpoint(stream, sync=True)
+        if arena is not None:
+            arena.release()
+
+    def swap_in(self, arena: "Arena | None" = None, stream=None, hbm_pass: bool = True) -> dict:
+        """Swap-in: re-acquire HBM at the recorded addresses, restore, verify."""
+        if arena is not None:
+            arena.reacquire()
+        self.restore(stream)
+        return self.verify(stream, hbm_pass=hbm_pass)
+
     def set_mechanism(self, mechanism: int | str):
         if isinstance(mechanism, str):
             mechanism = MECHANISMS[mechanism]
@@ -312,3 +347,152 @@ class Swapper:
 
     def __exit__(self, *a):
         self.close()
+
+
+# ------------------------------------------------------------------ Arena (releasable HBM)
+class _CudaArray:
+    """Minimal __cuda_array_interface__ exporter so torch can view arena memory (no ownership)."""
+
+    def __init__(self, ptr: int, nbytes: int):
+        self.__cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (ptr, False), "version": 3,
+                                         "strides": None, "stream": None}
+
+
+class Arena:
+    """Device memory whose physical HBM can be released and re-acquired at the same addresses
+    (swap_arena_* in include/swap.h). Carve engine tensors out of it with `tensor()`."""
+
+    def __init__(self, nbytes: int, device: int = 0):
+        h = ctypes.c_void_p()
+        st = load().swap_arena_create(device, nbytes, ctypes.byref(h))
+        if st:
+            raise SwapError(st, f"swap_arena_create({nbytes} B on device {device}) failed")
+        self._h = h
+        self.device = device
+        self._used = 0
+        addr, size, res = ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_int()
+        load().swap_arena_info(h, ctypes.byref(addr), ctypes.byref(size), ctypes.byref(res))
+        self.base, self.nbytes = addr.value, size.value
+
+    def _check(self, st):
+        if st:
+            raise SwapError(st, load().swap_arena_last_error(self._h).decode())
+
+    @property
+    def resident(self) -> bool:
+        res = ctypes.c_int()
+        load().swap_arena_info(self._h, None, None, ctypes.byref(res))
+        return bool(res.value)
+
+    def tensor(self, offset: int, nbytes: int):
+        """A torch uint8 CUDA tensor viewing arena bytes [offset, offset + nbytes)."""
+        import torch
+
+        assert 0 <= offset and offset + nbytes <= self.nbytes
+        return torch.as_tensor(_CudaArray(self.base + offset, nbytes), device=f"cuda:{self.device}")
+
+    def alloc(self, nbytes: int, align: int = 256):
+        """Bump-allocates `nbytes` (aligned) and returns (dev_addr, torch view)."""
+        off = (self._used + align - 1) // align * align
+        if off + nbytes > self.nbytes:
+            raise SwapError(SWAP_ENOMEM, "arena full")
+        self._used = off + nbytes
+        return self.base + off, self.tensor(off, nbytes)
+
+    def release(self):
+        self._check(load().swap_arena_release(self._h))
+
+    def reacquire(self):
+        self._check(load().swap_arena_reacquire(self._h))
+
+    def close(self):
+        if getattr(self, "_h", None):
+            load().swap_arena_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+# ------------------------------------------------------------------ Scheduler (task manager)
+class Scheduler:
+    """Reservations + demand-aware preemption (swap_sched_* in include/swap.h; §3.3-3.5, §6)."""
+
+    MAX_VICTIMS = 4096
+
+    def __init__(self, capacity_per_gpu):
+        caps = (ctypes.c_uint64 * len(capacity_per_gpu))(*capacity_per_gpu)
+        h = ctypes.c_void_p()
+        st = load().swap_sched_create(len(capacity_per_gpu), caps, ctypes.byref(h))
+        if st:
+            raise SwapError(st, "swap_sched_create")
+        self._h, self.n_gpus = h, len(capacity_per_gpu)
+        self._buf = (ctypes.c_uint32 * self.MAX_VICTIMS)()
+
+    def _check(self, st, what):
+        if st:
+            raise SwapError(st, what)
+
+    def add_backend(self, bid: int, need_per_gpu, resident: bool = False):
+        need = (ctypes.c_uint64 * self.n_gpus)(*need_per_gpu)
+        self._check(load().swap_sched_add_backend(self._h, bid, need, int(resident)), f"add_backend({bid})")
+
+    def touch(self, bid: int, queue_len: int, last_access: float):
+        self._check(load().swap_sched_touch(self._h, bid, queue_len, last_access), "touch")
+
+    def lock(self, bid: int, locked: bool = True):
+        self._check(load().swap_sched_lock(self._h, bid, int(locked)), "lock")
+
+    def plan(self, bid: int):
+        """Victims in eviction order, or None if infeasible."""
+        n = ctypes.c_uint32()
+        st = load().swap_sched_plan(self._h, bid, self._buf, self.MAX_VICTIMS, ctypes.byref(n))
+        if st == SWAP_ENOMEM:
+            return None
+        self._check(st, "plan")
+        return list(self._buf[:n.value])
+
+    def reserve(self, bid: int, priority: float):
+        self._check(load().swap_sched_reserve(self._h, bid, priority), f"reserve({bid})")
+
+    def cancel(self, bid: int):
+        self._check(load().swap_sched_cancel(self._h, bid), "cancel")
+
+    def grant(self):
+        """(backend, victims) for the head reservation; None if the queue is empty;
+        ('blocked', backend) if the head cannot be satisfied now."""
+        bid, n = ctypes.c_uint32(), ctypes.c_uint32()
+        st = load().swap_sched_grant(self._h, ctypes.byref(bid), self._buf, self.MAX_VICTIMS, ctypes.byref(n))
+        if st == SWAP_ENOMEM:
+            return ("blocked", bid.value)
+        self._check(st, "grant")
+        if bid.value == 0xFFFFFFFF:
+            return None
+        return bid.value, list(self._buf[:n.value])
+
+    def release(self, bid: int):
+        self._check(load().swap_sched_release(self._h, bid), "release")
+
+    def state(self, bid: int):
+        r, q = ctypes.c_int(), ctypes.c_int()
+        self._check(load().swap_sched_query(self._h, bid, ctypes.byref(r), ctypes.byref(q)), "query")
+        return {"resident": bool(r.value), "queued": bool(q.value)}
+
+    def free(self, gpu: int) -> int:
+        f = ctypes.c_uint64()
+        self._check(load().swap_sched_free(self._h, gpu, ctypes.byref(f)), "free")
+        return f.value
+
+    def close(self):
+        if getattr(self, "_h", None):
+            load().swap_sched_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
