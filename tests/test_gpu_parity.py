@@ -104,6 +104,14 @@ def test_launch_shapes(swp, orc, stream, grid, seg):
     roundtrip(swp, orc, stream, specs, 4, 1 << 20, 1, "sm", key=("A", 4, 1 << 20, 1), grid_ctas=grid, seg_bytes=seg)
 
 
+@pytest.mark.parametrize("mech", ["ce_region", "ce_pipe"])
+def test_xxh64_hash_kernels_many_and_few_chunks(swp, orc, stream, mech):
+    """XXH64 HBM passes: 1 KiB chunks (65 K chunks -> lane-per-chunk kernel) and 16 MiB chunks
+    (5 chunks -> TMA-ring kernel)."""
+    for C in (1024, 16 << 20):
+        roundtrip(swp, orc, stream, W.config_a(6), 6, C, 2, mech, key=("A", 6, C, 2))
+
+
 @pytest.mark.parametrize("pipe_mib", [1, 3, 16])
 @pytest.mark.parametrize("kind", [1, 2], ids=["crc32c", "xxh64"])
 def test_ce_pipe_groups(swp, orc, stream, pipe_mib, kind):

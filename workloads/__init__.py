@@ -107,6 +107,60 @@ def config_d(rank: int) -> list[RegionSpec]:
     return w + kv + _workspace(200 + rank, 2 * GiB)
 
 
+# ---------------------------------------------------------------- config E engines (hot-swap trace)
+# BASELINE.json configs[4]: three engines (8B / 14B / 32B TP=2) swapped on GPU pairs. Per-GPU KV pool
+# bytes/token/layer = 2 (K,V) x kv_heads/TP x head_dim 128 x 2 B. SURVEY.md §8(d) E uses 2^17 tokens;
+# the one-GPU replay in tools/trace_e.py uses kv_tokens = 2^16 so that every engine's pinned image
+# (about 158 GB in total) fits the GPU box's 196 GB of host RAM (DESIGN.md §"Config E").
+def engine_e(model: str, rank: int = 0, kv_tokens: int = 1 << 16) -> list[RegionSpec]:
+    if model == "8b":  # Llama-3.1-8B, TP=1
+        w = _decoder_weights(128256, 4096, 32, 6144, 4096, 14336, qkv_bias=False)
+        layers, kv_per_tok = 32, 2 * 8 * 128 * 2
+    elif model == "14b":  # DeepSeek-R1-Distill-Qwen-14B / Qwen2.5-14B, TP=1
+        w = _decoder_weights(152064, 5120, 48, 7168, 5120, 13824, qkv_bias=True)
+        layers, kv_per_tok = 48, 2 * 8 * 128 * 2
+    elif model == "32b":  # Qwen2.5-32B, TP=2 shard `rank`
+        w = _decoder_weights(76032, 5120, 64, 3584, 2560, 13824, qkv_bias=True)
+        layers, kv_per_tok = 64, 2 * 4 * 128 * 2
+    else:
+        raise ValueError(model)
+    kv = [RegionSpec(f"kv{l}", KIND_KV, kv_tokens * kv_per_tok) for l in range(layers)]
+    return w + kv + _workspace(300 + 10 * {"8b": 0, "14b": 1, "32b": 2}[model] + rank, 2 * GiB)
+
+
+def trace_e(seed: int, duration_s: float, rate_per_s: float = 0.25, day_s: float = 600.0,
+            shares=(("8b", 0.5), ("14b", 0.3), ("32b", 0.2)), burst_on_s: float = 30.0,
+            burst_off_s: float = 120.0, burst_factor: float = 10.0, service_mean_s: float = 2.0):
+    """Azure-shaped arrivals for config E (Fig. 1 shape):
+    non-homogeneous Poisson with a diurnal sinusoid (one "day" = day_s seconds) times an on/off
+    burst process (exponential ON/OFF periods, rate x burst_factor while ON), model shares, and
+    lognormal service times with the given mean (sigma 0.5). Returns [(t, model, service_s)]."""
+    rng = np.random.Generator(np.random.PCG64(seed))
+    # burst switching times
+    edges, t, on = [], 0.0, False
+    while t < duration_s:
+        t += rng.exponential(burst_on_s if on else burst_off_s)
+        edges.append((t, not on))
+        on = not on
+    lam_max = rate_per_s * 1.8 * burst_factor
+    out, t, k, on = [], 0.0, 0, False
+    names = [m for m, _ in shares]
+    probs = np.array([p for _, p in shares]) / sum(p for _, p in shares)
+    sigma = 0.5
+    mu = math.log(service_mean_s) - sigma * sigma / 2
+    while True:
+        t += rng.exponential(1.0 / lam_max)  # thinning
+        if t >= duration_s:
+            break
+        while k < len(edges) and edges[k][0] <= t:
+            on = edges[k][1]
+            k += 1
+        lam = rate_per_s * (1.0 + 0.8 * math.sin(2 * math.pi * t / day_s)) * (burst_factor if on else 1.0)
+        if rng.random() * lam_max <= lam:
+            out.append((t, names[int(rng.choice(len(names), p=probs))], float(rng.lognormal(mu, sigma))))
+    return out
+
+
 def scaled(specs: list[RegionSpec], total: int) -> list[RegionSpec]:
     """Same region mix with every size scaled so the sum is about `total` (cheap GPU cases)."""
     s = sum(r.nbytes for r in specs)
