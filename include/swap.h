@@ -163,6 +163,18 @@ SWAP_API swap_status swap_restore(swap_ctx_t* ctx, swap_stream_t stream);
  * Returns ECORRUPT iff a mismatch was found or the manifest is bad, else OK. */
 SWAP_API swap_status swap_verify(swap_ctx_t* ctx, swap_stream_t stream, int hbm_pass, swap_verify_result_t* res);
 
+/* Engine-aware state reduction (NEXT-3; "engine-specific optimizations, such as vLLM's sleep
+ * API ... reduce both GPU state size and checkpoint/restore latency"). Per-region swap policy: */
+#define SWAP_POLICY_SAVE 0u      /* default: gathered by every checkpoint, scattered by every restore */
+#define SWAP_POLICY_SAVE_ONCE 1u /* immutable after registration (weights): gathered by the first checkpoint
+                                    only; later checkpoints keep its image bytes and chunk checksums */
+#define SWAP_POLICY_DISCARD 2u   /* never saved (a KV pool the engine rebuilds, vLLM sleep level 2): captured
+                                    as zeros (image bytes 0, c_g = checksum of a zero chunk), restored by
+                                    zero-filling the device bytes, checked by the HBM pass like any region */
+/* Sets region `region_index`'s policy (index in registration order). Only between
+ * swap_register_regions and the first checkpoint (ESTATE otherwise). */
+SWAP_API swap_status swap_set_region_policy(swap_ctx_t* ctx, uint32_t region_index, uint32_t policy);
+
 /* Selects the data mover for later calls (SWAP_MECH_*). The image format is unchanged. */
 SWAP_API swap_status swap_set_mechanism(swap_ctx_t* ctx, uint32_t mechanism);
 /* The mechanism the next checkpoint/restore will use (SWAP_MECH_AUTO resolved; needs REGISTERED+). */

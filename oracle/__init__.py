@@ -191,6 +191,23 @@ def checkpoint(regions, mem: np.ndarray, mem_base: int, kind: int, chunk_bytes: 
     return rc, (image if rc == 0 else None), mo.value
 
 
+SAVE, SAVE_ONCE, DISCARD = 0, 1, 2
+
+
+def policy_view(regions, policies, mem_now: np.ndarray, mem_first: np.ndarray, mem_base: int) -> np.ndarray:
+    """The bytes a checkpoint captures under per-region swap policies (reading 24):
+    SAVE -> the region now; SAVE_ONCE -> the region as it was at the first checkpoint;
+    DISCARD -> zeros. Feed the result to checkpoint()."""
+    view = mem_now.copy()
+    for (rid, addr, nbytes, kind), pol in zip(regions, policies):
+        lo = addr - mem_base
+        if pol == DISCARD:
+            view[lo:lo + nbytes] = 0
+        elif pol == SAVE_ONCE:
+            view[lo:lo + nbytes] = mem_first[lo:lo + nbytes]
+    return view
+
+
 def summary(manifest: np.ndarray, image_bytes: int) -> bytes:
     out = np.zeros(64, np.uint8)
     rc = lib().oracle_summary(_ptr(manifest), manifest.size, image_bytes, _ptr(out))

@@ -44,6 +44,20 @@ struct Group {  // CE_PIPE unit: whole chunks, descriptor range [d0, d1)
   std::vector<Span> spans;
 };
 
+// The work of one pass over a subset of the regions (selected by their swap policy): segment
+// descriptors on the device plus the copy-engine views of the same bytes. A chunk's segments are
+// always contiguous, so per-chunk CRC combining works on any set.
+struct DescSet {
+  swk::SegDesc* d_desc = nullptr;
+  uint32_t n_desc = 0;
+  std::vector<Span> region_spans;         // CE_REGION
+  std::vector<void*> ce_dev, ce_host;     // CE_CHUNK / CE_BATCH, one entry per chunk
+  std::vector<size_t> ce_bytes;
+  std::vector<Group> groups;              // CE_PIPE
+  std::vector<cudaEvent_t> group_ev;
+  bool owned = false;                     // false: an alias of another set
+};
+
 struct swap_ctx {
   swap_config_t cfg{};
   St st = St::CREATED;
@@ -54,18 +68,18 @@ struct swap_ctx {
   size_t map_bytes = 0;
   bool host_registered = false;
   uint8_t* image_dev = nullptr;  // device (UVA) view of the image
-  // device-side work state
-  swk::SegDesc* d_desc = nullptr;
-  uint32_t n_desc = 0;
+  // device-side work state; sets: all regions (verify), SAVE|SAVE_ONCE (first checkpoint, restore),
+  // SAVE (later checkpoints), DISCARD chunks hashed from a zero buffer (their c_g)
+  std::vector<uint32_t> policy;
+  DescSet s_all, s_move, s_save, s_zero;
+  bool first_ckpt_done = false;
+  uint8_t* d_zero = nullptr;
   uint32_t* d_partial = nullptr;
   uint32_t* d_arrive = nullptr;
   swk::DevStatus* d_status = nullptr;
   swk::DevStatus* h_status = nullptr;  // pinned
   uint32_t* d_tables = nullptr;
   uint32_t zinit_c = 0, xseg = 0;
-  // copy-engine lists (per chunk and per region)
-  std::vector<void*> ce_dev, ce_host;
-  std::vector<size_t> ce_bytes;
   cudaEvent_t ev[6] = {};  // checkpoint, restore, verify: begin/end pairs
   bool pending[3] = {false, false, false};
   float ms[3] = {0.f, 0.f, 0.f};
@@ -73,8 +87,6 @@ struct swap_ctx {
   std::string err;
   std::vector<swap_shard_summary_t> global;
   // CE_PIPE
-  std::vector<Group> groups;
-  std::vector<cudaEvent_t> group_ev;
   cudaStream_t side = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };
@@ -93,10 +105,10 @@ swap_status cuda_fail(swap_ctx* c, cudaError_t e, const char* what) {
 
 uint8_t* manifest_ptr(swap_ctx* c) { return c->image + c->plan.manifest_off; }
 
-swk::Params base_params(swap_ctx* c) {
+swk::Params base_params(swap_ctx* c, const DescSet& S) {
   swk::Params p{};
-  p.desc = c->d_desc;
-  p.n_desc = c->n_desc;
+  p.desc = S.d_desc;
+  p.n_desc = S.n_desc;
   p.seg_bytes = c->cfg.seg_bytes;
   p.partial = c->d_partial;
   p.arrive = c->d_arrive;
@@ -157,19 +169,19 @@ swap_status memcpy_dir(swap_ctx* c, const Span& sp, int dir, cudaStream_t s) {
 }
 
 // Copy-engine data movement for CE_REGION / CE_CHUNK / CE_BATCH: dir 0 = device -> image, 1 = image -> device.
-swap_status ce_copy(swap_ctx* c, int dir, cudaStream_t s) {
+swap_status ce_copy(swap_ctx* c, DescSet& S, int dir, cudaStream_t s) {
   const uint32_t m = mech(c);
   if (m == SWAP_MECH_CE_REGION) {
-    for (const auto& r : c->plan.regions) {
-      if (!r.r.bytes) continue;
-      swap_status st = memcpy_dir(c, Span{r.r.dev_addr, c->image + r.off, r.r.bytes}, dir, s);
+    for (const Span& sp : S.region_spans) {
+      swap_status st = memcpy_dir(c, sp, dir, s);
       if (st != SWAP_OK) return st;
     }
     return SWAP_OK;
   }
   if (m == SWAP_MECH_CE_CHUNK) {
-    for (size_t i = 0; i < c->ce_bytes.size(); ++i) {
-      swap_status st = memcpy_dir(c, Span{(uint64_t)c->ce_dev[i], (uint8_t*)c->ce_host[i], c->ce_bytes[i]}, dir, s);
+    for (size_t i = 0; i < S.ce_bytes.size(); ++i) {
+      Span sp{reinterpret_cast<uint64_t>(S.ce_dev[i]), static_cast<uint8_t*>(S.ce_host[i]), S.ce_bytes[i]};
+      swap_status st = memcpy_dir(c, sp, dir, s);
       if (st != SWAP_OK) return st;
     }
     return SWAP_OK;
@@ -179,7 +191,7 @@ swap_status ce_copy(swap_ctx* c, int dir, cudaStream_t s) {
     c->err = "SWAP_MECH_CE_BATCH needs a non-default stream (cudaMemcpyBatchAsync restriction)";
     return SWAP_EUNSUPPORTED;
   }
-  if (c->ce_bytes.empty()) return SWAP_OK;
+  if (S.ce_bytes.empty()) return SWAP_OK;
   cudaMemcpyAttributes attr;
   std::memset(&attr, 0, sizeof(attr));
   attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
@@ -188,9 +200,9 @@ swap_status ce_copy(swap_ctx* c, int dir, cudaStream_t s) {
   attr.dstLocHint.type = dir == 0 ? cudaMemLocationTypeHost : cudaMemLocationTypeDevice;
   attr.dstLocHint.id = dir == 0 ? 0 : c->cfg.device;
   size_t attr_idx = 0, fail_idx = 0;
-  std::vector<void*>& dst = dir == 0 ? c->ce_host : c->ce_dev;
-  std::vector<void*>& src = dir == 0 ? c->ce_dev : c->ce_host;
-  CUDA_TRY(c, cudaMemcpyBatchAsync(dst.data(), src.data(), c->ce_bytes.data(), c->ce_bytes.size(), &attr, &attr_idx, 1,
+  std::vector<void*>& dst = dir == 0 ? S.ce_host : S.ce_dev;
+  std::vector<void*>& src = dir == 0 ? S.ce_dev : S.ce_host;
+  CUDA_TRY(c, cudaMemcpyBatchAsync(dst.data(), src.data(), S.ce_bytes.data(), S.ce_bytes.size(), &attr, &attr_idx, 1,
                                    &fail_idx, s));
   return SWAP_OK;
 }
@@ -198,18 +210,18 @@ swap_status ce_copy(swap_ctx* c, int dir, cudaStream_t s) {
 // CE_PIPE. Checkpoint (dir 0): the hash pass over HBM runs on the side stream concurrently with the
 // D2H copies (both only read HBM). Restore (dir 1): group g's H2D copies are followed by an event;
 // the side stream waits for it and checks group g from HBM while the copy engine moves group g+1.
-swap_status ce_pipe(swap_ctx* c, int dir, const swk::Params& base, cudaStream_t s) {
+swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, cudaStream_t s) {
   CUDA_TRY(c, cudaEventRecord(c->ev_fork, s));
   CUDA_TRY(c, cudaStreamWaitEvent(c->side, c->ev_fork, 0));
   swap_status st;
   if (dir == 0 && (st = launch(c, swk::HASH_STORE, hash_kind(c), base, c->side)) != SWAP_OK) return st;
-  for (size_t g = 0; g < c->groups.size(); ++g) {
-    const Group& G = c->groups[g];
+  for (size_t g = 0; g < S.groups.size(); ++g) {
+    const Group& G = S.groups[g];
     for (const Span& sp : G.spans)
       if ((st = memcpy_dir(c, sp, dir, s)) != SWAP_OK) return st;
     if (dir == 1) {
-      CUDA_TRY(c, cudaEventRecord(c->group_ev[g], s));
-      CUDA_TRY(c, cudaStreamWaitEvent(c->side, c->group_ev[g], 0));
+      CUDA_TRY(c, cudaEventRecord(S.group_ev[g], s));
+      CUDA_TRY(c, cudaStreamWaitEvent(c->side, S.group_ev[g], 0));
       swk::Params p = base;
       p.desc = base.desc + G.d0;
       p.partial = base.partial + G.d0;
@@ -232,8 +244,22 @@ swap_status collect_timing(swap_ctx* c, int p) {
 
 bool is_ce(uint32_t m) { return m == SWAP_MECH_CE_REGION || m == SWAP_MECH_CE_CHUNK || m == SWAP_MECH_CE_BATCH; }
 
+void free_set(DescSet& S) {
+  if (S.owned) {
+    if (S.d_desc) cudaFree(S.d_desc);
+    for (auto& e : S.group_ev)
+      if (e) cudaEventDestroy(e);
+  }
+  S = DescSet();
+}
+
 void release(swap_ctx* c) {
-  if (c->d_desc) cudaFree(c->d_desc);
+  free_set(c->s_move);
+  free_set(c->s_save);
+  free_set(c->s_zero);
+  free_set(c->s_all);
+  if (c->d_zero) cudaFree(c->d_zero);
+  c->d_zero = nullptr;
   if (c->d_partial) cudaFree(c->d_partial);
   if (c->d_arrive) cudaFree(c->d_arrive);
   if (c->d_status) cudaFree(c->d_status);
@@ -241,16 +267,127 @@ void release(swap_ctx* c) {
   if (c->d_tables) cudaFree(c->d_tables);
   for (auto& e : c->ev)
     if (e) cudaEventDestroy(e);
-  for (auto& e : c->group_ev)
-    if (e) cudaEventDestroy(e);
-  c->group_ev.clear();
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_join) cudaEventDestroy(c->ev_join);
   if (c->side) cudaStreamDestroy(c->side);
   if (c->host_registered) cudaHostUnregister(c->image);
   if (c->image) munmap(c->image, c->map_bytes);
-  c->d_desc = nullptr;
+  c->d_partial = nullptr;
   c->image = nullptr;
+}
+
+// Builds the descriptor set of the regions `pick` selects. zero_src: segment sources point into
+// the zero buffer instead of the region (hashing DISCARD chunks as zeros).
+template <class Pick>
+swap_status build_set(swap_ctx* c, DescSet* S, Pick pick, bool zero_src) {
+  const swp::Plan& P = c->plan;
+  const uint64_t seg = P.kind == SWAP_CHECKSUM_XXH64 ? P.C : std::min<uint64_t>(P.C, c->cfg.seg_bytes);
+  std::vector<swk::SegDesc> desc;
+  const uint64_t target = (uint64_t)c->cfg.pipe_mib << 20;
+  Group cur{0, 0, {}};
+  uint64_t cur_bytes = 0;
+  for (size_t i = 0; i < P.regions.size(); ++i) {
+    const auto& r = P.regions[i];
+    if (!pick(i) || r.r.bytes == 0) continue;
+    S->region_spans.push_back(Span{r.r.dev_addr, c->image + r.off, r.r.bytes});
+    for (uint64_t j = 0; j < r.nchunks; ++j) {
+      const uint64_t lo = j * P.C, len = std::min<uint64_t>(P.C, r.r.bytes - lo);
+      const uint32_t nseg = (uint32_t)((len + seg - 1) / seg);
+      for (uint32_t s = 0; s < nseg; ++s) {
+        swk::SegDesc d;
+        d.dev = zero_src ? reinterpret_cast<uint64_t>(c->d_zero) + s * seg : r.r.dev_addr + lo + s * seg;
+        d.host = reinterpret_cast<uint64_t>(c->image_dev + r.off + lo + s * seg);
+        d.bytes = (uint32_t)std::min<uint64_t>(seg, len - s * seg);
+        d.chunk = (uint32_t)(r.first + j);
+        d.seg = s;
+        d.nseg = nseg;
+        desc.push_back(d);
+      }
+      S->ce_dev.push_back(reinterpret_cast<void*>(r.r.dev_addr + lo));
+      S->ce_host.push_back(c->image + r.off + lo);
+      S->ce_bytes.push_back(len);
+      // CE_PIPE groups: consecutive whole chunks up to ~pipe_mib MiB; spans merge contiguous chunks
+      Span sp{r.r.dev_addr + lo, c->image + r.off + lo, len};
+      if (!cur.spans.empty() && cur.spans.back().dev + cur.spans.back().bytes == sp.dev &&
+          cur.spans.back().host + cur.spans.back().bytes == sp.host)
+        cur.spans.back().bytes += len;
+      else
+        cur.spans.push_back(sp);
+      cur.d1 = (uint32_t)desc.size();
+      cur_bytes += len;
+      if (cur_bytes >= target) {
+        S->groups.push_back(std::move(cur));
+        cur = Group{(uint32_t)desc.size(), (uint32_t)desc.size(), {}};
+        cur_bytes = 0;
+      }
+    }
+  }
+  if (!cur.spans.empty()) S->groups.push_back(std::move(cur));
+  if (desc.size() > 0xFFFFFFFFull) {
+    c->err = "too many segments";
+    return SWAP_EUNSUPPORTED;
+  }
+  S->owned = true;
+  S->n_desc = (uint32_t)desc.size();
+  CUDA_TRY(c, cudaMalloc(&S->d_desc, std::max<size_t>(1, desc.size()) * sizeof(swk::SegDesc)));
+  if (!desc.empty())
+    CUDA_TRY(c, cudaMemcpy(S->d_desc, desc.data(), desc.size() * sizeof(swk::SegDesc), cudaMemcpyHostToDevice));
+  S->group_ev.assign(S->groups.size(), nullptr);
+  for (auto& e : S->group_ev) CUDA_TRY(c, cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  return SWAP_OK;
+}
+
+DescSet alias_of(const DescSet& S) {
+  DescSet a = S;
+  a.owned = false;
+  return a;
+}
+
+// (Re)builds every set from the current policies.
+swap_status build_sets(swap_ctx* c) {
+  free_set(c->s_move);
+  free_set(c->s_save);
+  free_set(c->s_zero);
+  free_set(c->s_all);
+  if (c->d_zero) {
+    cudaFree(c->d_zero);
+    c->d_zero = nullptr;
+  }
+  const auto& pol = c->policy;
+  bool any_once = false, any_discard = false;
+  uint64_t zero_bytes = 0;
+  for (size_t i = 0; i < pol.size(); ++i) {
+    any_once |= pol[i] == SWAP_POLICY_SAVE_ONCE;
+    if (pol[i] == SWAP_POLICY_DISCARD) {
+      any_discard = true;
+      zero_bytes = std::max<uint64_t>(zero_bytes, std::min<uint64_t>(c->plan.C, c->plan.regions[i].r.bytes));
+    }
+  }
+  swap_status st = build_set(c, &c->s_all, [](size_t) { return true; }, false);
+  if (st != SWAP_OK) return st;
+  if (!any_once && !any_discard) {
+    c->s_move = alias_of(c->s_all);
+    c->s_save = alias_of(c->s_all);
+  } else {
+    st = build_set(c, &c->s_move, [&](size_t i) { return pol[i] != SWAP_POLICY_DISCARD; }, false);
+    if (st != SWAP_OK) return st;
+    if (any_once) {
+      st = build_set(c, &c->s_save, [&](size_t i) { return pol[i] == SWAP_POLICY_SAVE; }, false);
+      if (st != SWAP_OK) return st;
+    } else {
+      c->s_save = alias_of(c->s_move);
+    }
+  }
+  if (any_discard) {
+    CUDA_TRY(c, cudaMalloc(&c->d_zero, std::max<uint64_t>(16, (zero_bytes + 31) & ~31ull)));
+    CUDA_TRY(c, cudaMemset(c->d_zero, 0, std::max<uint64_t>(16, (zero_bytes + 31) & ~31ull)));
+    st = build_set(c, &c->s_zero, [&](size_t i) { return pol[i] == SWAP_POLICY_DISCARD; }, true);
+    if (st != SWAP_OK) return st;
+  }
+  if (c->d_partial) cudaFree(c->d_partial);
+  c->d_partial = nullptr;
+  CUDA_TRY(c, cudaMalloc(&c->d_partial, std::max<size_t>(1, c->s_all.n_desc) * 4));
+  return SWAP_OK;
 }
 
 }  // namespace
@@ -361,75 +498,14 @@ swap_status swap_register_regions(swap_ctx_t* c, const swap_region_t* regions, s
   c->image_dev = static_cast<uint8_t*>(dview);
   swp::write_manifest_skeleton(P, manifest_ptr(c));
 
-  // Segment descriptors: CRC-32C chunks split at seg_bytes; XXH64 segments are whole chunks.
-  const uint64_t seg = P.kind == SWAP_CHECKSUM_XXH64 ? P.C : std::min<uint64_t>(P.C, c->cfg.seg_bytes);
-  std::vector<swk::SegDesc> desc;
-  c->ce_dev.clear();
-  c->ce_host.clear();
-  c->ce_bytes.clear();
-  for (const auto& r : P.regions) {
-    for (uint64_t j = 0; j < r.nchunks; ++j) {
-      const uint64_t lo = j * P.C, len = std::min<uint64_t>(P.C, r.r.bytes - lo);
-      const uint32_t nseg = (uint32_t)((len + seg - 1) / seg);
-      for (uint32_t s = 0; s < nseg; ++s) {
-        swk::SegDesc d;
-        d.dev = r.r.dev_addr + lo + s * seg;
-        d.host = reinterpret_cast<uint64_t>(c->image_dev + r.off + lo + s * seg);
-        d.bytes = (uint32_t)std::min<uint64_t>(seg, len - s * seg);
-        d.chunk = (uint32_t)(r.first + j);
-        d.seg = s;
-        d.nseg = nseg;
-        desc.push_back(d);
-      }
-      c->ce_dev.push_back(reinterpret_cast<void*>(r.r.dev_addr + lo));
-      c->ce_host.push_back(c->image + r.off + lo);
-      c->ce_bytes.push_back(len);
-    }
-  }
-  // CE_PIPE groups: consecutive whole chunks up to ~pipe_mib MiB; spans merge chunks of one region.
-  {
-    const uint64_t target = (uint64_t)c->cfg.pipe_mib << 20;
-    Group cur{0, 0, {}};
-    uint64_t cur_bytes = 0;
-    size_t di = 0;
-    for (const auto& r : P.regions) {
-      for (uint64_t j = 0; j < r.nchunks; ++j) {
-        const uint64_t lo = j * P.C, len = std::min<uint64_t>(P.C, r.r.bytes - lo);
-        Span sp{r.r.dev_addr + lo, c->image + r.off + lo, len};
-        if (!cur.spans.empty() && cur.spans.back().dev + cur.spans.back().bytes == sp.dev &&
-            cur.spans.back().host + cur.spans.back().bytes == sp.host)
-          cur.spans.back().bytes += len;
-        else
-          cur.spans.push_back(sp);
-        while (di < desc.size() && desc[di].chunk == r.first + j) ++di;
-        cur.d1 = (uint32_t)di;
-        cur_bytes += len;
-        if (cur_bytes >= target) {
-          c->groups.push_back(std::move(cur));
-          cur = Group{(uint32_t)di, (uint32_t)di, {}};
-          cur_bytes = 0;
-        }
-      }
-    }
-    if (!cur.spans.empty()) c->groups.push_back(std::move(cur));
-    c->group_ev.assign(c->groups.size(), nullptr);
-    for (auto& e : c->group_ev) CUDA_TRY(c, cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-    CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
-    CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
-    CUDA_TRY(c, cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
-  }
-  if (desc.size() > 0xFFFFFFFFull) {
-    c->err = "too many segments";
-    return SWAP_EUNSUPPORTED;
-  }
-  c->n_desc = (uint32_t)desc.size();
-  const size_t nd = std::max<size_t>(1, desc.size());
-  CUDA_TRY(c, cudaMalloc(&c->d_desc, nd * sizeof(swk::SegDesc)));
-  if (!desc.empty())
-    CUDA_TRY(c, cudaMemcpy(c->d_desc, desc.data(), desc.size() * sizeof(swk::SegDesc), cudaMemcpyHostToDevice));
-  CUDA_TRY(c, cudaMalloc(&c->d_partial, nd * 4));
+  CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+  CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
+  CUDA_TRY(c, cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
   CUDA_TRY(c, cudaMalloc(&c->d_arrive, std::max<uint64_t>(1, P.n_chunks) * 4));
   CUDA_TRY(c, cudaMemset(c->d_arrive, 0, std::max<uint64_t>(1, P.n_chunks) * 4));
+  c->policy.assign(P.regions.size(), SWAP_POLICY_SAVE);
+  st = build_sets(c);
+  if (st != SWAP_OK) return st;
   c->st = St::REGISTERED;
   return SWAP_OK;
 }
@@ -442,18 +518,25 @@ swap_status swap_checkpoint(swap_ctx_t* c, swap_stream_t stream) {
   }
   DeviceGuard g(c->cfg.device);
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-  swk::Params p = base_params(c);
+  // SAVE_ONCE regions are gathered by the first checkpoint only; DISCARD regions never (their image
+  // bytes stay zero and their c_g are the checksums of zero chunks, hashed once from a zero buffer).
+  DescSet& S = c->first_ckpt_done ? c->s_save : c->s_move;
+  swk::Params p = base_params(c, S);
   CUDA_TRY(c, cudaEventRecord(c->ev[0], s));
   swap_status st;
+  if (!c->first_ckpt_done && c->s_zero.n_desc &&
+      (st = launch(c, swk::HASH_STORE, hash_kind(c), base_params(c, c->s_zero), s)) != SWAP_OK)
+    return st;
   if (mech(c) == SWAP_MECH_CE_PIPE) {
-    if ((st = ce_pipe(c, 0, p, s)) != SWAP_OK) return st;
+    if ((st = ce_pipe(c, S, 0, p, s)) != SWAP_OK) return st;
   } else if (is_ce(mech(c))) {
     if ((st = launch(c, swk::HASH_STORE, hash_kind(c), p, s)) != SWAP_OK) return st;
-    if ((st = ce_copy(c, 0, s)) != SWAP_OK) return st;
+    if ((st = ce_copy(c, S, 0, s)) != SWAP_OK) return st;
   } else {
     if ((st = launch(c, swk::GATHER, kind_of(c), p, s)) != SWAP_OK) return st;
   }
   CUDA_TRY(c, cudaEventRecord(c->ev[1], s));
+  c->first_ckpt_done = true;
   c->pending[0] = true;
   c->st = St::CKPT_PENDING;
   return SWAP_OK;
@@ -485,14 +568,19 @@ swap_status swap_restore(swap_ctx_t* c, swap_stream_t stream) {
   if (st != SWAP_OK) return st;
   DeviceGuard g(c->cfg.device);
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-  swk::Params p = base_params(c);
+  DescSet& S = c->s_move;
+  swk::Params p = base_params(c, S);
   CUDA_TRY(c, cudaMemsetAsync(&c->d_status->n_bad, 0, 8, s));
   CUDA_TRY(c, cudaMemsetAsync(&c->d_status->first_bad, 0xFF, 8, s));
   CUDA_TRY(c, cudaEventRecord(c->ev[2], s));
+  for (size_t i = 0; i < c->policy.size(); ++i)  // DISCARD regions come back as zeros
+    if (c->policy[i] == SWAP_POLICY_DISCARD && c->plan.regions[i].r.bytes)
+      CUDA_TRY(c, cudaMemsetAsync(reinterpret_cast<void*>(c->plan.regions[i].r.dev_addr), 0,
+                                  c->plan.regions[i].r.bytes, s));
   if (mech(c) == SWAP_MECH_CE_PIPE) {
-    if ((st = ce_pipe(c, 1, p, s)) != SWAP_OK) return st;
+    if ((st = ce_pipe(c, S, 1, p, s)) != SWAP_OK) return st;
   } else if (is_ce(mech(c))) {
-    if ((st = ce_copy(c, 1, s)) != SWAP_OK) return st;
+    if ((st = ce_copy(c, S, 1, s)) != SWAP_OK) return st;
     if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, s)) != SWAP_OK) return st;
   } else {
     if ((st = launch(c, swk::SCATTER, kind_of(c), p, s)) != SWAP_OK) return st;
@@ -512,7 +600,7 @@ swap_status swap_verify(swap_ctx_t* c, swap_stream_t stream, int hbm_pass, swap_
   DeviceGuard g(c->cfg.device);
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   if (hbm_pass) {
-    swk::Params p = base_params(c);
+    swk::Params p = base_params(c, c->s_all);
     p.n_bad = &c->d_status->hbm_n_bad;
     p.first_bad = &c->d_status->hbm_first_bad;
     CUDA_TRY(c, cudaMemsetAsync(&c->d_status->hbm_n_bad, 0, 8, s));
@@ -541,6 +629,19 @@ swap_status swap_verify(swap_ctx_t* c, swap_stream_t stream, int hbm_pass, swap_
     return SWAP_ECORRUPT;
   }
   return SWAP_OK;
+}
+
+swap_status swap_set_region_policy(swap_ctx_t* c, uint32_t region_index, uint32_t policy) {
+  if (!c || policy > SWAP_POLICY_DISCARD) return SWAP_EINVAL;
+  if (c->st != St::REGISTERED) {
+    c->err = "region policies can only change between swap_register_regions and the first checkpoint";
+    return SWAP_ESTATE;
+  }
+  if (region_index >= c->policy.size()) return SWAP_EINVAL;
+  if (c->policy[region_index] == policy) return SWAP_OK;
+  c->policy[region_index] = policy;
+  DeviceGuard g(c->cfg.device);
+  return build_sets(c);
 }
 
 swap_status swap_set_mechanism(swap_ctx_t* c, uint32_t mechanism) {
@@ -585,6 +686,7 @@ swap_status swap_import(swap_ctx_t* c) {
   swap_status st = swp::check_manifest(c->plan, manifest_ptr(c), &c->err);
   if (st != SWAP_OK) return st;
   c->st = St::CHECKPOINTED;
+  c->first_ckpt_done = true;  // the imported image already holds SAVE_ONCE bytes and DISCARD checksums
   return SWAP_OK;
 }
 

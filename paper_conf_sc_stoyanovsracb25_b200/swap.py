@@ -24,11 +24,13 @@ SWAP_MECH_AUTO, SWAP_MECH_SM, SWAP_MECH_CE_REGION, SWAP_MECH_CE_CHUNK = 0, 1, 2,
 SWAP_MECH_CE_BATCH, SWAP_MECH_CE_PIPE, SWAP_MECH_SM_NOCHECK = 4, 5, 6
 MECHANISMS = {"auto": 0, "sm": 1, "ce_region": 2, "ce_chunk": 3, "ce_batch": 4, "ce_pipe": 5, "sm_nocheck": 6}
 SWAP_KIND_WEIGHTS, SWAP_KIND_KV, SWAP_KIND_WORKSPACE, SWAP_KIND_OTHER = 0, 1, 2, 3
+SWAP_POLICY_SAVE, SWAP_POLICY_SAVE_ONCE, SWAP_POLICY_DISCARD = 0, 1, 2
+POLICIES = {"save": 0, "save_once": 1, "discard": 2}
 U64_MAX = (1 << 64) - 1
 
 EXPORTS = [
     "swap_config_default", "swap_create", "swap_register_regions", "swap_checkpoint", "swap_sync",
-    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_get_manifest", "swap_get_image",
+    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_set_region_policy", "swap_get_manifest", "swap_get_image",
     "swap_get_summary", "swap_import", "swap_set_global", "swap_merge_global", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
     "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
@@ -102,6 +104,7 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_verify": (st, [vp, vp, ctypes.c_int, P(swap_verify_result_t)]),
         "swap_set_mechanism": (st, [vp, u32]),
         "swap_get_mechanism": (st, [vp, P(u32)]),
+        "swap_set_region_policy": (st, [vp, u32, u32]),
         "swap_get_manifest": (st, [vp, P(vp), P(sz)]),
         "swap_get_image": (st, [vp, P(vp), P(sz)]),
         "swap_get_summary": (st, [vp, P(swap_shard_summary_t)]),
@@ -287,6 +290,12 @@ class Swapper:
         if isinstance(mechanism, str):
             mechanism = MECHANISMS[mechanism]
         self._check(load().swap_set_mechanism(self._ctx, mechanism))
+
+    def set_region_policy(self, region_index: int, policy: int | str):
+        """SAVE / SAVE_ONCE / DISCARD for one region (before the first checkpoint)."""
+        if isinstance(policy, str):
+            policy = POLICIES[policy]
+        self._check(load().swap_set_region_policy(self._ctx, region_index, policy))
 
     def mechanism(self) -> str:
         """Name of the mover the next call uses (AUTO resolved)."""
