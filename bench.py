@@ -322,8 +322,9 @@ def run_ours(args):
                           "swapin_GBps": round(payload / (statistics.mean(r2["swapin_ms"]) * 1e-3) / GB, 2)}
         sw.set_mechanism(args.mechanism)
 
-    # swap-in including the HBM release / re-acquire of the VMM arena (outside the timed region)
-    reacq = []
+    # swap-in including the HBM re-acquire of the VMM arena (outside the timed region): explicit
+    # re-acquire then restore, and the bound-arena restore that maps slabs group by group
+    reacq, lazy = [], []
     with torch.cuda.stream(stream):
         for _ in range(2):
             sw.checkpoint(stream, sync=True)
@@ -336,6 +337,17 @@ def run_ours(args):
             h2 = time.perf_counter()
             assert res["status"] == 0
             reacq.append((h1 - h0, h2 - h0))
+        sw.bind_arena(vmm)
+        for _ in range(2):
+            sw.checkpoint(stream, sync=True)
+            vmm.release()
+            h0 = time.perf_counter()
+            sw.restore(stream)
+            res = sw.verify(stream, hbm_pass=True)
+            h1 = time.perf_counter()
+            assert res["status"] == 0 and vmm.resident
+            lazy.append(h1 - h0)
+        sw.bind_arena(None)
 
     # copy-engine link peaks measured here (torch pinned copies, 2 GiB)
     ce = {}
@@ -401,6 +413,7 @@ def run_ours(args):
             "setup_s": {"fill": round(t_fill, 2), "register_pin": round(t_register, 2)},
             "swap_in_with_hbm_reacquire_s": round(statistics.mean(x[1] for x in reacq), 4),
             "hbm_reacquire_s": round(statistics.mean(x[0] for x in reacq), 4),
+            "swap_in_with_overlapped_reacquire_s": round(statistics.mean(lazy), 4),
             "e2e": {"value": round(total_payload / (host_ms * 1e-3) / GB, 3), "unit": "GB/s",
                     "h2d_bytes_per_step": payload, "d2h_bytes_per_step": 32,
                     "how": "host wall clock around swap_restore + swap_verify (C ABI via ctypes), image in pinned host DRAM"},

@@ -230,10 +230,17 @@ typedef struct swap_arena swap_arena_t;
  * ENOMEM if the device cannot back it; EUNSUPPORTED if the driver lacks VMM entry points. */
 SWAP_API swap_status swap_arena_create(int device, uint64_t bytes, swap_arena_t** out);
 SWAP_API swap_status swap_arena_info(const swap_arena_t* a, uint64_t* dev_addr, uint64_t* bytes, int* resident);
-/* Synchronises the device, unmaps and frees all physical memory. ESTATE if already released. */
+/* Synchronises the device, unmaps and frees all mapped physical memory. ESTATE if nothing is mapped. */
 SWAP_API swap_status swap_arena_release(swap_arena_t* a);
 /* Maps new physical memory at the original addresses. ESTATE if resident; ENOMEM if HBM is short. */
 SWAP_API swap_status swap_arena_reacquire(swap_arena_t* a);
+/* Maps only the slabs covering [offset, offset + bytes) (idempotent); the arena is resident once all are. */
+SWAP_API swap_status swap_arena_reacquire_range(swap_arena_t* a, uint64_t offset, uint64_t bytes);
+/* Binds an arena holding (some of) ctx's regions. Then swap_restore re-acquires the arena's HBM
+ * itself if it is released: with SWAP_MECH_CE_PIPE group by group, just before each group's copies are
+ * enqueued, so the host-side mapping overlaps the copy engine; with other movers all at once first.
+ * NULL unbinds. The arena must outlive the binding. */
+SWAP_API swap_status swap_bind_arena(swap_ctx_t* ctx, swap_arena_t* a);
 SWAP_API const char* swap_arena_last_error(const swap_arena_t* a);
 SWAP_API void swap_arena_destroy(swap_arena_t* a);
 

@@ -16,6 +16,7 @@
 #include <vector>
 
 #include "../../include/swap.h"
+#include "arena.h"
 
 namespace {
 
@@ -63,14 +64,22 @@ struct swap_arena {
   CUdeviceptr base = 0;
   uint64_t bytes = 0;  // rounded to the allocation granularity
   uint64_t gran = 0;
-  std::vector<CUmemGenericAllocationHandle> slabs;
-  bool resident = false;
+  std::vector<CUmemGenericAllocationHandle> slabs;  // one per 1-GiB slab; 0 = not mapped
+  uint64_t n_mapped = 0;
+  bool resident = false;  // every slab mapped
   std::string err;
 };
 
 namespace {
 
-swap_status map_all(swap_arena* a) {
+uint64_t n_slabs(const swap_arena* a) { return (a->bytes + kSlab - 1) / kSlab; }
+uint64_t slab_size(const swap_arena* a, uint64_t i) {
+  const uint64_t off = i * kSlab;
+  return a->bytes - off < kSlab ? a->bytes - off : kSlab;
+}
+
+swap_status map_slab(swap_arena* a, uint64_t i) {
+  if (a->slabs[i]) return SWAP_OK;
   const Drv& D = drv();
   CUmemAllocationProp prop;
   std::memset(&prop, 0, sizeof(prop));
@@ -81,39 +90,47 @@ swap_status map_all(swap_arena* a) {
   std::memset(&acc, 0, sizeof(acc));
   acc.location = prop.location;
   acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
-  for (uint64_t off = 0; off < a->bytes; off += kSlab) {
-    const uint64_t sz = a->bytes - off < kSlab ? a->bytes - off : kSlab;
-    CUmemGenericAllocationHandle h;
-    CUresult r = D.create(&h, sz, &prop, 0);
-    if (r != CUDA_SUCCESS) {
-      a->err = "cuMemCreate failed (" + std::to_string((int)r) + ") at offset " + std::to_string(off);
-      return r == CUDA_ERROR_OUT_OF_MEMORY ? SWAP_ENOMEM : SWAP_ECUDA;
-    }
-    if ((r = D.map(a->base + off, sz, 0, h, 0)) != CUDA_SUCCESS) {
-      D.release(h);
-      a->err = "cuMemMap failed (" + std::to_string((int)r) + ")";
-      return SWAP_ECUDA;
-    }
-    a->slabs.push_back(h);
-    if ((r = D.set_access(a->base + off, sz, &acc, 1)) != CUDA_SUCCESS) {
-      a->err = "cuMemSetAccess failed (" + std::to_string((int)r) + ")";
-      return SWAP_ECUDA;
-    }
+  const uint64_t off = i * kSlab, sz = slab_size(a, i);
+  CUmemGenericAllocationHandle h;
+  CUresult r = D.create(&h, sz, &prop, 0);
+  if (r != CUDA_SUCCESS) {
+    a->err = "cuMemCreate failed (" + std::to_string((int)r) + ") at offset " + std::to_string(off);
+    return r == CUDA_ERROR_OUT_OF_MEMORY ? SWAP_ENOMEM : SWAP_ECUDA;
   }
-  a->resident = true;
+  if ((r = D.map(a->base + off, sz, 0, h, 0)) != CUDA_SUCCESS) {
+    D.release(h);
+    a->err = "cuMemMap failed (" + std::to_string((int)r) + ")";
+    return SWAP_ECUDA;
+  }
+  if ((r = D.set_access(a->base + off, sz, &acc, 1)) != CUDA_SUCCESS) {
+    D.unmap(a->base + off, sz);
+    D.release(h);
+    a->err = "cuMemSetAccess failed (" + std::to_string((int)r) + ")";
+    return SWAP_ECUDA;
+  }
+  a->slabs[i] = h;
+  a->resident = ++a->n_mapped == n_slabs(a);
+  return SWAP_OK;
+}
+
+swap_status map_all(swap_arena* a) {
+  for (uint64_t i = 0; i < n_slabs(a); ++i) {
+    swap_status st = map_slab(a, i);
+    if (st != SWAP_OK) return st;
+  }
   return SWAP_OK;
 }
 
 swap_status unmap_all(swap_arena* a) {
   const Drv& D = drv();
   swap_status st = SWAP_OK;
-  for (size_t i = 0; i < a->slabs.size(); ++i) {
-    const uint64_t off = i * kSlab;
-    const uint64_t sz = a->bytes - off < kSlab ? a->bytes - off : kSlab;
-    if (D.unmap(a->base + off, sz) != CUDA_SUCCESS) st = SWAP_ECUDA;
+  for (uint64_t i = 0; i < a->slabs.size(); ++i) {
+    if (!a->slabs[i]) continue;
+    if (D.unmap(a->base + i * kSlab, slab_size(a, i)) != CUDA_SUCCESS) st = SWAP_ECUDA;
     if (D.release(a->slabs[i]) != CUDA_SUCCESS) st = SWAP_ECUDA;
+    a->slabs[i] = 0;
   }
-  a->slabs.clear();
+  a->n_mapped = 0;
   a->resident = false;
   if (st != SWAP_OK) a->err = "cuMemUnmap/cuMemRelease failed";
   return st;
@@ -158,6 +175,7 @@ swap_status swap_arena_create(int device, uint64_t bytes, swap_arena_t** out) {
   }
   a->gran = gran;
   a->bytes = (bytes + gran - 1) / gran * gran;
+  a->slabs.assign(n_slabs(a), 0);
   if (D.reserve(&a->base, a->bytes, kSlab, 0, 0) != CUDA_SUCCESS) {
     delete a;
     return SWAP_ENOMEM;
@@ -183,7 +201,7 @@ swap_status swap_arena_info(const swap_arena_t* a, uint64_t* dev_addr, uint64_t*
 
 swap_status swap_arena_release(swap_arena_t* a) {
   if (!a) return SWAP_EINVAL;
-  if (!a->resident) return SWAP_ESTATE;
+  if (a->n_mapped == 0) return SWAP_ESTATE;
   CtxGuard g(a->device);
   if (cudaDeviceSynchronize() != cudaSuccess) return SWAP_ECUDA;  // no kernel may still touch it
   return unmap_all(a);
@@ -198,6 +216,17 @@ swap_status swap_arena_reacquire(swap_arena_t* a) {
   return st;
 }
 
+swap_status swap_arena_reacquire_range(swap_arena_t* a, uint64_t offset, uint64_t bytes) {
+  if (!a || offset > a->bytes || bytes > a->bytes - offset) return SWAP_EINVAL;
+  if (bytes == 0) return SWAP_OK;
+  CtxGuard g(a->device);
+  for (uint64_t i = offset / kSlab; i <= (offset + bytes - 1) / kSlab; ++i) {
+    swap_status st = map_slab(a, i);
+    if (st != SWAP_OK) return st;
+  }
+  return SWAP_OK;
+}
+
 const char* swap_arena_last_error(const swap_arena_t* a) { return a ? a->err.c_str() : "null arena"; }
 
 void swap_arena_destroy(swap_arena_t* a) {
@@ -205,10 +234,20 @@ void swap_arena_destroy(swap_arena_t* a) {
   {
     CtxGuard g(a->device);
     cudaDeviceSynchronize();
-    if (a->resident) unmap_all(a);
+    unmap_all(a);
     drv().addr_free(a->base, a->bytes);
   }
   delete a;
 }
 
 }  // extern "C"
+
+namespace swarena {
+bool contains(const swap_arena* a, uint64_t lo, uint64_t hi) { return lo >= a->base && hi <= a->base + a->bytes; }
+bool resident(const swap_arena* a) { return a->resident; }
+int device(const swap_arena* a) { return a->device; }
+swap_status map_dev_range(swap_arena* a, uint64_t lo, uint64_t hi) {
+  if (hi <= lo) return SWAP_OK;
+  return swap_arena_reacquire_range(a, lo - a->base, hi - lo);
+}
+}  // namespace swarena

@@ -13,6 +13,7 @@
 #include <string>
 #include <vector>
 
+#include "arena.h"
 #include "kernels.cuh"
 #include "plan.h"
 
@@ -88,6 +89,7 @@ struct swap_ctx {
   std::vector<swap_shard_summary_t> global;
   // CE_PIPE
   cudaStream_t side = nullptr;
+  swap_arena* arena = nullptr;  // bound arena: restore re-acquires its HBM (swap_bind_arena)
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };
 
@@ -207,6 +209,20 @@ swap_status ce_copy(swap_ctx* c, DescSet& S, int dir, cudaStream_t s) {
   return SWAP_OK;
 }
 
+// Re-acquires the bound arena's slabs under `spans` (no-op without an arena or when resident).
+swap_status map_spans(swap_ctx* c, const std::vector<Span>& spans) {
+  if (!c->arena || swarena::resident(c->arena)) return SWAP_OK;
+  for (const Span& sp : spans) {
+    if (!swarena::contains(c->arena, sp.dev, sp.dev + sp.bytes)) continue;
+    swap_status st = swarena::map_dev_range(c->arena, sp.dev, sp.dev + sp.bytes);
+    if (st != SWAP_OK) {
+      c->err = "re-acquiring arena HBM failed";
+      return st;
+    }
+  }
+  return SWAP_OK;
+}
+
 // CE_PIPE. Checkpoint (dir 0): the hash pass over HBM runs on the side stream concurrently with the
 // D2H copies (both only read HBM). Restore (dir 1): group g's H2D copies are followed by an event;
 // the side stream waits for it and checks group g from HBM while the copy engine moves group g+1.
@@ -217,6 +233,7 @@ swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, c
   if (dir == 0 && (st = launch(c, swk::HASH_STORE, hash_kind(c), base, c->side)) != SWAP_OK) return st;
   for (size_t g = 0; g < S.groups.size(); ++g) {
     const Group& G = S.groups[g];
+    if (dir == 1 && (st = map_spans(c, G.spans)) != SWAP_OK) return st;  // lazy HBM re-acquire
     for (const Span& sp : G.spans)
       if ((st = memcpy_dir(c, sp, dir, s)) != SWAP_OK) return st;
     if (dir == 1) {
@@ -573,6 +590,14 @@ swap_status swap_restore(swap_ctx_t* c, swap_stream_t stream) {
   CUDA_TRY(c, cudaMemsetAsync(&c->d_status->n_bad, 0, 8, s));
   CUDA_TRY(c, cudaMemsetAsync(&c->d_status->first_bad, 0xFF, 8, s));
   CUDA_TRY(c, cudaEventRecord(c->ev[2], s));
+  if (c->arena && !swarena::resident(c->arena)) {
+    // DISCARD regions (zero-filled below) and, for movers other than CE_PIPE, everything, need HBM now
+    std::vector<Span> now;
+    for (size_t i = 0; i < c->policy.size(); ++i)
+      if (mech(c) != SWAP_MECH_CE_PIPE || c->policy[i] == SWAP_POLICY_DISCARD)
+        now.push_back(Span{c->plan.regions[i].r.dev_addr, nullptr, c->plan.regions[i].r.bytes});
+    if ((st = map_spans(c, now)) != SWAP_OK) return st;
+  }
   for (size_t i = 0; i < c->policy.size(); ++i)  // DISCARD regions come back as zeros
     if (c->policy[i] == SWAP_POLICY_DISCARD && c->plan.regions[i].r.bytes)
       CUDA_TRY(c, cudaMemsetAsync(reinterpret_cast<void*>(c->plan.regions[i].r.dev_addr), 0,
@@ -642,6 +667,16 @@ swap_status swap_set_region_policy(swap_ctx_t* c, uint32_t region_index, uint32_
   c->policy[region_index] = policy;
   DeviceGuard g(c->cfg.device);
   return build_sets(c);
+}
+
+swap_status swap_bind_arena(swap_ctx_t* c, swap_arena_t* a) {
+  if (!c) return SWAP_EINVAL;
+  if (a && swarena::device(a) != c->cfg.device) {
+    c->err = "arena and ctx are on different devices";
+    return SWAP_EINVAL;
+  }
+  c->arena = a;
+  return SWAP_OK;
 }
 
 swap_status swap_set_mechanism(swap_ctx_t* c, uint32_t mechanism) {

@@ -34,6 +34,7 @@ EXPORTS = [
     "swap_get_summary", "swap_import", "swap_set_global", "swap_merge_global", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
     "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
+    "swap_arena_reacquire_range", "swap_bind_arena",
     "swap_arena_destroy", "swap_sched_create", "swap_sched_add_backend", "swap_sched_touch", "swap_sched_lock",
     "swap_sched_plan", "swap_sched_reserve", "swap_sched_cancel", "swap_sched_grant", "swap_sched_release",
     "swap_sched_query", "swap_sched_free", "swap_sched_destroy",
@@ -120,6 +121,8 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_arena_info": (st, [vp, P(ctypes.c_uint64), P(ctypes.c_uint64), P(ctypes.c_int)]),
         "swap_arena_release": (st, [vp]),
         "swap_arena_reacquire": (st, [vp]),
+        "swap_arena_reacquire_range": (st, [vp, ctypes.c_uint64, ctypes.c_uint64]),
+        "swap_bind_arena": (st, [vp, vp]),
         "swap_arena_last_error": (ctypes.c_char_p, [vp]),
         "swap_arena_destroy": (None, [vp]),
         "swap_sched_create": (st, [u32, P(ctypes.c_uint64), P(vp)]),
@@ -279,9 +282,15 @@ class Swapper:
         if arena is not None:
             arena.release()
 
+    def bind_arena(self, arena: "Arena | None"):
+        """Let restore re-acquire this arena's HBM itself (group by group under CE_PIPE)."""
+        self._check(load().swap_bind_arena(self._ctx, arena._h if arena is not None else None))
+        self._arena = arena
+
     def swap_in(self, arena: "Arena | None" = None, stream=None, hbm_pass: bool = True) -> dict:
-        """Swap-in: re-acquire HBM at the recorded addresses, restore, verify."""
-        if arena is not None:
+        """Swap-in: re-acquire HBM at the recorded addresses, restore, verify. With an
+        arena bound (bind_arena) the re-acquire happens inside the restore, overlapped."""
+        if arena is not None and getattr(self, "_arena", None) is not arena and not arena.resident:
             arena.reacquire()
         self.restore(stream)
         return self.verify(stream, hbm_pass=hbm_pass)
@@ -410,6 +419,9 @@ class Arena:
 
     def release(self):
         self._check(load().swap_arena_release(self._h))
+
+    def reacquire_range(self, offset: int, nbytes: int):
+        self._check(load().swap_arena_reacquire_range(self._h, offset, nbytes))
 
     def reacquire(self):
         self._check(load().swap_arena_reacquire(self._h))

@@ -68,3 +68,34 @@ def test_swap_out_in_through_arena(swp, orc, mech, kind):
             for r, o in zip(specs, offs):
                 assert np.array_equal(back[o:o + r.nbytes], host[o:o + r.nbytes])
     arena.close()
+
+
+@pytest.mark.parametrize("mech", ["ce_pipe", "sm", "ce_region"])
+def test_bound_arena_lazy_reacquire(swp, orc, mech):
+    """With the arena bound to the ctx, restore re-acquires the HBM itself (CE_PIPE: group by group,
+    overlapped with the copies); regions come back bit-exact, DISCARD regions as zeros."""
+    specs = W.scaled(W.config_b(), 3 << 30)  # > 2 slabs of 1 GiB, several pipeline groups
+    offs, total = W.place(specs)
+    arena = swp.Arena(total)
+    base, view = arena.alloc(total)
+    W.fill_device_arena(view, specs, offs, seed=4)
+    host = view.cpu().numpy()
+    regions = [(base + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs, offs))]
+    s = torch.cuda.Stream()
+    with swp.Swapper(regions, mechanism=mech, pipe_mib=64) as sw, torch.cuda.stream(s):
+        kv = [i for i, r in enumerate(specs) if r.kind == W.KIND_KV]
+        for i in kv:
+            sw.set_region_policy(i, "discard")
+        sw.bind_arena(arena)
+        for _ in range(2):
+            sw.swap_out(arena, s)
+            assert not arena.resident
+            res = sw.swap_in(arena, s)
+            assert res["status"] == 0 and res["hbm_n_bad"] == 0
+            assert arena.resident
+            back = arena.tensor(0, total).cpu().numpy()
+            for i, (r, o) in enumerate(zip(specs, offs)):
+                want = np.zeros(r.nbytes, np.uint8) if i in kv else host[o:o + r.nbytes]
+                assert np.array_equal(back[o:o + r.nbytes], want), (i, r.name)
+        sw.bind_arena(None)
+    arena.close()

@@ -54,6 +54,7 @@ with torch.cuda.stream(stream):
             W.fill_device_arena(view, specs, offs, seed=100 * bid + rank)
             regions = [(base + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs, offs))]
             sw = Swapper(regions, mechanism=args.mechanism, device=0, rank=rank, world=len(gpus))
+            sw.bind_arena(arena)  # restore re-acquires HBM group by group, overlapped with the copies
             # snapshot right after initialisation, then park the engine
             sw.swap_out(arena, stream)
             e.shards.append(Shard(g, arena, sw, sum(r.nbytes for r in specs)))
