@@ -186,6 +186,14 @@ SWAP_API swap_status swap_get_manifest(const swap_ctx_t* ctx, const void** bytes
 SWAP_API swap_status swap_get_image(const swap_ctx_t* ctx, void** host, size_t* n);
 SWAP_API swap_status swap_get_summary(const swap_ctx_t* ctx, swap_shard_summary_t* out);
 
+/* Storage tier (NEXT-4): persist a sealed image to a file and load it back. swap_save needs a sealed
+ * checkpoint (ESTATE otherwise) and writes image_bytes bytes (O_DIRECT, several threads; buffered if
+ * the filesystem refuses O_DIRECT). swap_load reads a file of exactly image_bytes bytes into the image
+ * buffer (ECORRUPT if the size differs) and then behaves as swap_import (manifest CRC and layout
+ * checks; state -> CHECKPOINTED). I/O errors return EINVAL (open/read) or ENOMEM (write/space). */
+SWAP_API swap_status swap_save(const swap_ctx_t* ctx, const char* path);
+SWAP_API swap_status swap_load(swap_ctx_t* ctx, const char* path);
+
 /* Declares that the image buffer now holds a complete image (e.g. loaded from storage):
  * checks the manifest CRC and that it describes the registered layout (ECORRUPT if not).
  * Needs REGISTERED, CHECKPOINTED or RESTORED. State -> CHECKPOINTED. */

@@ -75,12 +75,18 @@ void build_tables(uint32_t* tab, uint64_t L1) {
   x2n[0] = 1u << 30;  // x^1
   for (int k = 1; k < 32; ++k) x2n[k] = host_multmodp(x2n[k - 1], x2n[k - 1]);
   for (int l = 0; l < 32; ++l) tab[TAB_LANE + l] = host_x2nmodp(16ull * (31 - l), 3, x2n);
-  // hash kernel: lane l hashes [l*q, min((l+1)*q, L1)); its register is shifted by the bytes after it.
-  const uint64_t q = hash_lane_run(L1);
+  // hash kernel: a lane's register is finally shifted by the bytes after its last piece (common length L1)
   for (int l = 0; l < 32; ++l) {
-    const uint64_t end = std::min<uint64_t>((uint64_t)(l + 1) * q, L1);
-    tab[TAB_HLANE + l] = (uint64_t)l * q < L1 ? host_x2nmodp(L1 - end, 3, x2n) : 0u;
+    const uint64_t end = hash_lane_end(L1, l);
+    tab[TAB_HLANE + l] = end ? host_x2nmodp(L1 - end, 3, x2n) : 0u;
   }
+  // Z^96 (the gap between a lane's consecutive 32-B pieces) of nibble v at nibble position k
+  for (int kk = 0; kk < 8; ++kk)
+    for (uint32_t v = 0; v < 16; ++v) {
+      uint32_t r = v << (4 * kk);
+      for (int z = 0; z < 96; ++z) r = t[r & 0xFFu] ^ (r >> 8);
+      tab[TAB_Z96N + kk * 16 + v] = r;
+    }
 }
 
 // ------------------------------------------------------------------ device helpers
@@ -422,27 +428,38 @@ __global__ void __launch_bounds__(THREADS, 2) mover_kernel(const Params p) {
 
 
 // ------------------------------------------------------------------ HBM hash kernel (CRC-32C)
-// HASH_STORE / HASH_CHECK read device memory only, so lanes need not own 512-B-coalesced slices:
-// lane l hashes the contiguous run [l*q, min((l+1)*q, len)) of its warp's segment with 256-bit
-// loads (one 32-B sector per lane per load) and slicing-by-4 tables replicated once per lane in
-// shared memory (entry (k, e) of lane l at word ((k*256 + e) * 32 + l): bank = lane, conflict-free).
-// The 32 lane registers are folded with x^(8 * bytes-after-run) and an XOR shuffle tree.
+// HASH_STORE / HASH_CHECK read device memory only, so the warp can choose any slicing of its segment.
+// Quad-line layout: the segment is cut into 8 strands, one per lane quad; in each step the 4 lanes of a
+// quad load the 4 sectors of one 128-B line of their strand with 256-bit loads, so a warp-wide load
+// touches 8 lines (8 L1 wavefronts per KiB instead of 32 with one line per lane). A lane's bytes are
+// then 32-B pieces 128 B apart: its register advances with T <- F(Z^96(T), piece) — Z^96 by 8 nibble
+// lookups, F by 8 slicing-by-4 word steps. All tables are replicated once per lane in shared memory
+// (entry e of table k for lane l at word (k*E + e)*32 + l: bank = lane, conflict-free): slicing-by-4
+// 4 x 256 entries (128 KB), Z^96 nibbles 8 x 16 (16 KB). Lanes are folded with x^(8 * bytes after the
+// lane's last piece) and an XOR shuffle tree. Per KiB per warp: 32 + 8 lookup wavefronts + 8 load
+// wavefronts (the r1 contiguous-run layout needed 32 + 32).
 constexpr int HT_THREADS = 1024;
 constexpr int HT_WARPS = HT_THREADS / 32;
-constexpr int HT_U = 4;  // 32-B loads in flight per lane
+constexpr int HT_U = 4;  // lines in flight per lane
 constexpr size_t HT_TAB_WORDS = 4 * 256 * 32;
-constexpr size_t HT_OFF_DESC = HT_TAB_WORDS * 4;
+constexpr size_t HT_Z_WORDS = 8 * 16 * 32;
+constexpr size_t HT_OFF_Z = HT_TAB_WORDS * 4;
+constexpr size_t HT_OFF_DESC = HT_OFF_Z + HT_Z_WORDS * 4;
 constexpr size_t HT_OFF_BAR = HT_OFF_DESC + 2 * HT_WARPS * sizeof(SegDesc);
 constexpr size_t HT_SMEM = HT_OFF_BAR + 16;
 
 __device__ __forceinline__ void ld32(const uint8_t* p, uint32_t (&w)[8]) {
   asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-               : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7])
-               : "l"(p));
+      : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7])
+      : "l"(p));
 }
 __device__ __forceinline__ void ld32_v4x2(const uint8_t* p, uint32_t (&w)[8]) {  // 16-B aligned fallback
   int4 a = __ldg(reinterpret_cast<const int4*>(p)), b = __ldg(reinterpret_cast<const int4*>(p + 16));
   w[0] = a.x; w[1] = a.y; w[2] = a.z; w[3] = a.w; w[4] = b.x; w[5] = b.y; w[6] = b.z; w[7] = b.w;
+}
+template <bool AL32>
+__device__ __forceinline__ void ld32a(const uint8_t* p, uint32_t (&w)[8]) {
+  if (AL32) ld32(p, w); else ld32_v4x2(p, w);
 }
 
 // slicing-by-4 word step on the lane's replicated tables (sT already offset by the lane)
@@ -451,34 +468,43 @@ __device__ __forceinline__ uint32_t crc_word4(uint32_t c, uint32_t w, const uint
   return sT[(3 * 256 + (c & 0xFF)) * 32] ^ sT[(2 * 256 + ((c >> 8) & 0xFF)) * 32] ^
          sT[(1 * 256 + ((c >> 16) & 0xFF)) * 32] ^ sT[(0 * 256 + (c >> 24)) * 32];
 }
-
-template <bool AL32>
-__device__ __forceinline__ void ld32a(const uint8_t* p, uint32_t (&w)[8]) {
-  if (AL32) ld32(p, w); else ld32_v4x2(p, w);
+// Z^96(T) from 8 nibble lookups (sZ already offset by the lane)
+__device__ __forceinline__ uint32_t z96(uint32_t T, const uint32_t* __restrict__ sZ) {
+  uint32_t r = 0;
+#pragma unroll
+  for (int k = 0; k < 8; ++k) r ^= sZ[(k * 16 + ((T >> (4 * k)) & 0xF)) * 32];
+  return r;
 }
 
-// CRC register of one lane's contiguous run [lo, hi) (hi - lo < 2^32), from 0.
+// Register of one lane over its pieces s0, s0+128, ... < send (send = min(strand end, len)).
 template <bool AL32>
-__device__ __forceinline__ uint32_t lane_run_crc(const uint8_t* src, uint64_t lo, uint64_t hi, const uint32_t* myT) {
+__device__ __forceinline__ uint32_t lane_pieces_crc(const uint8_t* src, uint64_t s0, uint64_t send,
+                                                    const uint32_t* myT, const uint32_t* myZ) {
   uint32_t c = 0;
-  uint64_t o = lo;
-  const uint64_t full_end = lo + (hi - lo) / 32 * 32;
-  for (; o + 32 * HT_U <= full_end; o += 32 * HT_U) {
+  uint64_t s = s0;
+  // full pieces, HT_U at a time
+  for (; s + (HT_U - 1) * 128 + 32 <= send; s += HT_U * 128) {
     uint32_t w[HT_U][8];
 #pragma unroll
-    for (int u = 0; u < HT_U; ++u) ld32a<AL32>(src + o + 32 * u, w[u]);
+    for (int u = 0; u < HT_U; ++u) ld32a<AL32>(src + s + 128 * u, w[u]);
 #pragma unroll
-    for (int u = 0; u < HT_U; ++u)
+    for (int u = 0; u < HT_U; ++u) {
+      c = z96(c, myZ);
 #pragma unroll
       for (int j = 0; j < 8; ++j) c = crc_word4(c, w[u][j], myT);
+    }
   }
-  for (; o < full_end; o += 32) {
+  for (; s + 32 <= send; s += 128) {
     uint32_t w[8];
-    ld32a<AL32>(src + o, w);
+    ld32a<AL32>(src + s, w);
+    c = z96(c, myZ);
 #pragma unroll
     for (int j = 0; j < 8; ++j) c = crc_word4(c, w[j], myT);
   }
-  for (; o < hi; ++o) c = myT[((c ^ src[o]) & 0xFFu) * 32] ^ (c >> 8);  // ragged tail, T0 = one byte
+  if (s < send) {  // a partial last piece (only at the end of the segment)
+    c = z96(c, myZ);
+    for (; s < send; ++s) c = myT[((c ^ src[s]) & 0xFFu) * 32] ^ (c >> 8);  // T0 = one byte
+  }
   return c;
 }
 
@@ -486,14 +512,15 @@ template <int MODE>
 __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
   extern __shared__ __align__(128) uint8_t smem[];
   uint32_t* sT = reinterpret_cast<uint32_t*>(smem);
+  uint32_t* sZ = reinterpret_cast<uint32_t*>(smem + HT_OFF_Z);
   SegDesc* sDesc = reinterpret_cast<SegDesc*>(smem + HT_OFF_DESC);
   uint64_t* sBar = reinterpret_cast<uint64_t*>(smem + HT_OFF_BAR);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 
-  // replicate T0..T3 (the first four slicing tables) once per lane
-  for (int i = tid; i < 4 * 256; i += HT_THREADS) {
-    const uint32_t v = __ldg(p.tables + TAB_T16 + i);
-    uint4* dst = reinterpret_cast<uint4*>(sT + (size_t)i * 32);
+  // replicate T0..T3 (the first four slicing tables) and the Z^96 nibble table once per lane
+  for (int i = tid; i < 4 * 256 + 8 * 16; i += HT_THREADS) {
+    const uint32_t v = i < 4 * 256 ? __ldg(p.tables + TAB_T16 + i) : __ldg(p.tables + TAB_Z96N + (i - 4 * 256));
+    uint4* dst = reinterpret_cast<uint4*>(sT + (size_t)i * 32);  // sZ follows sT contiguously
 #pragma unroll
     for (int r = 0; r < 8; ++r) dst[r] = make_uint4(v, v, v, v);
   }
@@ -517,6 +544,7 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
   }
   __syncthreads();
   const uint32_t* myT = sT + lane;
+  const uint32_t* myZ = sZ + lane;
   const uint32_t* x2n = p.tables + TAB_X2N;
 
   for (uint32_t r = 0; r < rounds; ++r) {
@@ -525,17 +553,18 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
     if (idx < p.n_desc) {
       const SegDesc d = sDesc[(r & 1) * HT_WARPS + warp];
       const uint64_t len = d.bytes;
-      const uint64_t q = hash_lane_run(len);
-      const uint64_t lo = (uint64_t)lane * q;
-      const uint64_t hi = lo + q < len ? lo + q : len;
+      const uint64_t Ls = hash_strand(len);
+      const uint64_t q = (uint64_t)(lane >> 2), jj = (uint64_t)(lane & 3);
+      const uint64_t s0 = q * Ls + jj * 32;
+      const uint64_t send = (q + 1) * Ls < len ? (q + 1) * Ls : len;
       const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
       const bool al32 = ((d.dev & 31) == 0);
-      uint32_t c = 0;
-      if (lo < hi) c = al32 ? lane_run_crc<true>(src, lo, hi, myT) : lane_run_crc<false>(src, lo, hi, myT);
-      // fold: X = XOR_l Z^(len - hi_l)(c_l)
       uint32_t X = 0;
-      if (lo < hi) {
-        const uint32_t k = (len == p.hlane_len) ? __ldg(p.tables + TAB_HLANE + lane) : x2nmodp(len - hi, 3, x2n);
+      if (s0 < send) {
+        const uint32_t c = al32 ? lane_pieces_crc<true>(src, s0, send, myT, myZ)
+                                : lane_pieces_crc<false>(src, s0, send, myT, myZ);
+        const uint32_t k = (len == p.hlane_len) ? __ldg(p.tables + TAB_HLANE + lane)
+                                                : x2nmodp(len - hash_lane_end(len, lane), 3, x2n);
         X = multmodp(k, c);
       }
 #pragma unroll
@@ -730,7 +759,7 @@ static cudaError_t launch_xxh_ring(const Params& p, int sm_count, cudaStream_t s
 // sector), XK_U stripes in flight. Used for HASH_STORE / HASH_CHECK when there are enough chunks
 // to occupy the GPU (hash_xxh_lane_ok); otherwise the warp-per-chunk mover handles it.
 constexpr int XK_THREADS = 256;
-constexpr int XK_U = 4;
+constexpr int XK_U = 4;  // 128 B in flight per lane (U = 8 with 2 CTAs/SM measured slower: 2.7 vs 3.6 TB/s)
 constexpr size_t XK_OFF_BAR = 2 * XK_THREADS * sizeof(SegDesc);
 constexpr size_t XK_SMEM = XK_OFF_BAR + 16;
 

@@ -40,7 +40,8 @@ constexpr int TAB_Z496 = 16 * 256;  // [4][256]  Z^496 applied to byte j of a re
 constexpr int TAB_LANE = TAB_Z496 + 4 * 256;  // [32] x^(8*16*(31-l)) mod P
 constexpr int TAB_X2N = TAB_LANE + 32;        // [32] x^(2^k) mod P
 constexpr int TAB_HLANE = TAB_X2N + 32;       // [32] hash kernel: Z^(L1 - end_l) for the common segment length L1
-constexpr int TAB_WORDS = TAB_HLANE + 32;
+constexpr int TAB_Z96N = TAB_HLANE + 32;       // [8][16] hash kernel: Z^96 of nibble v at position k
+constexpr int TAB_WORDS = TAB_Z96N + 128;
 constexpr int TAB_SMEM_WORDS = TAB_LANE + 32;  // the part staged in shared memory
 
 struct Params {
@@ -61,8 +62,19 @@ struct Params {
 };
 
 void build_tables(uint32_t* tab /* TAB_WORDS */, uint64_t common_seg_len);
-// Per-lane run length of the HBM hash kernel for a segment of `len` bytes (multiple of 32).
-__host__ __device__ inline uint64_t hash_lane_run(uint64_t len) { return ((len + 31) / 32 + 31) / 32 * 32; }
+// Quad-line geometry of the CRC-32C HBM hash kernel for a segment of `len` bytes: 8 strands (one per
+// lane quad) of hash_strand(len) bytes (a multiple of 128); lane (q = lane/4, j = lane%4) owns the 32-B
+// pieces at q*Ls + j*32 + t*128 that start inside its strand and the segment.
+__host__ __device__ inline uint64_t hash_strand(uint64_t len) { return ((len + 7) / 8 + 127) / 128 * 128; }
+// One past the lane's last byte (0 if the lane owns none).
+__host__ __device__ inline uint64_t hash_lane_end(uint64_t len, int lane) {
+  const uint64_t Ls = hash_strand(len), q = (uint64_t)(lane >> 2), j = (uint64_t)(lane & 3);
+  const uint64_t s0 = q * Ls + j * 32;
+  const uint64_t strand_end = (q + 1) * Ls < len ? (q + 1) * Ls : len;
+  if (s0 >= strand_end) return 0;
+  const uint64_t last = s0 + (strand_end - 1 - s0) / 128 * 128;
+  return last + 32 < strand_end ? last + 32 : strand_end;
+}
 uint32_t host_x2nmodp(uint64_t n, unsigned k, const uint32_t* x2n);
 uint32_t host_multmodp(uint32_t a, uint32_t b);
 

@@ -31,7 +31,7 @@ U64_MAX = (1 << 64) - 1
 EXPORTS = [
     "swap_config_default", "swap_create", "swap_register_regions", "swap_checkpoint", "swap_sync",
     "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_set_region_policy", "swap_get_manifest", "swap_get_image",
-    "swap_get_summary", "swap_import", "swap_set_global", "swap_merge_global", "swap_get_timings",
+    "swap_get_summary", "swap_import", "swap_save", "swap_load", "swap_set_global", "swap_merge_global", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
     "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
     "swap_arena_reacquire_range", "swap_bind_arena",
@@ -110,6 +110,8 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_get_image": (st, [vp, P(vp), P(sz)]),
         "swap_get_summary": (st, [vp, P(swap_shard_summary_t)]),
         "swap_import": (st, [vp]),
+        "swap_save": (st, [vp, ctypes.c_char_p]),
+        "swap_load": (st, [vp, ctypes.c_char_p]),
         "swap_set_global": (st, [vp, P(swap_shard_summary_t), ctypes.c_int, P(ctypes.c_uint64)]),
         "swap_merge_global": (st, [P(swap_shard_summary_t), ctypes.c_int, P(ctypes.c_uint64)]),
         "swap_get_timings": (st, [vp, P(swap_timings_t)]),
@@ -311,6 +313,14 @@ class Swapper:
         m = ctypes.c_uint32()
         self._check(load().swap_get_mechanism(self._ctx, ctypes.byref(m)))
         return {v: k for k, v in MECHANISMS.items()}[m.value]
+
+    def save(self, path: str):
+        """Persist the sealed image to `path` (swap_save)."""
+        self._check(load().swap_save(self._ctx, os.fsencode(path)))
+
+    def load_image(self, path: str):
+        """Load an image file written by save() and validate it (swap_load)."""
+        self._check(load().swap_load(self._ctx, os.fsencode(path)))
 
     def import_image(self):
         self._check(load().swap_import(self._ctx))

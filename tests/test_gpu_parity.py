@@ -47,7 +47,7 @@ def oracle_image(orc, key, or_regions, host, base, kind, C):
 
 def roundtrip(swp, orc, stream, specs, seed, C, kind, mech, key=None, **kw):
     arena, host, base, offs, sw_regions, or_regions = device_case(specs, seed)
-    img_ref, moff = oracle_image(orc, key or (id(specs), seed, C, kind), or_regions, host, base, kind, C)
+    img_ref, moff = oracle_image(orc, (key or (id(specs), seed, C, kind)) + (base,), or_regions, host, base, kind, C)
     sw = swp.Swapper(sw_regions, chunk_bytes=C, checksum=kind, mechanism=mech, **kw)
     try:
         with torch.cuda.stream(stream):
