@@ -69,6 +69,34 @@ def parse():
     return ap.parse_args()
 
 
+def host_mem_available() -> int:
+    try:
+        with open("/proc/meminfo") as f:
+            for line in f:
+                if line.startswith("MemAvailable:"):
+                    return int(line.split()[1]) * 1024
+    except OSError:
+        pass
+    return 0
+
+
+def fit_host(specs, local_ranks: int):
+    """Every rank pins an image as large as its payload. If the node's free RAM cannot hold all local
+    ranks' images (with 20 % headroom), shrink the KV-pool regions uniformly and say so; weights and
+    workspace keep their shapes. Returns (specs, kv_scale)."""
+    avail = host_mem_available()
+    need = sum(r.nbytes for r in specs) * local_ranks
+    if not avail or need <= 0.8 * avail:
+        return specs, 1.0
+    kv = sum(r.nbytes for r in specs if r.kind == W.KIND_KV)
+    other = sum(r.nbytes for r in specs) - kv
+    budget = 0.8 * avail / local_ranks - other
+    scale = max(0.05, budget / kv) if kv else 1.0
+    out = [W.RegionSpec(r.name, r.kind, int(r.nbytes * scale) // 4096 * 4096, r.dtype) if r.kind == W.KIND_KV else r
+           for r in specs]
+    return out, round(scale, 4)
+
+
 def workload(cfg: str, rank: int, world: int):
     if cfg == "auto":
         cfg = "B" if world == 1 else "D"
@@ -234,6 +262,7 @@ def run_ours(args):
         return float(t.item())
 
     name, specs, desc = workload(args.config, rank, world)
+    specs, kv_scale = fit_host(specs, int(os.environ.get("LOCAL_WORLD_SIZE", "1")))
     offs, arena_bytes = W.place(specs)
     payload = sum(r.nbytes for r in specs)
     t0 = time.perf_counter()
@@ -390,7 +419,8 @@ def run_ours(args):
             "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": round(step_ms, 3), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "u8", "data": "synthetic",
-            "config": {"workload": f"{name}: {desc}", "regions_per_rank": len(specs),
+            "config": {"workload": f"{name}: {desc}" + ("" if kv_scale == 1.0 else f" (KV pool scaled x{kv_scale} to fit host RAM)"),
+                       "regions_per_rank": len(specs),
                        "payload_bytes_per_rank": payload, "chunk_bytes": args.chunk, "checksum": args.checksum,
                        "mechanism": f"{args.mechanism} -> {eff_mech}",
                        "l2": "no flush: every step moves the whole image (>> 126 MB L2)",

@@ -480,7 +480,7 @@ swap_status swap_register_regions(swap_ctx_t* c, const swap_region_t* regions, s
   swp::Plan plan;
   swap_status st = swp::build_plan(regions, n, c->cfg, &plan, &c->err);
   if (st != SWAP_OK) return st;
-  if (c->st != St::CREATED) {
+  if (c->st != St::CREATED || c->image) {  // registered, or a failed registration left its image
     c->err = "regions already registered";
     return SWAP_ESTATE;
   }
