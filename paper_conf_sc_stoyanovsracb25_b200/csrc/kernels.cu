@@ -441,12 +441,15 @@ __global__ void __launch_bounds__(THREADS, 2) mover_kernel(const Params p) {
 constexpr int HT_THREADS = 1024;
 constexpr int HT_WARPS = HT_THREADS / 32;
 constexpr int HT_U = 4;  // lines in flight per lane
-constexpr size_t HT_TAB_WORDS = 4 * 256 * 32;
-constexpr size_t HT_Z_WORDS = 8 * 16 * 32;
-constexpr size_t HT_OFF_Z = HT_TAB_WORDS * 4;
-constexpr size_t HT_OFF_DESC = HT_OFF_Z + HT_Z_WORDS * 4;
-constexpr size_t HT_OFF_BAR = HT_OFF_DESC + 2 * HT_WARPS * sizeof(SegDesc);
-constexpr size_t HT_SMEM = HT_OFF_BAR + 16;
+// Shared layout (offsets from a 32-KiB-aligned base B inside the dynamic allocation): slicing table k at
+// B + k*32 KiB, entry e of lane l at + e*128 + l*4; Z^96 nibble table k at B + 128 KiB + k*2 KiB. With
+// B 32-KiB aligned, a lookup address is (index << 7) | (B + 4*lane) plus an immediate table offset: one
+// shift + one LOP3 per lookup.
+constexpr uint32_t HT_TAB_BYTES = 4 * 256 * 128;
+constexpr uint32_t HT_Z_BYTES = 8 * 16 * 128;
+constexpr uint32_t HT_OFF_DESC = HT_TAB_BYTES + HT_Z_BYTES;
+constexpr uint32_t HT_OFF_BAR = HT_OFF_DESC + 2 * HT_WARPS * sizeof(SegDesc);
+constexpr size_t HT_SMEM = 32768 + HT_OFF_BAR + 16;  // + worst-case alignment padding
 
 __device__ __forceinline__ void ld32(const uint8_t* p, uint32_t (&w)[8]) {
   asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
@@ -462,24 +465,36 @@ __device__ __forceinline__ void ld32a(const uint8_t* p, uint32_t (&w)[8]) {
   if (AL32) ld32(p, w); else ld32_v4x2(p, w);
 }
 
-// slicing-by-4 word step on the lane's replicated tables (sT already offset by the lane)
-__device__ __forceinline__ uint32_t crc_word4(uint32_t c, uint32_t w, const uint32_t* __restrict__ sT) {
-  c ^= w;
-  return sT[(3 * 256 + (c & 0xFF)) * 32] ^ sT[(2 * 256 + ((c >> 8) & 0xFF)) * 32] ^
-         sT[(1 * 256 + ((c >> 16) & 0xFF)) * 32] ^ sT[(0 * 256 + (c >> 24)) * 32];
+__device__ __forceinline__ uint32_t lds_at(uint32_t addr) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+  return v;
 }
-// Z^96(T) from 8 nibble lookups (sZ already offset by the lane)
-__device__ __forceinline__ uint32_t z96(uint32_t T, const uint32_t* __restrict__ sZ) {
-  uint32_t r = 0;
-#pragma unroll
-  for (int k = 0; k < 8; ++k) r ^= sZ[(k * 16 + ((T >> (4 * k)) & 0xF)) * 32];
-  return r;
+template <uint32_t OFF>
+__device__ __forceinline__ uint32_t lds_off(uint32_t addr) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1+%2];" : "=r"(v) : "r"(addr), "n"(OFF));
+  return v;
+}
+
+// slicing-by-4 word step; lb = B + 4*lane (B 32-KiB aligned): table k entry e at lb + k*32K + e*128
+__device__ __forceinline__ uint32_t crc_word4(uint32_t c, uint32_t w, uint32_t lb) {
+  c ^= w;
+  return lds_off<3 * 32768>(((c << 7) & 0x7F80u) | lb) ^ lds_off<2 * 32768>(((c >> 1) & 0x7F80u) | lb) ^
+         lds_off<1 * 32768>(((c >> 9) & 0x7F80u) | lb) ^ lds_off<0>(((c >> 17) & 0x7F80u) | lb);
+}
+// Z^96(T) from 8 nibble lookups; lz = B + 128K + 4*lane: nibble table k entry v at lz + k*2K + v*128
+__device__ __forceinline__ uint32_t z96(uint32_t T, uint32_t lz) {
+  return lds_off<0 * 2048>(((T << 7) & 0x780u) | lz) ^ lds_off<1 * 2048>(((T << 3) & 0x780u) | lz) ^
+         lds_off<2 * 2048>(((T >> 1) & 0x780u) | lz) ^ lds_off<3 * 2048>(((T >> 5) & 0x780u) | lz) ^
+         lds_off<4 * 2048>(((T >> 9) & 0x780u) | lz) ^ lds_off<5 * 2048>(((T >> 13) & 0x780u) | lz) ^
+         lds_off<6 * 2048>(((T >> 17) & 0x780u) | lz) ^ lds_off<7 * 2048>(((T >> 21) & 0x780u) | lz);
 }
 
 // Register of one lane over its pieces s0, s0+128, ... < send (send = min(strand end, len)).
 template <bool AL32>
-__device__ __forceinline__ uint32_t lane_pieces_crc(const uint8_t* src, uint64_t s0, uint64_t send,
-                                                    const uint32_t* myT, const uint32_t* myZ) {
+__device__ __forceinline__ uint32_t lane_pieces_crc(const uint8_t* src, uint64_t s0, uint64_t send, uint32_t lb,
+                                                    uint32_t lz) {
   uint32_t c = 0;
   uint64_t s = s0;
   // full pieces, HT_U at a time
@@ -489,30 +504,32 @@ __device__ __forceinline__ uint32_t lane_pieces_crc(const uint8_t* src, uint64_t
     for (int u = 0; u < HT_U; ++u) ld32a<AL32>(src + s + 128 * u, w[u]);
 #pragma unroll
     for (int u = 0; u < HT_U; ++u) {
-      c = z96(c, myZ);
+      c = z96(c, lz);
 #pragma unroll
-      for (int j = 0; j < 8; ++j) c = crc_word4(c, w[u][j], myT);
+      for (int j = 0; j < 8; ++j) c = crc_word4(c, w[u][j], lb);
     }
   }
   for (; s + 32 <= send; s += 128) {
     uint32_t w[8];
     ld32a<AL32>(src + s, w);
-    c = z96(c, myZ);
+    c = z96(c, lz);
 #pragma unroll
-    for (int j = 0; j < 8; ++j) c = crc_word4(c, w[j], myT);
+    for (int j = 0; j < 8; ++j) c = crc_word4(c, w[j], lb);
   }
   if (s < send) {  // a partial last piece (only at the end of the segment)
-    c = z96(c, myZ);
-    for (; s < send; ++s) c = myT[((c ^ src[s]) & 0xFFu) * 32] ^ (c >> 8);  // T0 = one byte
+    c = z96(c, lz);
+    for (; s < send; ++s) c = lds_at((((c ^ src[s]) & 0xFFu) << 7) | lb) ^ (c >> 8);  // table 0 = one byte
   }
   return c;
 }
 
 template <int MODE>
 __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
-  extern __shared__ __align__(128) uint8_t smem[];
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  const uint32_t B = (raw + 32767u) & ~32767u;  // 32-KiB aligned table base (shared address)
+  uint8_t* smem = smem_raw + (B - raw);
   uint32_t* sT = reinterpret_cast<uint32_t*>(smem);
-  uint32_t* sZ = reinterpret_cast<uint32_t*>(smem + HT_OFF_Z);
   SegDesc* sDesc = reinterpret_cast<SegDesc*>(smem + HT_OFF_DESC);
   uint64_t* sBar = reinterpret_cast<uint64_t*>(smem + HT_OFF_BAR);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -520,7 +537,7 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
   // replicate T0..T3 (the first four slicing tables) and the Z^96 nibble table once per lane
   for (int i = tid; i < 4 * 256 + 8 * 16; i += HT_THREADS) {
     const uint32_t v = i < 4 * 256 ? __ldg(p.tables + TAB_T16 + i) : __ldg(p.tables + TAB_Z96N + (i - 4 * 256));
-    uint4* dst = reinterpret_cast<uint4*>(sT + (size_t)i * 32);  // sZ follows sT contiguously
+    uint4* dst = reinterpret_cast<uint4*>(sT + (size_t)i * 32);  // the Z table follows the slicing tables
 #pragma unroll
     for (int r = 0; r < 8; ++r) dst[r] = make_uint4(v, v, v, v);
   }
@@ -543,8 +560,7 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
     if (rounds > 1) issue(1);
   }
   __syncthreads();
-  const uint32_t* myT = sT + lane;
-  const uint32_t* myZ = sZ + lane;
+  const uint32_t lb = B + 4u * lane, lz = B + HT_TAB_BYTES + 4u * lane;
   const uint32_t* x2n = p.tables + TAB_X2N;
 
   for (uint32_t r = 0; r < rounds; ++r) {
@@ -561,8 +577,8 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
       const bool al32 = ((d.dev & 31) == 0);
       uint32_t X = 0;
       if (s0 < send) {
-        const uint32_t c = al32 ? lane_pieces_crc<true>(src, s0, send, myT, myZ)
-                                : lane_pieces_crc<false>(src, s0, send, myT, myZ);
+        const uint32_t c = al32 ? lane_pieces_crc<true>(src, s0, send, lb, lz)
+                                : lane_pieces_crc<false>(src, s0, send, lb, lz);
         const uint32_t k = (len == p.hlane_len) ? __ldg(p.tables + TAB_HLANE + lane)
                                                 : x2nmodp(len - hash_lane_end(len, lane), 3, x2n);
         X = multmodp(k, c);
