@@ -18,6 +18,8 @@
 //    lanes with shuffles, the tail and finalisation run on lane 0.
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
+#include <cstring>
 
 #include "kernels.cuh"
 
@@ -890,6 +892,7 @@ static cudaError_t launch_xxh_lane(const Params& p, int sm_count, cudaStream_t s
   return cudaGetLastError();
 }
 
+
 // Many chunks: one lane per chunk keeps all 32 lanes issuing rounds (5+ TB/s measured); few
 // (large) chunks: the TMA ring keeps the memory pipe full with one warp per chunk.
 bool hash_xxh_lane_ok(int sm_count, uint32_t n_desc) { return n_desc >= (uint32_t)sm_count * 192u; }
@@ -915,9 +918,22 @@ static cudaError_t launch_t(const Params& p, int grid, cudaStream_t s) {
   return cudaGetLastError();
 }
 
+// Kernel choice for XXH64 hash passes: 0 = automatic, 1 = lane per chunk, 3 = TMA ring
+// (SWAP_XXH_KERNEL=lane|ring forces one, for measurements and tests).
+static int xxh_variant() {
+  static int v = [] {
+    const char* e = getenv("SWAP_XXH_KERNEL");
+    if (!e) return 0;
+    if (!strcmp(e, "lane")) return 1;
+    if (!strcmp(e, "ring")) return 3;
+    return 0;
+  }();
+  return v;
+}
+
 cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_t s) {
   if (p.n_desc == 0) return cudaSuccess;
-  if (hash_xxh_lane_ok(sm_count, p.n_desc))
+  if (xxh_variant() == 1 || (xxh_variant() == 0 && hash_xxh_lane_ok(sm_count, p.n_desc)))
     return mode == HASH_STORE ? launch_xxh_lane<HASH_STORE>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK>(p, sm_count, s);
   return mode == HASH_STORE ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
 }
