@@ -204,6 +204,17 @@ SWAP_API swap_status swap_import(swap_ctx_t* ctx);
  * global manifest and writes the global digest (CRC-32C of the world*64 bytes). */
 SWAP_API swap_status swap_set_global(swap_ctx_t* ctx, const swap_shard_summary_t* all, int world, uint64_t* global_digest);
 
+/* Ctx-free host planning (needs no GPU): the layout and the sealed manifest libswap produces for a
+ * region table under cfg (same validation as swap_register_regions). swap_plan_manifest writes the
+ * manifest (header, region and chunk records with the given chunk checksums, CRC trailer) into out
+ * (cap >= manifest bytes, else EINVAL with *manifest_bytes set). chunk_checksums may be NULL (zeros). */
+SWAP_API swap_status swap_plan_layout(const swap_region_t* regions, size_t n, const swap_config_t* cfg,
+                                      uint64_t* payload_bytes, uint64_t* n_chunks, uint64_t* manifest_off,
+                                      uint64_t* image_bytes);
+SWAP_API swap_status swap_plan_manifest(const swap_region_t* regions, size_t n, const swap_config_t* cfg,
+                                        const uint64_t* chunk_checksums, void* out, size_t cap,
+                                        size_t* manifest_bytes);
+
 /* Ctx-free half of swap_set_global, usable without a GPU: checks that `all` holds `world`
  * summaries with all[r].rank == r and all[r].world == world (ENCCL otherwise) and writes
  * the global digest = CRC-32C of the world*64 summary bytes. */

@@ -725,6 +725,43 @@ swap_status swap_import(swap_ctx_t* c) {
   return SWAP_OK;
 }
 
+swap_status swap_plan_layout(const swap_region_t* regions, size_t n, const swap_config_t* cfg_in, uint64_t* payload,
+                             uint64_t* n_chunks, uint64_t* manifest_off, uint64_t* image_bytes) {
+  if (!cfg_in) return SWAP_EINVAL;
+  swap_config_t cfg = *cfg_in;
+  std::string err;
+  swap_status st = swp::normalize_config(&cfg, &err);
+  if (st != SWAP_OK) return st;
+  swp::Plan P;
+  if ((st = swp::build_plan(regions, n, cfg, &P, &err)) != SWAP_OK) return st;
+  if (payload) *payload = P.payload_bytes;
+  if (n_chunks) *n_chunks = P.n_chunks;
+  if (manifest_off) *manifest_off = P.manifest_off;
+  if (image_bytes) *image_bytes = P.image_bytes;
+  return SWAP_OK;
+}
+
+swap_status swap_plan_manifest(const swap_region_t* regions, size_t n, const swap_config_t* cfg_in,
+                               const uint64_t* cs, void* out, size_t cap, size_t* manifest_bytes) {
+  if (!cfg_in || !manifest_bytes) return SWAP_EINVAL;
+  swap_config_t cfg = *cfg_in;
+  std::string err;
+  swap_status st = swp::normalize_config(&cfg, &err);
+  if (st != SWAP_OK) return st;
+  swp::Plan P;
+  if ((st = swp::build_plan(regions, n, cfg, &P, &err)) != SWAP_OK) return st;
+  *manifest_bytes = P.manifest_bytes;
+  if (!out || cap < P.manifest_bytes) return SWAP_EINVAL;
+  uint8_t* man = static_cast<uint8_t*>(out);
+  swp::write_manifest_skeleton(P, man);
+  if (cs) {
+    uint8_t* cr = man + swp::kHeaderBytes + swp::kRegionRecBytes * P.regions.size();
+    for (uint64_t g = 0; g < P.n_chunks; ++g) std::memcpy(cr + swp::kChunkRecBytes * g + 24, cs + g, 8);
+  }
+  swp::seal_manifest(P, man);
+  return SWAP_OK;
+}
+
 swap_status swap_merge_global(const swap_shard_summary_t* all, int world, uint64_t* digest) {
   if (!all || world < 1) return SWAP_EINVAL;
   for (int r = 0; r < world; ++r)

@@ -31,7 +31,7 @@ U64_MAX = (1 << 64) - 1
 EXPORTS = [
     "swap_config_default", "swap_create", "swap_register_regions", "swap_checkpoint", "swap_sync",
     "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_set_region_policy", "swap_get_manifest", "swap_get_image",
-    "swap_get_summary", "swap_import", "swap_save", "swap_load", "swap_set_global", "swap_merge_global", "swap_get_timings",
+    "swap_get_summary", "swap_import", "swap_save", "swap_load", "swap_set_global", "swap_merge_global", "swap_plan_layout", "swap_plan_manifest", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
     "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
     "swap_arena_reacquire_range", "swap_bind_arena",
@@ -114,6 +114,9 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_load": (st, [vp, ctypes.c_char_p]),
         "swap_set_global": (st, [vp, P(swap_shard_summary_t), ctypes.c_int, P(ctypes.c_uint64)]),
         "swap_merge_global": (st, [P(swap_shard_summary_t), ctypes.c_int, P(ctypes.c_uint64)]),
+        "swap_plan_layout": (st, [P(swap_region_t), sz, P(swap_config_t), P(ctypes.c_uint64), P(ctypes.c_uint64),
+                                  P(ctypes.c_uint64), P(ctypes.c_uint64)]),
+        "swap_plan_manifest": (st, [P(swap_region_t), sz, P(swap_config_t), P(ctypes.c_uint64), vp, sz, P(sz)]),
         "swap_get_timings": (st, [vp, P(swap_timings_t)]),
         "swap_get_launch_count": (st, [vp, P(ctypes.c_uint64)]),
         "swap_status_str": (ctypes.c_char_p, [st]),
@@ -197,6 +200,33 @@ def swap_merge_global(summaries: bytes, world: int):
     d = ctypes.c_uint64()
     st = load().swap_merge_global(arr, world, ctypes.byref(d))
     return st, d.value
+
+
+def _region_array(regions):
+    arr = (swap_region_t * max(1, len(regions)))()
+    for i, (addr, nb, rid, kind) in enumerate(regions):
+        arr[i].dev_addr, arr[i].bytes, arr[i].id, arr[i].kind = addr, nb, rid, kind
+    return arr
+
+
+def swap_plan_layout(regions, cfg: swap_config_t):
+    """(status, payload_bytes, n_chunks, manifest_off, image_bytes) for (dev_addr, nbytes, id, kind) rows."""
+    vals = [ctypes.c_uint64() for _ in range(4)]
+    st = load().swap_plan_layout(_region_array(regions), len(regions), ctypes.byref(cfg), *[ctypes.byref(v) for v in vals])
+    return (st, *[v.value for v in vals])
+
+
+def swap_plan_manifest(regions, cfg: swap_config_t, checksums=None):
+    """(status, manifest bytes) with the given chunk checksums (list of ints) or zeros."""
+    st, payload, m, moff, ib = swap_plan_layout(regions, cfg)
+    if st:
+        return st, b""
+    cs = (ctypes.c_uint64 * max(1, m))(*(checksums or []))
+    n = ctypes.c_size_t()
+    buf = ctypes.create_string_buffer(ib - moff)
+    st = load().swap_plan_manifest(_region_array(regions), len(regions), ctypes.byref(cfg),
+                                   cs if checksums is not None else None, buf, len(buf), ctypes.byref(n))
+    return st, buf.raw[:n.value]
 
 
 def _torch_stream(stream) -> int:
