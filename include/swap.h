@@ -260,6 +260,19 @@ SWAP_API swap_status swap_arena_reacquire_range(swap_arena_t* a, uint64_t offset
  * enqueued, so the host-side mapping overlaps the copy engine; with other movers all at once first.
  * NULL unbinds. The arena must outlive the binding. */
 SWAP_API swap_status swap_bind_arena(swap_ctx_t* ctx, swap_arena_t* a);
+
+/* Full-duplex exchange on one device (NEXT-1; §3.4-3.5 swap-out of victims then swap-in of the
+ * requested backend, here overlapped on the duplex PCIe link): checkpoints + seals + releases every victim
+ * (each with a bound, mapped arena) on s_out while scattering `incoming` (bound, released arena; sealed
+ * image) on s_in. Incoming HBM is mapped slab by slab just before each pipeline group, and only while
+ * (victim HBM still mapped + incoming HBM mapped) <= (victim HBM at the start + headroom): victim slabs are
+ * released as soon as the last group reading them has left the device. Either side may be empty
+ * (nv == 0 or incoming == NULL). Victims end CHECKPOINTED, incoming RESTORED (call swap_verify on it).
+ * *peak_extra (optional) = the most HBM held above the victims' starting amount (<= headroom). ENOMEM if
+ * the incoming arena cannot fit. The device is synchronised first; calls on the ctxs are serialised. */
+SWAP_API swap_status swap_exchange(swap_ctx_t* const* victims, size_t n_victims, swap_ctx_t* incoming,
+                                   swap_stream_t s_out, swap_stream_t s_in, uint64_t headroom,
+                                   uint64_t* peak_extra);
 SWAP_API const char* swap_arena_last_error(const swap_arena_t* a);
 SWAP_API void swap_arena_destroy(swap_arena_t* a);
 

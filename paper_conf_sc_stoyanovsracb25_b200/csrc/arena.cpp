@@ -243,6 +243,27 @@ void swap_arena_destroy(swap_arena_t* a) {
 }  // extern "C"
 
 namespace swarena {
+uint64_t slab_bytes() { return kSlab; }
+uint64_t n_slabs(const swap_arena* a) { return ::n_slabs(a); }
+uint64_t slab_size(const swap_arena* a, uint64_t i) { return ::slab_size(a, i); }
+bool slab_mapped(const swap_arena* a, uint64_t i) { return a->slabs[i] != 0; }
+uint64_t mapped_bytes(const swap_arena* a) {
+  uint64_t b = 0;
+  for (uint64_t i = 0; i < a->slabs.size(); ++i)
+    if (a->slabs[i]) b += ::slab_size(a, i);
+  return b;
+}
+uint64_t slab_of(const swap_arena* a, uint64_t dev) { return (dev - a->base) / kSlab; }
+swap_status map_slab(swap_arena* a, uint64_t i) { return ::map_slab(a, i); }
+swap_status unmap_slab(swap_arena* a, uint64_t i) {  // caller guarantees no pending device work uses it
+  if (!a->slabs[i]) return SWAP_OK;
+  const Drv& D = drv();
+  const bool ok = D.unmap(a->base + i * kSlab, ::slab_size(a, i)) == CUDA_SUCCESS && D.release(a->slabs[i]) == CUDA_SUCCESS;
+  a->slabs[i] = 0;
+  --a->n_mapped;
+  a->resident = false;
+  return ok ? SWAP_OK : SWAP_ECUDA;
+}
 bool contains(const swap_arena* a, uint64_t lo, uint64_t hi) { return lo >= a->base && hi <= a->base + a->bytes; }
 bool resident(const swap_arena* a) { return a->resident; }
 int device(const swap_arena* a) { return a->device; }

@@ -16,7 +16,7 @@ from __future__ import annotations
 import time
 from dataclasses import dataclass, field
 
-from .swap import Arena, Scheduler, Swapper
+from .swap import Arena, Scheduler, Swapper, exchange
 
 
 @dataclass
@@ -45,11 +45,13 @@ class Engine:
 class HotSwapController:
     """Serves swap-in requests for a fixed set of engines under per-GPU memory budgets."""
 
-    def __init__(self, engines: list, budget_per_gpu: list, stream=None):
+    def __init__(self, engines: list, budget_per_gpu: list, stream=None, duplex: bool = False, stream_in=None):
         self.engines = {e.bid: e for e in engines}
         self.n_gpus = len(budget_per_gpu)
         self.sched = Scheduler(budget_per_gpu)
         self.stream = stream
+        self.duplex = duplex  # overlap victims' swap-out with the swap-in (swap_exchange), per GPU
+        self.stream_in = stream_in if stream_in is not None else stream
         self.log = []  # (op, engine, seconds, bytes)
         for e in engines:
             need = [0] * self.n_gpus
@@ -86,16 +88,43 @@ class HotSwapController:
         self.log.append(("in", e.name, dt, e.payload))
         return dt
 
+    def exchange(self, bid: int, victims: list, free_before: list) -> float:
+        """Victims out and `bid` in, overlapped per GPU on the duplex link (swap_exchange). Each GPU's
+        exchange may use that GPU's free budget before the grant as headroom."""
+        e = self.engines[bid]
+        t0 = time.perf_counter()
+        for g in range(self.n_gpus):
+            vs = [s.swapper for v in victims for s in self.engines[v].shards if s.gpu == g]
+            ins = [s for s in e.shards if s.gpu == g]
+            if not vs and not ins:
+                continue
+            for v in victims:
+                self.sched.lock(v, True)
+            exchange(vs, ins[0].swapper if ins else None, self.stream, self.stream_in, headroom=free_before[g])
+            for v in victims:
+                self.sched.lock(v, False)
+            for s in ins:
+                res = s.swapper.verify(self.stream_in, hbm_pass=True)
+                if res["status"] != 0:
+                    raise RuntimeError(f"swap-in of {e.name} failed verification: {res}")
+        dt = time.perf_counter() - t0
+        self.log.append(("exchange", e.name, dt, e.payload + sum(self.engines[v].payload for v in victims)))
+        return dt
+
     def ensure_resident(self, bid: int, priority: float):
-        """Steps (4)-(9) for one request. Returns (hit, victims, t_out, t_in) in seconds."""
+        """Steps (4)-(9) for one request. Returns (hit, victims, t_out, t_in) in seconds; with duplex
+        exchanges t_out is 0 and t_in is the whole overlapped exchange."""
         if self.resident(bid):
             return True, [], 0.0, 0.0
+        free_before = [self.sched.free(g) for g in range(self.n_gpus)]
         self.sched.reserve(bid, priority)
         g = self.sched.grant()
         if g is None or g[0] == "blocked" or g[0] != bid:
             self.sched.cancel(bid)
             raise RuntimeError(f"reservation for engine {bid} could not be granted: {g}")
         _, victims = g
+        if self.duplex:
+            return False, victims, 0.0, self.exchange(bid, victims, free_before)
         t_out = sum(self.swap_out(v) for v in victims)
         t_in = self.swap_in(bid)
         return False, victims, t_out, t_in

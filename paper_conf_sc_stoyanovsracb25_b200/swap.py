@@ -34,7 +34,7 @@ EXPORTS = [
     "swap_get_summary", "swap_import", "swap_save", "swap_load", "swap_set_global", "swap_merge_global", "swap_plan_layout", "swap_plan_manifest", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
     "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
-    "swap_arena_reacquire_range", "swap_bind_arena",
+    "swap_arena_reacquire_range", "swap_bind_arena", "swap_exchange",
     "swap_arena_destroy", "swap_sched_create", "swap_sched_add_backend", "swap_sched_touch", "swap_sched_lock",
     "swap_sched_plan", "swap_sched_reserve", "swap_sched_cancel", "swap_sched_grant", "swap_sched_release",
     "swap_sched_query", "swap_sched_free", "swap_sched_destroy",
@@ -128,6 +128,7 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_arena_reacquire": (st, [vp]),
         "swap_arena_reacquire_range": (st, [vp, ctypes.c_uint64, ctypes.c_uint64]),
         "swap_bind_arena": (st, [vp, vp]),
+        "swap_exchange": (st, [P(vp), sz, vp, vp, vp, ctypes.c_uint64, P(ctypes.c_uint64)]),
         "swap_arena_last_error": (ctypes.c_char_p, [vp]),
         "swap_arena_destroy": (None, [vp]),
         "swap_sched_create": (st, [u32, P(ctypes.c_uint64), P(vp)]),
@@ -405,6 +406,21 @@ class Swapper:
 
     def __exit__(self, *a):
         self.close()
+
+
+def exchange(victims, incoming, stream_out=None, stream_in=None, headroom: int = 0) -> int:
+    """swap_exchange: victims (Swappers with bound, mapped arenas) out, `incoming` (bound, released) in,
+    overlapped on the duplex link within the victims' HBM + headroom. Returns the peak extra HBM."""
+    arr = (ctypes.c_void_p * max(1, len(victims)))(*[v.ctx.value if hasattr(v.ctx, "value") else v.ctx for v in victims])
+    peak = ctypes.c_uint64()
+    so = _torch_stream(stream_out)
+    si = _torch_stream(stream_in)
+    st = load().swap_exchange(arr, len(victims), incoming.ctx if incoming is not None else None,
+                              ctypes.c_void_p(so), ctypes.c_void_p(si), headroom, ctypes.byref(peak))
+    if st:
+        who = incoming if incoming is not None else victims[0]
+        raise SwapError(st, load().swap_last_error(who.ctx).decode())
+    return peak.value
 
 
 # ------------------------------------------------------------------ Arena (releasable HBM)

@@ -99,3 +99,55 @@ def test_bound_arena_lazy_reacquire(swp, orc, mech):
                 assert np.array_equal(back[o:o + r.nbytes], want), (i, r.name)
         sw.bind_arena(None)
     arena.close()
+
+
+def _engine(swp, orc, seed, gib):
+    specs = W.scaled(W.config_b(), int(gib * (1 << 30)))
+    offs, total = W.place(specs)
+    arena = swp.Arena(total)
+    base, view = arena.alloc(total)
+    W.fill_device_arena(view, specs, offs, seed=seed)
+    regions = [(base + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs, offs))]
+    sw = swp.Swapper(regions, mechanism="ce_pipe", pipe_mib=128)
+    sw.bind_arena(arena)
+    return specs, offs, total, arena, view, sw, regions, base
+
+
+def test_exchange_full_duplex(swp, orc):
+    """Two victims out, one engine in, overlapped; the incoming maps HBM only as victims release it."""
+    s_out, s_in = torch.cuda.Stream(), torch.cuda.Stream()
+    ea = _engine(swp, orc, 1, 2.2)
+    eb = _engine(swp, orc, 2, 1.5)
+    ec = _engine(swp, orc, 3, 3.1)
+    # C is parked: snapshot after init, HBM released
+    c_specs, c_offs, c_total, c_arena, c_view, c_sw, c_regions, c_base = ec
+    c_host = c_view.cpu().numpy()
+    c_sw.swap_out(c_arena, s_in)
+    # A and B run for a while: change some bytes, so their images must be re-gathered
+    snaps = []
+    for (specs, offs, total, arena, view, sw, regions, base) in (ea, eb):
+        view[offs[3]:offs[3] + 999].fill_(0x42)
+        torch.cuda.synchronize()
+        snaps.append(view.cpu().numpy())
+    headroom = 256 << 20
+    peak = swp.exchange([ea[5], eb[5]], c_sw, s_out, s_in, headroom=headroom)
+    assert peak <= headroom
+    res = c_sw.verify(s_in)
+    assert res["status"] == 0 and res["hbm_n_bad"] == 0 and c_arena.resident
+    back = c_arena.tensor(0, c_total).cpu().numpy()
+    for r, o in zip(c_specs, c_offs):
+        assert np.array_equal(back[o:o + r.nbytes], c_host[o:o + r.nbytes])
+    for (specs, offs, total, arena, view, sw, regions, base), host in zip((ea, eb), snaps):
+        assert not arena.resident
+        rc, ref, _ = orc.checkpoint([(i, a, n, k) for (a, n, k, i) in regions], host, base, 1, 1 << 20, 4096,
+                                    threads=8)
+        assert np.array_equal(sw.image(), ref)
+        # and the victim comes back intact later
+        res = sw.swap_in(arena, s_in)
+        assert res["status"] == 0
+        back = arena.tensor(0, total).cpu().numpy()
+        for r, o in zip(specs, offs):
+            assert np.array_equal(back[o:o + r.nbytes], host[o:o + r.nbytes])
+    for e in (ea, eb, ec):
+        e[5].close()
+        e[3].close()

@@ -35,6 +35,7 @@ ap.add_argument("--rate", type=float, default=0.25, help="base arrivals per seco
 ap.add_argument("--kv-tokens", type=int, default=1 << 16)
 ap.add_argument("--budget-gb", type=float, default=60.0, help="per logical GPU")
 ap.add_argument("--mechanism", default="auto")
+ap.add_argument("--duplex", action="store_true", help="overlap swap-out and swap-in (swap_exchange)")
 ap.add_argument("--out", default=None)
 args = ap.parse_args()
 
@@ -60,7 +61,8 @@ with torch.cuda.stream(stream):
             e.shards.append(Shard(g, arena, sw, sum(r.nbytes for r in specs)))
         engines.append(e)
 t_setup = time.perf_counter() - t0
-ctl = HotSwapController(engines, [int(args.budget_gb * 1e9)] * 2, stream)
+ctl = HotSwapController(engines, [int(args.budget_gb * 1e9)] * 2, stream, duplex=args.duplex,
+                        stream_in=torch.cuda.Stream() if args.duplex else None)
 
 trace = W.trace_e(args.seed, args.duration, rate_per_s=args.rate)
 names = {e.name: e.bid for e in engines}
@@ -68,7 +70,7 @@ busy_until = {e.bid: 0.0 for e in engines}
 last_access = {e.bid: 0.0 for e in engines}
 inflight = {e.bid: [] for e in engines}  # (arrival, end)
 vt = 0.0
-lat, swapin, hits, req_lat = [], [], 0, []
+lat, swapin, hits, req_lat, swaptotal = [], [], 0, [], []
 wall0 = time.perf_counter()
 with torch.cuda.stream(stream):
     for (t, model, svc) in trace:
@@ -89,6 +91,7 @@ with torch.cuda.stream(stream):
             vt = max(vt, victims_busy) + t_out + t_in
             ready = vt
             swapin.append((model, t_in, engines[bid].payload))
+            swaptotal.append(t_out + t_in)
         start = max(ready, busy_until[bid])
         end = start + svc
         busy_until[bid] = end
@@ -122,10 +125,13 @@ rec = {
     "swap_out_GBps_mean": round(statistics.mean(x[3] / x[2] for x in outs) / 1e9, 2) if outs else None,
     "swaps_per_hour": round((len(swapin) + len(outs)) / virtual_h, 1) if virtual_h else None,
     "request_latency_s": {"p50": round(pct(req_lat, 50), 3), "p99": round(pct(req_lat, 99), 3)},
+    "swap_time_s": {"p50": pct(swaptotal, 50), "p99": pct(swaptotal, 99), "mean": round(statistics.mean(swaptotal), 4)
+                    if swaptotal else None,
+                    "what": "request-visible swap time: victims out + requested engine in (+ HBM verify)"},
     "per_model": per_model,
     "config": {"duration_s": args.duration, "seed": args.seed, "rate_per_s": args.rate,
                "kv_tokens": args.kv_tokens, "budget_GB_per_logical_gpu": args.budget_gb,
-               "mechanism": args.mechanism},
+               "mechanism": args.mechanism, "duplex": args.duplex},
     "wall_s": round(wall, 1), "setup_s": round(t_setup, 1), "virtual_s": round(vt, 1),
 }
 s = json.dumps(rec)
