@@ -58,7 +58,7 @@ typedef int32_t swap_status;
 #define SWAP_CHECKSUM_XXH64 2u  /* XXH64, seed 0 for every chunk */
 
 /* Data mover for checkpoint/restore (the image bytes are identical for all of them): */
-#define SWAP_MECH_AUTO 0u        /* default: SWAP_MECH_CE_PIPE when the payload is >= 512 MiB (and, for XXH64,
+#define SWAP_MECH_AUTO 0u        /* default: SWAP_MECH_CE_PIPE when the payload is >= 1 GiB (and, for XXH64,
                                     chunk_bytes <= 1 MiB), else SWAP_MECH_SM (DESIGN.md §6 mechanism sweep) */
 #define SWAP_MECH_SM 1u          /* one SM kernel: 16-B vector loads/stores to mapped pinned host memory with the
                                     chunk checksum fused from the same registers (one pass, bytes checked in flight) */
@@ -98,8 +98,10 @@ typedef struct {
   int32_t rank;         /* 0 <= rank < world (tensor-parallel shard index) */
   int32_t world;        /* >= 1 */
   uint32_t grid_ctas;   /* SM mover grid; 0 -> auto (2 CTAs per SM) */
-  uint32_t seg_bytes;   /* CRC32C work split inside a chunk: power of 2, >= 4096; 0 -> 256 KiB */
-  uint32_t pipe_mib;    /* SWAP_MECH_CE_PIPE group size in MiB (rounded to whole chunks); 0 -> 256 */
+  uint32_t seg_bytes;   /* CRC32C work split inside a chunk: power of 2, >= 4096; 0 -> auto (at registration:
+                           one segment per warp slot of the GPU, 4 KiB .. 256 KiB) */
+  uint32_t pipe_mib;    /* SWAP_MECH_CE_PIPE group size in MiB (rounded to whole chunks); 0 -> auto: payload/32
+                           clamped to [2, 256] MiB */
 } swap_config_t;
 
 typedef struct {

@@ -65,7 +65,6 @@ swap_status normalize_config(swap_config_t* c, std::string* err) {
   if (c->chunk_bytes == 0) c->chunk_bytes = 1ull << 20;
   if (c->align == 0) c->align = 4096;
   if (c->checksum == 0) c->checksum = SWAP_CHECKSUM_CRC32C;
-  if (c->seg_bytes == 0) c->seg_bytes = 256u << 10;
   if (!pow2_ge(c->chunk_bytes, 16) || !pow2_ge(c->align, 16)) {
     *err = "chunk_bytes and align must be powers of 2 >= 16";
     return SWAP_EINVAL;
@@ -74,7 +73,6 @@ swap_status normalize_config(swap_config_t* c, std::string* err) {
     *err = "checksum must be SWAP_CHECKSUM_CRC32C or SWAP_CHECKSUM_XXH64";
     return SWAP_EINVAL;
   }
-  if (c->pipe_mib == 0) c->pipe_mib = 256;
   if (c->mechanism >= SWAP_MECH_COUNT) {
     *err = "unknown mechanism";
     return SWAP_EINVAL;
@@ -83,8 +81,8 @@ swap_status normalize_config(swap_config_t* c, std::string* err) {
     *err = "need world >= 1, 0 <= rank < world, device >= 0";
     return SWAP_EINVAL;
   }
-  if (!pow2_ge(c->seg_bytes, 4096)) {
-    *err = "seg_bytes must be a power of 2 >= 4096";
+  if (c->seg_bytes != 0 && !pow2_ge(c->seg_bytes, 4096)) {
+    *err = "seg_bytes must be 0 (auto) or a power of 2 >= 4096";
     return SWAP_EINVAL;
   }
   if (c->chunk_bytes > (1ull << 31)) {

@@ -81,6 +81,7 @@ struct swap_ctx {
   swk::DevStatus* h_status = nullptr;  // pinned
   uint32_t* d_tables = nullptr;
   uint32_t zinit_c = 0, xseg = 0;
+  uint32_t seg = 0;  // CRC-32C segment size in use (cfg.seg_bytes, or chosen at registration when 0)
   cudaEvent_t ev[6] = {};  // checkpoint, restore, verify: begin/end pairs
   bool pending[3] = {false, false, false};
   float ms[3] = {0.f, 0.f, 0.f};
@@ -111,7 +112,7 @@ swk::Params base_params(swap_ctx* c, const DescSet& S) {
   swk::Params p{};
   p.desc = S.d_desc;
   p.n_desc = S.n_desc;
-  p.seg_bytes = c->cfg.seg_bytes;
+  p.seg_bytes = c->seg;
   p.partial = c->d_partial;
   p.arrive = c->d_arrive;
   const uint64_t cs_off = c->plan.manifest_off + swp::kHeaderBytes + swp::kRegionRecBytes * c->plan.regions.size() + 24;
@@ -123,7 +124,7 @@ swk::Params base_params(swap_ctx* c, const DescSet& S) {
   p.chunk_bytes = c->plan.C;
   p.zinit_c = c->zinit_c;
   p.xseg = c->xseg;
-  p.hlane_len = (uint32_t)std::min<uint64_t>(c->plan.C, c->cfg.seg_bytes);
+  p.hlane_len = (uint32_t)std::min<uint64_t>(c->plan.C, c->seg);
   return p;
 }
 
@@ -132,7 +133,7 @@ int grid_of(swap_ctx* c) { return c->cfg.grid_ctas ? (int)c->cfg.grid_ctas : 2 *
 // The mechanism actually used: AUTO picks the copy-engine pipeline for large images (the copy
 // engines reach a higher link rate than SM-issued accesses) and the single fused
 // SM pass for small ones (no per-copy launch overhead).
-constexpr uint64_t kAutoPipeBytes = 512ull << 20;
+constexpr uint64_t kAutoPipeBytes = 1ull << 30;  // crossover measured: 1 GiB ties, 4 GiB CE_PIPE +5 %, <= 256 MiB SM
 // XXH64 is not combinable: with chunks > 1 MiB a pipeline group holds too few chunks for the
 // side-stream hash to keep up with the link, while the fused SM pass hashes every chunk in flight.
 uint32_t mech(const swap_ctx* c) {
@@ -270,6 +271,28 @@ void free_set(DescSet& S) {
   S = DescSet();
 }
 
+// CRC tables for the ctx's chunk and segment sizes (the hash kernels fold lanes with constants that
+// depend on min(C, seg)); uploads them and derives the init / segment shift constants.
+swap_status upload_tables(swap_ctx* c) {
+  std::vector<uint32_t> tab(swk::TAB_WORDS);
+  swk::build_tables(tab.data(), std::min<uint64_t>(c->cfg.chunk_bytes, c->seg));
+  if (!c->d_tables) CUDA_TRY(c, cudaMalloc(&c->d_tables, tab.size() * 4));
+  CUDA_TRY(c, cudaMemcpy(c->d_tables, tab.data(), tab.size() * 4, cudaMemcpyHostToDevice));
+  const uint32_t* x2n = tab.data() + swk::TAB_X2N;
+  c->zinit_c = swk::host_multmodp(swk::host_x2nmodp(c->cfg.chunk_bytes, 3, x2n), 0xFFFFFFFFu);
+  c->xseg = swk::host_x2nmodp(c->seg, 3, x2n);
+  return SWAP_OK;
+}
+
+// Auto segment size: enough CRC work items to give every warp slot of the GPU (SMs x 32) one, between
+// 4 KiB and 256 KiB (large images keep 256 KiB; a 64 MiB image gets 8 KiB).
+uint32_t auto_seg(const swap_ctx* c, uint64_t payload) {
+  const uint64_t per = payload / ((uint64_t)c->sm_count * 32 + 1);
+  uint64_t s = 4096;
+  while (s * 2 <= per && s < (256u << 10)) s *= 2;
+  return (uint32_t)s;
+}
+
 void release(swap_ctx* c) {
   free_set(c->s_move);
   free_set(c->s_save);
@@ -298,9 +321,12 @@ void release(swap_ctx* c) {
 template <class Pick>
 swap_status build_set(swap_ctx* c, DescSet* S, Pick pick, bool zero_src) {
   const swp::Plan& P = c->plan;
-  const uint64_t seg = P.kind == SWAP_CHECKSUM_XXH64 ? P.C : std::min<uint64_t>(P.C, c->cfg.seg_bytes);
+  const uint64_t seg = P.kind == SWAP_CHECKSUM_XXH64 ? P.C : std::min<uint64_t>(P.C, c->seg);
   std::vector<swk::SegDesc> desc;
-  const uint64_t target = (uint64_t)c->cfg.pipe_mib << 20;
+  // group size: cfg.pipe_mib, or auto = payload / 32 clamped to [16 MiB, 256 MiB] (smaller groups cost
+  // more in per-copy and per-launch overhead than they gain in overlap)
+  uint64_t target = (uint64_t)c->cfg.pipe_mib << 20;
+  if (!target) target = std::min<uint64_t>(256ull << 20, std::max<uint64_t>(16ull << 20, c->plan.payload_bytes / 32));
   Group cur{0, 0, {}};
   uint64_t cur_bytes = 0;
   for (size_t i = 0; i < P.regions.size(); ++i) {
@@ -419,8 +445,8 @@ void swap_config_default(swap_config_t* cfg) {
   cfg->checksum = SWAP_CHECKSUM_CRC32C;
   cfg->mechanism = SWAP_MECH_AUTO;
   cfg->world = 1;
-  cfg->seg_bytes = 256u << 10;
-  cfg->pipe_mib = 256;
+  cfg->seg_bytes = 0;  // auto
+  cfg->pipe_mib = 0;  // auto
 }
 
 swap_status swap_create(const swap_config_t* cfg_in, swap_ctx_t** out) {
@@ -452,11 +478,7 @@ swap_status swap_create(const swap_config_t* cfg_in, swap_ctx_t** out) {
   }
   c->sm_count = prop.multiProcessorCount;
   DeviceGuard g(c->cfg.device);
-  std::vector<uint32_t> tab(swk::TAB_WORDS);
-  swk::build_tables(tab.data(), std::min<uint64_t>(c->cfg.chunk_bytes, c->cfg.seg_bytes));
-  if ((e = cudaMalloc(&c->d_tables, tab.size() * 4)) != cudaSuccess ||
-      (e = cudaMemcpy(c->d_tables, tab.data(), tab.size() * 4, cudaMemcpyHostToDevice)) != cudaSuccess ||
-      (e = cudaMalloc(&c->d_status, sizeof(swk::DevStatus))) != cudaSuccess ||
+  if ((e = cudaMalloc(&c->d_status, sizeof(swk::DevStatus))) != cudaSuccess ||
       (e = cudaMemset(c->d_status, 0, sizeof(swk::DevStatus))) != cudaSuccess ||
       (e = cudaHostAlloc(&c->h_status, sizeof(swk::DevStatus), cudaHostAllocDefault)) != cudaSuccess ||
       (e = cudaEventCreate(&c->ev[0])) != cudaSuccess || (e = cudaEventCreate(&c->ev[1])) != cudaSuccess ||
@@ -468,9 +490,6 @@ swap_status swap_create(const swap_config_t* cfg_in, swap_ctx_t** out) {
     delete c;
     return SWAP_ECUDA;
   }
-  const uint32_t* x2n = tab.data() + swk::TAB_X2N;
-  c->zinit_c = swk::host_multmodp(swk::host_x2nmodp(c->cfg.chunk_bytes, 3, x2n), 0xFFFFFFFFu);
-  c->xseg = swk::host_x2nmodp(c->cfg.seg_bytes, 3, x2n);
   *out = c;
   return SWAP_OK;
 }
@@ -520,6 +539,8 @@ swap_status swap_register_regions(swap_ctx_t* c, const swap_region_t* regions, s
   CUDA_TRY(c, cudaStreamCreateWithFlags(&c->side, cudaStreamNonBlocking));
   CUDA_TRY(c, cudaMalloc(&c->d_arrive, std::max<uint64_t>(1, P.n_chunks) * 4));
   CUDA_TRY(c, cudaMemset(c->d_arrive, 0, std::max<uint64_t>(1, P.n_chunks) * 4));
+  c->seg = c->cfg.seg_bytes ? c->cfg.seg_bytes : auto_seg(c, P.payload_bytes);
+  if ((st = upload_tables(c)) != SWAP_OK) return st;
   c->policy.assign(P.regions.size(), SWAP_POLICY_SAVE);
   st = build_sets(c);
   if (st != SWAP_OK) return st;

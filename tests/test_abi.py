@@ -53,7 +53,7 @@ def test_struct_sizes_match_header(swp):
 
 def test_config_default(swp):
     c = swp.swap_config_default()
-    assert (c.chunk_bytes, c.align, c.checksum, c.mechanism, c.world, c.seg_bytes) == (1 << 20, 4096, 1, 0, 1, 256 << 10)
+    assert (c.chunk_bytes, c.align, c.checksum, c.mechanism, c.world, c.seg_bytes) == (1 << 20, 4096, 1, 0, 1, 0)
 
 
 def test_status_strings(swp):
