@@ -263,6 +263,15 @@ SWAP_API swap_status swap_arena_reacquire_range(swap_arena_t* a, uint64_t offset
  * NULL unbinds. The arena must outlive the binding. */
 SWAP_API swap_status swap_bind_arena(swap_ctx_t* ctx, swap_arena_t* a);
 
+/* NVLink-assisted restore (NEXT-2): with SWAP_MECH_CE_PIPE, restore groups are striped round-robin over
+ * this device and the `n` helper devices; a helper copies its groups' image range from the pinned host
+ * image into its own HBM staging buffer over its own PCIe link, then to this device's regions with
+ * peer copies (NVLink via NVSwitch), and this device's side stream checks each group as usual. Helpers
+ * should be idle GPUs of the node; peer access to this device is enabled on each. A helper equal to this
+ * device degenerates to an on-device staging copy (used by the one-GPU tests). n = 0 removes them.
+ * Needs REGISTERED+ (staging is sized from the restore groups). The checkpoint path is unchanged. */
+SWAP_API swap_status swap_set_helpers(swap_ctx_t* ctx, const int* devices, int n);
+
 /* Full-duplex exchange on one device (NEXT-1; §3.4-3.5 swap-out of victims then swap-in of the
  * requested backend, here overlapped on the duplex PCIe link): checkpoints + seals + releases every victim
  * (each with a bound, mapped arena) on s_out while scattering `incoming` (bound, released arena; sealed

@@ -91,6 +91,15 @@ struct swap_ctx {
   // CE_PIPE
   cudaStream_t side = nullptr;
   swap_arena* arena = nullptr;  // bound arena: restore re-acquires its HBM (swap_bind_arena)
+  // NVLink-assisted restore (swap_set_helpers): peers pull groups over their own PCIe links into
+  // HBM staging and copy them to this device over NVLink
+  struct Helper {
+    int dev = -1;
+    cudaStream_t s = nullptr;
+    uint8_t* staging = nullptr;
+    cudaEvent_t ev = nullptr, done = nullptr;
+  };
+  std::vector<Helper> helpers;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };
 
@@ -232,9 +241,34 @@ swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, c
   CUDA_TRY(c, cudaStreamWaitEvent(c->side, c->ev_fork, 0));
   swap_status st;
   if (dir == 0 && (st = launch(c, swk::HASH_STORE, hash_kind(c), base, c->side)) != SWAP_OK) return st;
+  const size_t H = dir == 1 ? c->helpers.size() : 0;
+  for (auto& h : c->helpers)
+    if (H) CUDA_TRY(c, cudaStreamWaitEvent(h.s, c->ev_fork, 0));
   for (size_t g = 0; g < S.groups.size(); ++g) {
     const Group& G = S.groups[g];
     if (dir == 1 && (st = map_spans(c, G.spans)) != SWAP_OK) return st;  // lazy HBM re-acquire
+    const size_t k = H ? g % (H + 1) : 0;
+    if (k > 0) {
+      // helper k-1: H2D of the group's image range into its staging over its own PCIe link, then
+      // NVLink peer copies of each span to this device; the side stream checks it as usual
+      auto& h = c->helpers[k - 1];
+      uint8_t* lo = G.spans.front().host;
+      uint8_t* hi = G.spans.back().host + G.spans.back().bytes;
+      CUDA_TRY(c, cudaSetDevice(h.dev));
+      CUDA_TRY(c, cudaMemcpyAsync(h.staging, lo, (size_t)(hi - lo), cudaMemcpyHostToDevice, h.s));
+      for (const Span& sp : G.spans)
+        CUDA_TRY(c, cudaMemcpyPeerAsync(reinterpret_cast<void*>(sp.dev), c->cfg.device, h.staging + (sp.host - lo), h.dev,
+                                        sp.bytes, h.s));
+      CUDA_TRY(c, cudaEventRecord(h.ev, h.s));
+      CUDA_TRY(c, cudaSetDevice(c->cfg.device));
+      CUDA_TRY(c, cudaStreamWaitEvent(c->side, h.ev, 0));
+      swk::Params p = base;
+      p.desc = base.desc + G.d0;
+      p.partial = base.partial + G.d0;
+      p.n_desc = G.d1 - G.d0;
+      if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, c->side)) != SWAP_OK) return st;
+      continue;
+    }
     for (const Span& sp : G.spans)
       if ((st = memcpy_dir(c, sp, dir, s)) != SWAP_OK) return st;
     if (dir == 1) {
@@ -246,6 +280,13 @@ swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, c
       p.n_desc = G.d1 - G.d0;
       if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, c->side)) != SWAP_OK) return st;
     }
+  }
+  for (auto& h : c->helpers) {
+    if (!H) break;
+    CUDA_TRY(c, cudaSetDevice(h.dev));
+    CUDA_TRY(c, cudaEventRecord(h.done, h.s));
+    CUDA_TRY(c, cudaSetDevice(c->cfg.device));
+    CUDA_TRY(c, cudaStreamWaitEvent(s, h.done, 0));
   }
   CUDA_TRY(c, cudaEventRecord(c->ev_join, c->side));
   CUDA_TRY(c, cudaStreamWaitEvent(s, c->ev_join, 0));
@@ -293,7 +334,23 @@ uint32_t auto_seg(const swap_ctx* c, uint64_t payload) {
   return (uint32_t)s;
 }
 
+void free_helpers(swap_ctx* c) {
+  int cur = -1;
+  cudaGetDevice(&cur);
+  for (auto& h : c->helpers) {
+    cudaSetDevice(h.dev);
+    if (h.s) cudaStreamSynchronize(h.s);
+    if (h.staging) cudaFree(h.staging);
+    if (h.ev) cudaEventDestroy(h.ev);
+    if (h.done) cudaEventDestroy(h.done);
+    if (h.s) cudaStreamDestroy(h.s);
+  }
+  c->helpers.clear();
+  if (cur >= 0) cudaSetDevice(cur);
+}
+
 void release(swap_ctx* c) {
+  free_helpers(c);
   free_set(c->s_move);
   free_set(c->s_save);
   free_set(c->s_zero);
@@ -687,7 +744,11 @@ swap_status swap_set_region_policy(swap_ctx_t* c, uint32_t region_index, uint32_
   if (c->policy[region_index] == policy) return SWAP_OK;
   c->policy[region_index] = policy;
   DeviceGuard g(c->cfg.device);
-  return build_sets(c);
+  swap_status st = build_sets(c);
+  if (st != SWAP_OK || c->helpers.empty()) return st;
+  std::vector<int> devs;  // restore groups changed: re-size the helpers' staging
+  for (auto& h : c->helpers) devs.push_back(h.dev);
+  return swap_set_helpers(c, devs.data(), (int)devs.size());
 }
 
 // Full-duplex exchange (see include/swap.h). Victims are gathered group by group on s_out (hash pass of
@@ -866,6 +927,37 @@ swap_status swap_exchange(swap_ctx_t* const* victims, size_t nv, swap_ctx_t* in,
     v->st = St::CHECKPOINTED;
   }
   if (peak_extra) *peak_extra = peak;
+  return SWAP_OK;
+}
+
+swap_status swap_set_helpers(swap_ctx_t* c, const int* devices, int n) {
+  if (!c || n < 0 || (n && !devices)) return SWAP_EINVAL;
+  if (c->st == St::CREATED) return SWAP_ESTATE;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess) return SWAP_ECUDA;
+  for (int i = 0; i < n; ++i)
+    if (devices[i] < 0 || devices[i] >= ndev) return SWAP_EINVAL;
+  DeviceGuard g(c->cfg.device);
+  free_helpers(c);
+  uint64_t stage = 0;  // largest image range of one restore group
+  for (const Group& G : c->s_move.groups)
+    stage = std::max<uint64_t>(stage, (uint64_t)(G.spans.back().host + G.spans.back().bytes - G.spans.front().host));
+  for (int i = 0; i < n; ++i) {
+    swap_ctx::Helper h;
+    h.dev = devices[i];
+    CUDA_TRY(c, cudaSetDevice(h.dev));
+    if (h.dev != c->cfg.device) {
+      cudaError_t e = cudaDeviceEnablePeerAccess(c->cfg.device, 0);  // NVLink P2P to the target
+      if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return cuda_fail(c, e, "peer access");
+      cudaGetLastError();
+    }
+    CUDA_TRY(c, cudaStreamCreateWithFlags(&h.s, cudaStreamNonBlocking));
+    CUDA_TRY(c, cudaEventCreateWithFlags(&h.ev, cudaEventDisableTiming));
+    CUDA_TRY(c, cudaEventCreateWithFlags(&h.done, cudaEventDisableTiming));
+    CUDA_TRY(c, cudaMalloc(&h.staging, std::max<uint64_t>(stage, 16)));
+    c->helpers.push_back(h);
+  }
+  CUDA_TRY(c, cudaSetDevice(c->cfg.device));
   return SWAP_OK;
 }
 

@@ -34,7 +34,7 @@ EXPORTS = [
     "swap_get_summary", "swap_import", "swap_save", "swap_load", "swap_set_global", "swap_merge_global", "swap_plan_layout", "swap_plan_manifest", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
     "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
-    "swap_arena_reacquire_range", "swap_bind_arena", "swap_exchange",
+    "swap_arena_reacquire_range", "swap_bind_arena", "swap_exchange", "swap_set_helpers",
     "swap_arena_destroy", "swap_sched_create", "swap_sched_add_backend", "swap_sched_touch", "swap_sched_lock",
     "swap_sched_plan", "swap_sched_reserve", "swap_sched_cancel", "swap_sched_grant", "swap_sched_release",
     "swap_sched_query", "swap_sched_free", "swap_sched_destroy",
@@ -128,6 +128,7 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_arena_reacquire": (st, [vp]),
         "swap_arena_reacquire_range": (st, [vp, ctypes.c_uint64, ctypes.c_uint64]),
         "swap_bind_arena": (st, [vp, vp]),
+        "swap_set_helpers": (st, [vp, P(ctypes.c_int), ctypes.c_int]),
         "swap_exchange": (st, [P(vp), sz, vp, vp, vp, ctypes.c_uint64, P(ctypes.c_uint64)]),
         "swap_arena_last_error": (ctypes.c_char_p, [vp]),
         "swap_arena_destroy": (None, [vp]),
@@ -314,6 +315,11 @@ class Swapper:
         self.checkpoint(stream, sync=True)
         if arena is not None:
             arena.release()
+
+    def set_helpers(self, devices):
+        """NVLink-assisted restore: stripe CE_PIPE restore groups over these (idle) peer GPUs."""
+        arr = (ctypes.c_int * max(1, len(devices)))(*devices)
+        self._check(load().swap_set_helpers(self._ctx, arr, len(devices)))
 
     def bind_arena(self, arena: "Arena | None"):
         """Let restore re-acquire this arena's HBM itself (group by group under CE_PIPE)."""
