@@ -42,8 +42,8 @@ RESTORE_KERNEL = {
     "ce_chunk": "restore phase: cudaMemcpyAsync per chunk + HBM hash pass",
     "ce_batch": "restore phase: cudaMemcpyBatchAsync + HBM hash pass",
 }
-VERIFY_KERNEL = {"crc32c": "hash_kernel<HASH_CHECK> (CRC-32C, per-lane runs, replicated slice-by-4 tables)",
-                 "xxh64": "xxh_lane_kernel<HASH_CHECK> (XXH64, one lane per chunk)"}
+VERIFY_KERNEL = {"crc32c": "hash_kernel<HASH_CHECK> (CRC-32C: quad-line 256-bit loads, per-lane replicated slice-by-4 + Z^96 tables)",
+                 "xxh64": "xxh_lane_kernel<HASH_CHECK> (XXH64, one lane per chunk; TMA-ring kernel for few large chunks)"}
 PCIE_GEN5_X16_GBPS = 63.015  # 64 GB/s x 128/130 (nominal, per direction)
 MEASURED_PEAKS = os.path.join(ROOT, "MEASURED_PEAKS.json")
 
