@@ -1,0 +1,52 @@
+"""compute-sanitizer workload: every kernel family and mover on small images (tools/sanitize.sh)."""
+import os
+import sys
+
+ROOT = os.environ.get("GRAFT_REPO_ROOT", os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, ROOT)
+sys.path.insert(0, os.path.join(ROOT, "tests"))
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import workloads as W  # noqa: E402
+from gpu_util import device_case, poison  # noqa: E402
+from paper_conf_sc_stoyanovsracb25_b200 import swap  # noqa: E402
+
+s = torch.cuda.Stream()
+specs = W.config_a(3)[:6] + W.edge_tables(4096)["edge_sizes"]
+arena, host, base, offs, regions, _ = device_case(specs, 3)
+for kind in (1, 2):
+    for mech, extra in (("sm", {}), ("ce_pipe", {"pipe_mib": 4}), ("ce_region", {}), ("ce_batch", {})):
+        for C in (4096, 1 << 20):
+            with swap.Swapper(regions, chunk_bytes=C, checksum=kind, mechanism=mech, **extra) as sw, \
+                    torch.cuda.stream(s):
+                if mech == "ce_pipe":
+                    sw.set_helpers([0])
+                sw.set_region_policy(1, "discard")
+                sw.checkpoint(s)
+                poison(arena, specs, offs)
+                sw.restore(s)
+                assert sw.verify(s)["status"] == 0, (kind, mech, C)
+# XXH64 kernel variants are chosen by chunk count; a 1 KiB-chunk case exercises the lane kernel
+with swap.Swapper(regions, chunk_bytes=1024, checksum=2, mechanism="ce_region") as sw, torch.cuda.stream(s):
+    sw.checkpoint(s)
+    sw.restore(s)
+    assert sw.verify(s)["status"] == 0
+# VMM arenas + full-duplex exchange
+def engine(seed):
+    sp = W.scaled(W.config_b(), 48 << 20)
+    of, total = W.place(sp)
+    a = swap.Arena(total)
+    b, view = a.alloc(total)
+    W.fill_device_arena(view, sp, of, seed=seed)
+    sw = swap.Swapper([(b + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(sp, of))], mechanism="ce_pipe",
+                      pipe_mib=4)
+    sw.bind_arena(a)
+    return a, sw
+a1, v1 = engine(1)
+a2, inc = engine(2)
+inc.swap_out(a2, s)
+swap.exchange([v1], inc, s, s, headroom=0)
+assert inc.verify(s)["status"] == 0
+print("sanitize case ok")
