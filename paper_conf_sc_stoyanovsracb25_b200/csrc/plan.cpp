@@ -4,6 +4,10 @@
 
 #include <algorithm>
 #include <cstring>
+#if defined(__x86_64__)
+#include <cpuid.h>
+#include <nmmintrin.h>
+#endif
 
 namespace swp {
 
@@ -42,7 +46,76 @@ const Crc8Tables& crc_tables() {
 }
 }  // namespace
 
+#if defined(__x86_64__)
+bool have_crc32_insn() {
+  static const bool ok = [] {
+    unsigned a, b, c, d;
+    return __get_cpuid(1, &a, &b, &c, &d) && (c & bit_SSE4_2);
+  }();
+  return ok;
+}
+// The SSE4.2 crc32 instruction implements the CRC-32C register update; three independent streams
+// hide its 3-cycle latency and are merged with the GF(2) shift (crc_shift_bytes below).
+uint32_t crc_shift_bytes(uint32_t c, uint64_t n);
+__attribute__((target("sse4.2"))) uint32_t crc32c_hw(const uint8_t* p, size_t n, uint32_t c32) {
+  uint64_t c = c32;
+  if (n >= 3 * 4096) {
+    const size_t blk = n / 3 / 8 * 8;
+    uint64_t c1 = 0, c2 = 0;
+    const uint8_t* q1 = p + blk;
+    const uint8_t* q2 = p + 2 * blk;
+    for (size_t i = 0; i < blk; i += 8) {
+      uint64_t w0, w1, w2;
+      std::memcpy(&w0, p + i, 8);
+      std::memcpy(&w1, q1 + i, 8);
+      std::memcpy(&w2, q2 + i, 8);
+      c = _mm_crc32_u64(c, w0);
+      c1 = _mm_crc32_u64(c1, w1);
+      c2 = _mm_crc32_u64(c2, w2);
+    }
+    // register after stream 0 then stream 1 then stream 2 (streams 1, 2 started from 0: linearity)
+    c = crc_shift_bytes((uint32_t)c, blk) ^ (uint32_t)c1;
+    c = crc_shift_bytes((uint32_t)c, blk) ^ (uint32_t)c2;
+    p += 3 * blk;
+    n -= 3 * blk;
+  }
+  for (; n >= 8; n -= 8, p += 8) {
+    uint64_t w;
+    std::memcpy(&w, p, 8);
+    c = _mm_crc32_u64(c, w);
+  }
+  uint32_t r = (uint32_t)c;
+  for (; n; --n) r = _mm_crc32_u8(r, *p++);
+  return r;
+}
+#endif
+
+// Z^n (n zero bytes) of a register: square-and-multiply with x^(2^k) mod P, reflected.
+uint32_t gf2_mul(uint32_t a, uint32_t b) {
+  uint32_t p = 0;
+  for (int i = 0; i < 32; ++i) {
+    if ((a >> (31 - i)) & 1u) p ^= b;
+    b = (b & 1u) ? (b >> 1) ^ 0x82F63B78u : (b >> 1);
+  }
+  return p;
+}
+uint32_t crc_shift_bytes(uint32_t c, uint64_t n) {
+  static const std::vector<uint32_t> x2n = [] {
+    std::vector<uint32_t> t(64);
+    t[0] = 1u << 30;  // x^1
+    for (int k = 1; k < 64; ++k) t[k] = gf2_mul(t[k - 1], t[k - 1]);
+    return t;
+  }();
+  uint32_t x = 1u << 31;  // x^0
+  for (unsigned k = 3; n; n >>= 1, ++k)
+    if (n & 1) x = gf2_mul(x2n[k & 63], x);
+  return gf2_mul(x, c);
+}
+
 uint32_t crc32c_host(const void* data, size_t n, uint32_t crc) {
+#if defined(__x86_64__)
+  if (have_crc32_insn()) return ~crc32c_hw(static_cast<const uint8_t*>(data), n, ~crc);
+#endif
   const auto& T = crc_tables().t;
   const uint8_t* p = static_cast<const uint8_t*>(data);
   uint32_t c = ~crc;
@@ -213,8 +286,11 @@ swap_status check_manifest(const Plan& p, const uint8_t* man, std::string* err) 
     return SWAP_ECORRUPT;
   }
   // The CRC holds: the manifest must also describe this ctx's registered layout.
-  std::vector<uint8_t> want(p.manifest_bytes);
-  write_manifest_skeleton(p, want.data());
+  if (p.skeleton.size() != p.manifest_bytes) {
+    p.skeleton.resize(p.manifest_bytes);
+    write_manifest_skeleton(p, p.skeleton.data());
+  }
+  const std::vector<uint8_t>& want = p.skeleton;
   const uint64_t chunk_base = kHeaderBytes + kRegionRecBytes * p.regions.size();
   if (std::memcmp(want.data(), man, chunk_base) != 0) {
     *err = "manifest header/regions do not match the registered layout";

@@ -27,6 +27,7 @@ struct Plan {
   std::vector<RegionPlan> regions;
   uint64_t payload_bytes = 0, n_chunks = 0;
   uint64_t manifest_off = 0, manifest_bytes = 0, image_bytes = 0;
+  mutable std::vector<uint8_t> skeleton;  // cached static manifest bytes (c_g = 0, no trailer) for checks
 };
 
 constexpr uint64_t kHeaderBytes = 64, kRegionRecBytes = 48, kChunkRecBytes = 32, kTrailerBytes = 8;
@@ -45,7 +46,8 @@ swap_status check_manifest(const Plan& p, const uint8_t* man, std::string* err);
 bool manifest_crc_ok(const Plan& p, const uint8_t* man);
 void make_summary(const Plan& p, const uint8_t* man, swap_shard_summary_t* out);
 
-// Host CRC-32C (slicing-by-8), standard init/xorout.
+// Host CRC-32C, standard init/xorout: SSE4.2 crc32 instruction (3 interleaved streams) when present,
+// else slicing-by-8.
 uint32_t crc32c_host(const void* data, size_t n, uint32_t crc = 0);
 
 }  // namespace swp

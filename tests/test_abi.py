@@ -102,3 +102,13 @@ def test_merge_global_vs_oracle(swp, orc):
     assert swp.swap_merge_global(swapped, world)[0] == swp.SWAP_ENCCL
     wrong_world = SUM.pack(0, 2, 1, 1, 1, 1, 1, 1, 1, 0) + SUM.pack(1, 3, 1, 1, 1, 1, 1, 1, 1, 0)
     assert swp.swap_merge_global(wrong_world, 2)[0] == swp.SWAP_ENCCL
+
+
+def test_host_crc_paths_vs_oracle(swp, orc):
+    """libswap's host CRC-32C (hardware crc32 in three interleaved streams for long inputs, merged with
+    GF(2) shifts) against the oracle's table CRC, through swap_merge_global's digest."""
+    for world in (1, 3, 64, 193, 1000, 4099):
+        allb = b"".join(SUM.pack(r, world, 1 + r % 2, r % 7, r * 3, r * 5 + 1, r * 7 + 2, r * 11, r * 13, 0)
+                        for r in range(world))
+        st, d = swp.swap_merge_global(allb, world)
+        assert st == 0 and d == orc.global_digest(allb), world
