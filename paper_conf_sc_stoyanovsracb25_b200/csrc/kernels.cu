@@ -59,7 +59,7 @@ uint32_t host_x2nmodp(uint64_t n, unsigned k, const uint32_t* x2n) {  // x^(n*2^
   return p;
 }
 
-void build_tables(uint32_t* tab, uint64_t L1) {
+void build_tables(uint32_t* tab, uint64_t L1, uint64_t seg) {
   uint32_t* t = tab + TAB_T16;
   for (uint32_t b = 0; b < 256; ++b) t[b] = step_byte(b);  // T_0 = one byte
   for (int k = 1; k < 16; ++k)
@@ -82,6 +82,7 @@ void build_tables(uint32_t* tab, uint64_t L1) {
     const uint64_t end = hash_lane_end(L1, l);
     tab[TAB_HLANE + l] = end ? host_x2nmodp(L1 - end, 3, x2n) : 0u;
   }
+  for (int m = 0; m < ZS_N; ++m) tab[TAB_ZS + m] = host_x2nmodp((uint64_t)m * seg, 3, x2n);
   // Z^96 (the gap between a lane's consecutive 32-B pieces) of nibble v at nibble position k
   for (int kk = 0; kk < 8; ++kk)
     for (uint32_t v = 0; v < 16; ++v) {
@@ -190,6 +191,61 @@ __device__ __forceinline__ void chunk_result(const Params& p, uint32_t g, uint64
       atomicAdd(p.n_bad, 1ull);
       atomicMin(p.first_bad, static_cast<unsigned long long>(g));
     }
+  }
+}
+
+// Segment `idx` (descriptor d) of a CRC-32C chunk ends with register S (valid in lane 0). A one-segment
+// chunk is finished here; otherwise S is stored and the warp whose segment completes the chunk (atomic
+// arrival count) combines all partials, warp-parallel: lane l folds a contiguous range of segments with
+// Horner steps (crc(A||B) = Z^|B|(crc A) ^ crc B), shifts it past the segments that follow (a table of
+// x^(8*m*seg) for m whole segments, then the last one), and an XOR shuffle tree sums the lanes.
+template <int MODE>
+__device__ __forceinline__ void crc_segment_done(const Params& p, const SegDesc& d, uint32_t idx, uint32_t S, int lane) {
+  const uint32_t* x2n = p.tables + TAB_X2N;
+  if (d.nseg == 1) {
+    if (lane == 0) {
+      const uint64_t len = d.bytes;
+      const uint32_t zi = (len == p.chunk_bytes) ? p.zinit_c : crc_shift(0xFFFFFFFFu, len, x2n);
+      chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ S)));
+    }
+    return;
+  }
+  uint32_t prev = 0;
+  if (lane == 0) {
+    p.partial[idx] = S;
+    __threadfence();
+    prev = atomicAdd(p.arrive + d.chunk, 1u);
+  }
+  prev = __shfl_sync(0xffffffffu, prev, 0);
+  if (prev != d.nseg - 1) return;
+  __threadfence();
+  const uint32_t nseg = d.nseg, first = idx - d.seg;
+  const uint32_t last_len = __ldcg(&p.desc[first + nseg - 1].bytes);
+  const uint32_t k = (nseg + 31) / 32;
+  const uint32_t a = min((uint32_t)lane * k, nseg), b = min(a + k, nseg);
+  uint32_t X = 0;
+  if (a < b) {
+    uint32_t H = 0;
+    for (uint32_t s = a; s < b; ++s) {
+      const uint32_t f = __ldcg(p.partial + first + s);
+      if (s == a) H = f;
+      else if (s + 1 < nseg || last_len == p.seg_bytes) H = multmodp(p.xseg, H) ^ f;
+      else H = crc_shift(H, last_len, x2n) ^ f;
+    }
+    if (b < nseg) {  // past segments b .. nseg-2 (whole) and nseg-1 (last_len bytes)
+      const uint32_t m = nseg - 1 - b;
+      H = m < (uint32_t)ZS_N ? multmodp(__ldg(p.tables + TAB_ZS + m), H) : crc_shift(H, (uint64_t)m * p.seg_bytes, x2n);
+      H = last_len == p.seg_bytes ? multmodp(p.xseg, H) : crc_shift(H, last_len, x2n);
+    }
+    X = H;
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) X ^= __shfl_xor_sync(0xffffffffu, X, o);
+  if (lane == 0) {
+    p.arrive[d.chunk] = 0;
+    const uint64_t L = (uint64_t)(nseg - 1) * p.seg_bytes + last_len;
+    const uint32_t zi = (L == p.chunk_bytes) ? p.zinit_c : crc_shift(0xFFFFFFFFu, L, x2n);
+    chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ X)));
   }
 }
 
@@ -335,39 +391,10 @@ __device__ __forceinline__ void move_segment(const Params& p, const SegDesc& d, 
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) X ^= __shfl_xor_sync(0xffffffffu, X, o);
   if (r) stage_tail<MODE>(src + base, COPY ? dst + base : nullptr, r, tail, lane);
-  if (lane == 0) {
-    uint32_t S = X;  // continue the register through the tail: F(X, tail) = F(0, full || tail)
+  uint32_t S = X;  // lane 0 continues the register through the tail: F(X, tail) = F(0, full || tail)
+  if (lane == 0)
     for (uint32_t i = 0; i < r; ++i) S = sT[(S ^ tail[i]) & 0xFFu] ^ (S >> 8);
-    const uint32_t* x2n = p.tables + TAB_X2N;
-    if (d.nseg == 1) {
-      const uint32_t zi = (len == p.chunk_bytes) ? p.zinit_c : crc_shift(0xFFFFFFFFu, len, x2n);
-      chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ S)));
-      return;
-    }
-    p.partial[idx] = S;
-    __threadfence();
-    const uint32_t prev = atomicAdd(p.arrive + d.chunk, 1u);
-    if (prev == d.nseg - 1) {  // last arriver combines the chunk's segments in order
-      __threadfence();
-      const uint32_t first = idx - d.seg;
-      const uint32_t last_len = __ldcg(&p.desc[first + d.nseg - 1].bytes);
-      uint32_t acc = 0;
-      for (uint32_t s = 0; s < d.nseg; ++s) {
-        const uint32_t f = __ldcg(p.partial + first + s);
-        if (s == 0) {
-          acc = f;
-        } else if (s + 1 < d.nseg || last_len == p.seg_bytes) {
-          acc = multmodp(p.xseg, acc) ^ f;
-        } else {
-          acc = crc_shift(acc, last_len, x2n) ^ f;
-        }
-      }
-      p.arrive[d.chunk] = 0;
-      const uint64_t L = (uint64_t)(d.nseg - 1) * p.seg_bytes + last_len;
-      const uint32_t zi = (L == p.chunk_bytes) ? p.zinit_c : crc_shift(0xFFFFFFFFu, L, x2n);
-      chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ acc)));
-    }
-  }
+  crc_segment_done<MODE>(p, d, idx, S, lane);
 }
 
 // ------------------------------------------------------------------ the persistent kernel
@@ -587,32 +614,7 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
       }
 #pragma unroll
       for (int s = 16; s > 0; s >>= 1) X ^= __shfl_xor_sync(0xffffffffu, X, s);
-      if (lane == 0) {
-        if (d.nseg == 1) {
-          const uint32_t zi = (len == p.chunk_bytes) ? p.zinit_c : crc_shift(0xFFFFFFFFu, len, x2n);
-          chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ X)));
-        } else {
-          p.partial[idx] = X;
-          __threadfence();
-          const uint32_t prev = atomicAdd(p.arrive + d.chunk, 1u);
-          if (prev == d.nseg - 1) {
-            __threadfence();
-            const uint32_t first = idx - d.seg;
-            const uint32_t last_len = __ldcg(&p.desc[first + d.nseg - 1].bytes);
-            uint32_t acc = 0;
-            for (uint32_t s = 0; s < d.nseg; ++s) {
-              const uint32_t f = __ldcg(p.partial + first + s);
-              if (s == 0) acc = f;
-              else if (s + 1 < d.nseg || last_len == p.seg_bytes) acc = multmodp(p.xseg, acc) ^ f;
-              else acc = crc_shift(acc, last_len, x2n) ^ f;
-            }
-            p.arrive[d.chunk] = 0;
-            const uint64_t L = (uint64_t)(d.nseg - 1) * p.seg_bytes + last_len;
-            const uint32_t zi = (L == p.chunk_bytes) ? p.zinit_c : crc_shift(0xFFFFFFFFu, L, x2n);
-            chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ acc)));
-          }
-        }
-      }
+      crc_segment_done<MODE>(p, d, idx, X, lane);
     }
     __syncthreads();
     if (tid == 0 && r + 2 < rounds) {

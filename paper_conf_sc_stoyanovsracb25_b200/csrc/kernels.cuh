@@ -41,7 +41,9 @@ constexpr int TAB_LANE = TAB_Z496 + 4 * 256;  // [32] x^(8*16*(31-l)) mod P
 constexpr int TAB_X2N = TAB_LANE + 32;        // [32] x^(2^k) mod P
 constexpr int TAB_HLANE = TAB_X2N + 32;       // [32] hash kernel: Z^(L1 - end_l) for the common segment length L1
 constexpr int TAB_Z96N = TAB_HLANE + 32;       // [8][16] hash kernel: Z^96 of nibble v at position k
-constexpr int TAB_WORDS = TAB_Z96N + 128;
+constexpr int ZS_N = 1024;
+constexpr int TAB_ZS = TAB_Z96N + 128;         // [ZS_N] x^(8*m*seg) mod P: shift by m whole segments
+constexpr int TAB_WORDS = TAB_ZS + ZS_N;
 constexpr int TAB_SMEM_WORDS = TAB_LANE + 32;  // the part staged in shared memory
 
 struct Params {
@@ -61,7 +63,7 @@ struct Params {
   uint32_t hlane_len;            // L1: the segment length TAB_HLANE was built for
 };
 
-void build_tables(uint32_t* tab /* TAB_WORDS */, uint64_t common_seg_len);
+void build_tables(uint32_t* tab /* TAB_WORDS */, uint64_t common_seg_len, uint64_t seg_bytes);
 // Quad-line geometry of the CRC-32C HBM hash kernel for a segment of `len` bytes: 8 strands (one per
 // lane quad) of hash_strand(len) bytes (a multiple of 128); lane (q = lane/4, j = lane%4) owns the 32-B
 // pieces at q*Ls + j*32 + t*128 that start inside its strand and the segment.

@@ -316,7 +316,7 @@ void free_set(DescSet& S) {
 // depend on min(C, seg)); uploads them and derives the init / segment shift constants.
 swap_status upload_tables(swap_ctx* c) {
   std::vector<uint32_t> tab(swk::TAB_WORDS);
-  swk::build_tables(tab.data(), std::min<uint64_t>(c->cfg.chunk_bytes, c->seg));
+  swk::build_tables(tab.data(), std::min<uint64_t>(c->cfg.chunk_bytes, c->seg), c->seg);
   if (!c->d_tables) CUDA_TRY(c, cudaMalloc(&c->d_tables, tab.size() * 4));
   CUDA_TRY(c, cudaMemcpy(c->d_tables, tab.data(), tab.size() * 4, cudaMemcpyHostToDevice));
   const uint32_t* x2n = tab.data() + swk::TAB_X2N;
