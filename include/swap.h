@@ -58,8 +58,9 @@ typedef int32_t swap_status;
 #define SWAP_CHECKSUM_XXH64 2u  /* XXH64, seed 0 for every chunk */
 
 /* Data mover for checkpoint/restore (the image bytes are identical for all of them): */
-#define SWAP_MECH_AUTO 0u        /* default: SWAP_MECH_CE_PIPE when the payload is >= 1 GiB (and, for XXH64,
-                                    chunk_bytes <= 1 MiB), else SWAP_MECH_SM (DESIGN.md §6 mechanism sweep) */
+#define SWAP_MECH_AUTO 0u        /* default, resolved per call from the measured crossover: restore
+                                    SM < 128 MiB, CE_BATCH < 2 GiB (SM on the legacy default stream), else
+                                    CE_PIPE; checkpoint SM < 1 GiB, else CE_PIPE; XXH64 with chunks > 1 MiB: SM */
 #define SWAP_MECH_SM 1u          /* one SM kernel: 16-B vector loads/stores to mapped pinned host memory with the
                                     chunk checksum fused from the same registers (one pass, bytes checked in flight) */
 #define SWAP_MECH_CE_REGION 2u   /* copy engine: cudaMemcpyAsync per region + separate HBM hash pass */
@@ -179,7 +180,7 @@ SWAP_API swap_status swap_set_region_policy(swap_ctx_t* ctx, uint32_t region_ind
 
 /* Selects the data mover for later calls (SWAP_MECH_*). The image format is unchanged. */
 SWAP_API swap_status swap_set_mechanism(swap_ctx_t* ctx, uint32_t mechanism);
-/* The mechanism the next checkpoint/restore will use (SWAP_MECH_AUTO resolved; needs REGISTERED+). */
+/* The mechanism the next restore on a non-default stream will use (SWAP_MECH_AUTO resolved; REGISTERED+). */
 SWAP_API swap_status swap_get_mechanism(const swap_ctx_t* ctx, uint32_t* effective);
 
 /* Borrowed views, valid until swap_destroy. The manifest is final only after swap_sync.

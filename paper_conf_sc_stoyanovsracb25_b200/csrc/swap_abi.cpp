@@ -82,6 +82,7 @@ struct swap_ctx {
   uint32_t* d_tables = nullptr;
   uint32_t zinit_c = 0, xseg = 0;
   uint32_t seg = 0;  // CRC-32C segment size in use (cfg.seg_bytes, or chosen at registration when 0)
+  uint32_t cur_mech = SWAP_MECH_SM;  // mechanism of the call in progress (resolve_mech)
   cudaEvent_t ev[6] = {};  // checkpoint, restore, verify: begin/end pairs
   bool pending[3] = {false, false, false};
   float ms[3] = {0.f, 0.f, 0.f};
@@ -139,18 +140,23 @@ swk::Params base_params(swap_ctx* c, const DescSet& S) {
 
 int grid_of(swap_ctx* c) { return c->cfg.grid_ctas ? (int)c->cfg.grid_ctas : 2 * c->sm_count; }
 
-// The mechanism actually used: AUTO picks the copy-engine pipeline for large images (the copy
-// engines reach a higher link rate than SM-issued accesses) and the single fused
-// SM pass for small ones (no per-copy launch overhead).
-constexpr uint64_t kAutoPipeBytes = 1ull << 30;  // crossover measured: 1 GiB ties, 4 GiB CE_PIPE +5 %, <= 256 MiB SM
-// XXH64 is not combinable: with chunks > 1 MiB a pipeline group holds too few chunks for the
-// side-stream hash to keep up with the link, while the fused SM pass hashes every chunk in flight.
-uint32_t mech(const swap_ctx* c) {
+// The mechanism a call uses. AUTO resolves per direction from the measured crossover (DESIGN.md §6,
+// `profiles/r01_crossover.md`): the copy engines reach a higher link rate than SM-issued accesses, but
+// per-copy and per-launch costs make the single fused SM pass faster for small images.
+//   restore:    < 128 MiB SM;  < 2 GiB CE_BATCH (needs a non-default stream, else SM);  else CE_PIPE
+//   checkpoint: < 1 GiB SM;    else CE_PIPE
+// XXH64 is not combinable: with chunks > 1 MiB a pipeline group holds too few chunks for the side-stream
+// hash to keep up with the link, while the fused SM pass hashes every chunk in flight — SM then.
+uint32_t resolve_mech(const swap_ctx* c, int dir, bool default_stream) {
   if (c->cfg.mechanism != SWAP_MECH_AUTO) return c->cfg.mechanism;
-  if (c->plan.payload_bytes < kAutoPipeBytes) return SWAP_MECH_SM;
+  const uint64_t S = c->plan.payload_bytes;
   if (c->plan.kind == SWAP_CHECKSUM_XXH64 && c->plan.C > (1ull << 20)) return SWAP_MECH_SM;
+  if (dir == 0) return S < (1ull << 30) ? SWAP_MECH_SM : SWAP_MECH_CE_PIPE;
+  if (S < (128ull << 20)) return SWAP_MECH_SM;
+  if (S < (2ull << 30)) return default_stream ? SWAP_MECH_SM : SWAP_MECH_CE_BATCH;
   return SWAP_MECH_CE_PIPE;
 }
+uint32_t mech(const swap_ctx* c) { return c->cur_mech; }
 int kind_of(swap_ctx* c) {
   if (mech(c) == SWAP_MECH_SM_NOCHECK) return swk::KIND_NONE;
   return c->plan.kind == SWAP_CHECKSUM_XXH64 ? swk::KIND_XXH64 : swk::KIND_CRC32C;
@@ -613,6 +619,7 @@ swap_status swap_checkpoint(swap_ctx_t* c, swap_stream_t stream) {
   }
   DeviceGuard g(c->cfg.device);
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  c->cur_mech = resolve_mech(c, 0, s == nullptr);
   // SAVE_ONCE regions are gathered by the first checkpoint only; DISCARD regions never (their image
   // bytes stay zero and their c_g are the checksums of zero chunks, hashed once from a zero buffer).
   DescSet& S = c->first_ckpt_done ? c->s_save : c->s_move;
@@ -663,6 +670,7 @@ swap_status swap_restore(swap_ctx_t* c, swap_stream_t stream) {
   if (st != SWAP_OK) return st;
   DeviceGuard g(c->cfg.device);
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  c->cur_mech = resolve_mech(c, 1, s == nullptr);
   DescSet& S = c->s_move;
   swk::Params p = base_params(c, S);
   CUDA_TRY(c, cudaMemsetAsync(&c->d_status->n_bad, 0, 8, s));
@@ -980,7 +988,7 @@ swap_status swap_set_mechanism(swap_ctx_t* c, uint32_t mechanism) {
 swap_status swap_get_mechanism(const swap_ctx_t* c, uint32_t* effective) {
   if (!c || !effective) return SWAP_EINVAL;
   if (c->st == St::CREATED) return SWAP_ESTATE;
-  *effective = mech(c);
+  *effective = resolve_mech(c, 1, false);
   return SWAP_OK;
 }
 
