@@ -12,8 +12,9 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libswap.so")
-SOURCES = ["kernels.cu", "plan.cpp", "swap_abi.cpp", "arena.cpp", "sched.cpp", "storage.cpp"]
-HEADERS = ["kernels.cuh", "plan.h", "arena.h"]
+SOURCES = ["kernels.cu", "plan.cpp", "swap_abi.cpp", "movers.cpp", "exchange.cpp", "arena.cpp", "sched.cpp",
+           "storage.cpp"]
+HEADERS = ["kernels.cuh", "plan.h", "arena.h", "ctx.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

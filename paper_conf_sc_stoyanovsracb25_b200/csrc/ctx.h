@@ -1,0 +1,127 @@
+// ctx.h — libswap-internal context (the opaque swap_ctx of include/swap.h) and the helpers shared by
+// the ABI (swap_abi.cpp), the movers (movers.cpp) and the exchange / assisted restore (exchange.cpp).
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "arena.h"
+#include "kernels.cuh"
+#include "plan.h"
+
+namespace swc {
+enum class St { CREATED, REGISTERED, CKPT_PENDING, CHECKPOINTED, RESTORED };
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+}  // namespace swc
+
+struct Span {  // one copy-engine transfer: contiguous on the device and in the image
+  uint64_t dev;
+  uint8_t* host;
+  uint64_t bytes;
+};
+struct Group {  // CE_PIPE unit: whole chunks, descriptor range [d0, d1)
+  uint32_t d0, d1;
+  std::vector<Span> spans;
+};
+
+// The work of one pass over a subset of the regions (selected by their swap policy): segment
+// descriptors on the device plus the copy-engine views of the same bytes. A chunk's segments are
+// always contiguous, so per-chunk CRC combining works on any set.
+struct DescSet {
+  swk::SegDesc* d_desc = nullptr;
+  uint32_t n_desc = 0;
+  std::vector<Span> region_spans;         // CE_REGION
+  std::vector<void*> ce_dev, ce_host;     // CE_CHUNK / CE_BATCH, one entry per chunk
+  std::vector<size_t> ce_bytes;
+  std::vector<Group> groups;              // CE_PIPE
+  std::vector<cudaEvent_t> group_ev;
+  bool owned = false;                     // false: an alias of another set
+};
+
+struct swap_ctx {
+  swap_config_t cfg{};
+  swc::St st = swc::St::CREATED;
+  int sm_count = 0;
+  swp::Plan plan;
+  // host image: mmap'd, pinned + mapped with cudaHostRegister (library-owned)
+  uint8_t* image = nullptr;
+  size_t map_bytes = 0;
+  bool host_registered = false;
+  uint8_t* image_dev = nullptr;  // device (UVA) view of the image
+  // device-side work state; sets: all regions (verify), SAVE|SAVE_ONCE (first checkpoint, restore),
+  // SAVE (later checkpoints), DISCARD chunks hashed from a zero buffer (their c_g)
+  std::vector<uint32_t> policy;
+  DescSet s_all, s_move, s_save, s_zero;
+  bool first_ckpt_done = false;
+  uint8_t* d_zero = nullptr;
+  uint32_t* d_partial = nullptr;
+  uint32_t* d_arrive = nullptr;
+  swk::DevStatus* d_status = nullptr;
+  swk::DevStatus* h_status = nullptr;  // pinned
+  uint32_t* d_tables = nullptr;
+  uint32_t zinit_c = 0, xseg = 0;
+  uint32_t seg = 0;  // CRC-32C segment size in use (cfg.seg_bytes, or chosen at registration when 0)
+  uint32_t cur_mech = SWAP_MECH_SM;  // mechanism of the call in progress (resolve_mech)
+  cudaEvent_t ev[6] = {};  // checkpoint, restore, verify: begin/end pairs
+  bool pending[3] = {false, false, false};
+  float ms[3] = {0.f, 0.f, 0.f};
+  uint64_t launches = 0;
+  std::string err;
+  std::vector<swap_shard_summary_t> global;
+  // CE_PIPE
+  cudaStream_t side = nullptr;
+  swap_arena* arena = nullptr;  // bound arena: restore re-acquires its HBM (swap_bind_arena)
+  // NVLink-assisted restore (swap_set_helpers): peers pull groups over their own PCIe links into
+  // HBM staging and copy them to this device over NVLink
+  struct Helper {
+    int dev = -1;
+    cudaStream_t s = nullptr;
+    uint8_t* staging = nullptr;
+    cudaEvent_t ev = nullptr, done = nullptr;
+  };
+  std::vector<Helper> helpers;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+};
+
+namespace swc {
+
+#define CUDA_TRY(ctx, expr)                                    \
+  do {                                                         \
+    cudaError_t e_ = (expr);                                   \
+    if (e_ != cudaSuccess) return cuda_fail((ctx), e_, #expr); \
+  } while (0)
+
+swap_status cuda_fail(swap_ctx* c, cudaError_t e, const char* what);
+uint8_t* manifest_ptr(swap_ctx* c);
+swk::Params base_params(swap_ctx* c, const DescSet& S);
+int grid_of(swap_ctx* c);
+uint32_t resolve_mech(const swap_ctx* c, int dir, bool default_stream);
+uint32_t mech(const swap_ctx* c);
+int kind_of(swap_ctx* c);
+int hash_kind(swap_ctx* c);
+swap_status launch(swap_ctx* c, int mode, int kind, const swk::Params& p, cudaStream_t s);
+swap_status memcpy_dir(swap_ctx* c, const Span& sp, int dir, cudaStream_t s);
+swap_status ce_copy(swap_ctx* c, DescSet& S, int dir, cudaStream_t s);
+swap_status map_spans(swap_ctx* c, const std::vector<Span>& spans);
+swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, cudaStream_t s);
+swap_status collect_timing(swap_ctx* c, int p);
+bool is_ce(uint32_t m);
+void free_set(DescSet& S);
+swap_status upload_tables(swap_ctx* c);
+uint32_t auto_seg(const swap_ctx* c, uint64_t payload);
+void free_helpers(swap_ctx* c);
+void release(swap_ctx* c);
+swap_status build_sets(swap_ctx* c);
+
+}  // namespace swc

@@ -1,0 +1,398 @@
+// movers.cpp — libswap internals: kernel launches, copy-engine movers, the CE_PIPE pipeline, the
+// descriptor sets of the region policies, CRC tables and context teardown (see ctx.h).
+#include <sys/mman.h>
+
+#include <algorithm>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "ctx.h"
+
+namespace swc {
+swap_status cuda_fail(swap_ctx* c, cudaError_t e, const char* what) {
+  c->err = std::string(what) + ": " + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ")";
+  return SWAP_ECUDA;
+}
+
+uint8_t* manifest_ptr(swap_ctx* c) { return c->image + c->plan.manifest_off; }
+
+swk::Params base_params(swap_ctx* c, const DescSet& S) {
+  swk::Params p{};
+  p.desc = S.d_desc;
+  p.n_desc = S.n_desc;
+  p.seg_bytes = c->seg;
+  p.partial = c->d_partial;
+  p.arrive = c->d_arrive;
+  const uint64_t cs_off = c->plan.manifest_off + swp::kHeaderBytes + swp::kRegionRecBytes * c->plan.regions.size() + 24;
+  p.cs_out = reinterpret_cast<uint64_t*>(c->image_dev + cs_off);
+  p.cs_exp = p.cs_out;
+  p.n_bad = &c->d_status->n_bad;
+  p.first_bad = &c->d_status->first_bad;
+  p.tables = c->d_tables;
+  p.chunk_bytes = c->plan.C;
+  p.zinit_c = c->zinit_c;
+  p.xseg = c->xseg;
+  p.hlane_len = (uint32_t)std::min<uint64_t>(c->plan.C, c->seg);
+  return p;
+}
+
+int grid_of(swap_ctx* c) { return c->cfg.grid_ctas ? (int)c->cfg.grid_ctas : 2 * c->sm_count; }
+
+// The mechanism a call uses. AUTO resolves per direction from the measured crossover (DESIGN.md §6,
+// `profiles/r01_crossover.md`): the copy engines reach a higher link rate than SM-issued accesses, but
+// per-copy and per-launch costs make the single fused SM pass faster for small images.
+//   restore:    < 128 MiB SM;  < 2 GiB CE_BATCH (needs a non-default stream, else SM);  else CE_PIPE
+//   checkpoint: < 1 GiB SM;    else CE_PIPE
+// XXH64 is not combinable: with chunks > 1 MiB a pipeline group holds too few chunks for the side-stream
+// hash to keep up with the link, while the fused SM pass hashes every chunk in flight — SM then.
+uint32_t resolve_mech(const swap_ctx* c, int dir, bool default_stream) {
+  if (c->cfg.mechanism != SWAP_MECH_AUTO) return c->cfg.mechanism;
+  const uint64_t S = c->plan.payload_bytes;
+  if (c->plan.kind == SWAP_CHECKSUM_XXH64 && c->plan.C > (1ull << 20)) return SWAP_MECH_SM;
+  if (dir == 0) return S < (1ull << 30) ? SWAP_MECH_SM : SWAP_MECH_CE_PIPE;
+  if (S < (128ull << 20)) return SWAP_MECH_SM;
+  if (S < (2ull << 30)) return default_stream ? SWAP_MECH_SM : SWAP_MECH_CE_BATCH;
+  return SWAP_MECH_CE_PIPE;
+}
+uint32_t mech(const swap_ctx* c) { return c->cur_mech; }
+int kind_of(swap_ctx* c) {
+  if (mech(c) == SWAP_MECH_SM_NOCHECK) return swk::KIND_NONE;
+  return c->plan.kind == SWAP_CHECKSUM_XXH64 ? swk::KIND_XXH64 : swk::KIND_CRC32C;
+}
+int hash_kind(swap_ctx* c) { return c->plan.kind == SWAP_CHECKSUM_XXH64 ? swk::KIND_XXH64 : swk::KIND_CRC32C; }
+
+swap_status launch(swap_ctx* c, int mode, int kind, const swk::Params& p, cudaStream_t s) {
+  if (p.n_desc == 0) return SWAP_OK;
+  // never more CTAs than descriptor batches (idle CTAs would only load tables)
+  int want = (int)std::min<uint64_t>((uint64_t)grid_of(c), (p.n_desc + 15) / 16);
+  if ((mode == swk::HASH_STORE || mode == swk::HASH_CHECK) && kind == swk::KIND_CRC32C)
+    want = c->cfg.grid_ctas ? std::min<int>(want, (int)c->cfg.grid_ctas) : swk::hash_grid(c->sm_count, p.n_desc);
+  cudaError_t e;
+  if ((mode == swk::HASH_STORE || mode == swk::HASH_CHECK) && kind == swk::KIND_XXH64 && !c->cfg.grid_ctas)
+    e = swk::launch_xxh_hash(mode, p, c->sm_count, s);
+  else
+    e = swk::launch_mover(mode, kind, p, std::max(1, want), s);
+  if (e != cudaSuccess) return cuda_fail(c, e, "mover kernel launch");
+  ++c->launches;
+  return SWAP_OK;
+}
+
+swap_status memcpy_dir(swap_ctx* c, const Span& sp, int dir, cudaStream_t s) {
+  void* dev = reinterpret_cast<void*>(sp.dev);
+  CUDA_TRY(c, dir == 0 ? cudaMemcpyAsync(sp.host, dev, sp.bytes, cudaMemcpyDeviceToHost, s)
+                       : cudaMemcpyAsync(dev, sp.host, sp.bytes, cudaMemcpyHostToDevice, s));
+  return SWAP_OK;
+}
+
+// Copy-engine data movement for CE_REGION / CE_CHUNK / CE_BATCH: dir 0 = device -> image, 1 = image -> device.
+swap_status ce_copy(swap_ctx* c, DescSet& S, int dir, cudaStream_t s) {
+  const uint32_t m = mech(c);
+  if (m == SWAP_MECH_CE_REGION) {
+    for (const Span& sp : S.region_spans) {
+      swap_status st = memcpy_dir(c, sp, dir, s);
+      if (st != SWAP_OK) return st;
+    }
+    return SWAP_OK;
+  }
+  if (m == SWAP_MECH_CE_CHUNK) {
+    for (size_t i = 0; i < S.ce_bytes.size(); ++i) {
+      Span sp{reinterpret_cast<uint64_t>(S.ce_dev[i]), static_cast<uint8_t*>(S.ce_host[i]), S.ce_bytes[i]};
+      swap_status st = memcpy_dir(c, sp, dir, s);
+      if (st != SWAP_OK) return st;
+    }
+    return SWAP_OK;
+  }
+  // CE_BATCH: one cudaMemcpyBatchAsync over every chunk.
+  if (s == nullptr) {
+    c->err = "SWAP_MECH_CE_BATCH needs a non-default stream (cudaMemcpyBatchAsync restriction)";
+    return SWAP_EUNSUPPORTED;
+  }
+  if (S.ce_bytes.empty()) return SWAP_OK;
+  cudaMemcpyAttributes attr;
+  std::memset(&attr, 0, sizeof(attr));
+  attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
+  attr.srcLocHint.type = dir == 0 ? cudaMemLocationTypeDevice : cudaMemLocationTypeHost;
+  attr.srcLocHint.id = dir == 0 ? c->cfg.device : 0;
+  attr.dstLocHint.type = dir == 0 ? cudaMemLocationTypeHost : cudaMemLocationTypeDevice;
+  attr.dstLocHint.id = dir == 0 ? 0 : c->cfg.device;
+  size_t attr_idx = 0, fail_idx = 0;
+  std::vector<void*>& dst = dir == 0 ? S.ce_host : S.ce_dev;
+  std::vector<void*>& src = dir == 0 ? S.ce_dev : S.ce_host;
+  CUDA_TRY(c, cudaMemcpyBatchAsync(dst.data(), src.data(), S.ce_bytes.data(), S.ce_bytes.size(), &attr, &attr_idx, 1,
+                                   &fail_idx, s));
+  return SWAP_OK;
+}
+
+// Re-acquires the bound arena's slabs under `spans` (no-op without an arena or when resident).
+swap_status map_spans(swap_ctx* c, const std::vector<Span>& spans) {
+  if (!c->arena || swarena::resident(c->arena)) return SWAP_OK;
+  for (const Span& sp : spans) {
+    if (!swarena::contains(c->arena, sp.dev, sp.dev + sp.bytes)) continue;
+    swap_status st = swarena::map_dev_range(c->arena, sp.dev, sp.dev + sp.bytes);
+    if (st != SWAP_OK) {
+      c->err = "re-acquiring arena HBM failed";
+      return st;
+    }
+  }
+  return SWAP_OK;
+}
+
+// CE_PIPE. Checkpoint (dir 0): the hash pass over HBM runs on the side stream concurrently with the
+// D2H copies (both only read HBM). Restore (dir 1): group g's H2D copies are followed by an event;
+// the side stream waits for it and checks group g from HBM while the copy engine moves group g+1.
+swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, cudaStream_t s) {
+  CUDA_TRY(c, cudaEventRecord(c->ev_fork, s));
+  CUDA_TRY(c, cudaStreamWaitEvent(c->side, c->ev_fork, 0));
+  swap_status st;
+  if (dir == 0 && (st = launch(c, swk::HASH_STORE, hash_kind(c), base, c->side)) != SWAP_OK) return st;
+  const size_t H = dir == 1 ? c->helpers.size() : 0;
+  for (auto& h : c->helpers)
+    if (H) CUDA_TRY(c, cudaStreamWaitEvent(h.s, c->ev_fork, 0));
+  for (size_t g = 0; g < S.groups.size(); ++g) {
+    const Group& G = S.groups[g];
+    if (dir == 1 && (st = map_spans(c, G.spans)) != SWAP_OK) return st;  // lazy HBM re-acquire
+    const size_t k = H ? g % (H + 1) : 0;
+    if (k > 0) {
+      // helper k-1: H2D of the group's image range into its staging over its own PCIe link, then
+      // NVLink peer copies of each span to this device; the side stream checks it as usual
+      auto& h = c->helpers[k - 1];
+      uint8_t* lo = G.spans.front().host;
+      uint8_t* hi = G.spans.back().host + G.spans.back().bytes;
+      CUDA_TRY(c, cudaSetDevice(h.dev));
+      CUDA_TRY(c, cudaMemcpyAsync(h.staging, lo, (size_t)(hi - lo), cudaMemcpyHostToDevice, h.s));
+      for (const Span& sp : G.spans)
+        CUDA_TRY(c, cudaMemcpyPeerAsync(reinterpret_cast<void*>(sp.dev), c->cfg.device, h.staging + (sp.host - lo), h.dev,
+                                        sp.bytes, h.s));
+      CUDA_TRY(c, cudaEventRecord(h.ev, h.s));
+      CUDA_TRY(c, cudaSetDevice(c->cfg.device));
+      CUDA_TRY(c, cudaStreamWaitEvent(c->side, h.ev, 0));
+      swk::Params p = base;
+      p.desc = base.desc + G.d0;
+      p.partial = base.partial + G.d0;
+      p.n_desc = G.d1 - G.d0;
+      if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, c->side)) != SWAP_OK) return st;
+      continue;
+    }
+    for (const Span& sp : G.spans)
+      if ((st = memcpy_dir(c, sp, dir, s)) != SWAP_OK) return st;
+    if (dir == 1) {
+      CUDA_TRY(c, cudaEventRecord(S.group_ev[g], s));
+      CUDA_TRY(c, cudaStreamWaitEvent(c->side, S.group_ev[g], 0));
+      swk::Params p = base;
+      p.desc = base.desc + G.d0;
+      p.partial = base.partial + G.d0;
+      p.n_desc = G.d1 - G.d0;
+      if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, c->side)) != SWAP_OK) return st;
+    }
+  }
+  for (auto& h : c->helpers) {
+    if (!H) break;
+    CUDA_TRY(c, cudaSetDevice(h.dev));
+    CUDA_TRY(c, cudaEventRecord(h.done, h.s));
+    CUDA_TRY(c, cudaSetDevice(c->cfg.device));
+    CUDA_TRY(c, cudaStreamWaitEvent(s, h.done, 0));
+  }
+  CUDA_TRY(c, cudaEventRecord(c->ev_join, c->side));
+  CUDA_TRY(c, cudaStreamWaitEvent(s, c->ev_join, 0));
+  return SWAP_OK;
+}
+
+// Phase p: 0 checkpoint, 1 restore, 2 verify. Call after the stream has been synchronised.
+swap_status collect_timing(swap_ctx* c, int p) {
+  if (!c->pending[p]) return SWAP_OK;
+  CUDA_TRY(c, cudaEventElapsedTime(&c->ms[p], c->ev[2 * p], c->ev[2 * p + 1]));
+  c->pending[p] = false;
+  return SWAP_OK;
+}
+
+bool is_ce(uint32_t m) { return m == SWAP_MECH_CE_REGION || m == SWAP_MECH_CE_CHUNK || m == SWAP_MECH_CE_BATCH; }
+
+void free_set(DescSet& S) {
+  if (S.owned) {
+    if (S.d_desc) cudaFree(S.d_desc);
+    for (auto& e : S.group_ev)
+      if (e) cudaEventDestroy(e);
+  }
+  S = DescSet();
+}
+
+// CRC tables for the ctx's chunk and segment sizes (the hash kernels fold lanes with constants that
+// depend on min(C, seg)); uploads them and derives the init / segment shift constants.
+swap_status upload_tables(swap_ctx* c) {
+  std::vector<uint32_t> tab(swk::TAB_WORDS);
+  swk::build_tables(tab.data(), std::min<uint64_t>(c->cfg.chunk_bytes, c->seg), c->seg);
+  if (!c->d_tables) CUDA_TRY(c, cudaMalloc(&c->d_tables, tab.size() * 4));
+  CUDA_TRY(c, cudaMemcpy(c->d_tables, tab.data(), tab.size() * 4, cudaMemcpyHostToDevice));
+  const uint32_t* x2n = tab.data() + swk::TAB_X2N;
+  c->zinit_c = swk::host_multmodp(swk::host_x2nmodp(c->cfg.chunk_bytes, 3, x2n), 0xFFFFFFFFu);
+  c->xseg = swk::host_x2nmodp(c->seg, 3, x2n);
+  return SWAP_OK;
+}
+
+// Auto segment size: enough CRC work items to give every warp slot of the GPU (SMs x 32) one, between
+// 4 KiB and 256 KiB (large images keep 256 KiB; a 64 MiB image gets 8 KiB).
+uint32_t auto_seg(const swap_ctx* c, uint64_t payload) {
+  const uint64_t per = payload / ((uint64_t)c->sm_count * 32 + 1);
+  uint64_t s = 4096;
+  while (s * 2 <= per && s < (256u << 10)) s *= 2;
+  return (uint32_t)s;
+}
+
+void free_helpers(swap_ctx* c) {
+  int cur = -1;
+  cudaGetDevice(&cur);
+  for (auto& h : c->helpers) {
+    cudaSetDevice(h.dev);
+    if (h.s) cudaStreamSynchronize(h.s);
+    if (h.staging) cudaFree(h.staging);
+    if (h.ev) cudaEventDestroy(h.ev);
+    if (h.done) cudaEventDestroy(h.done);
+    if (h.s) cudaStreamDestroy(h.s);
+  }
+  c->helpers.clear();
+  if (cur >= 0) cudaSetDevice(cur);
+}
+
+void release(swap_ctx* c) {
+  free_helpers(c);
+  free_set(c->s_move);
+  free_set(c->s_save);
+  free_set(c->s_zero);
+  free_set(c->s_all);
+  if (c->d_zero) cudaFree(c->d_zero);
+  c->d_zero = nullptr;
+  if (c->d_partial) cudaFree(c->d_partial);
+  if (c->d_arrive) cudaFree(c->d_arrive);
+  if (c->d_status) cudaFree(c->d_status);
+  if (c->h_status) cudaFreeHost(c->h_status);
+  if (c->d_tables) cudaFree(c->d_tables);
+  for (auto& e : c->ev)
+    if (e) cudaEventDestroy(e);
+  if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+  if (c->ev_join) cudaEventDestroy(c->ev_join);
+  if (c->side) cudaStreamDestroy(c->side);
+  if (c->host_registered) cudaHostUnregister(c->image);
+  if (c->image) munmap(c->image, c->map_bytes);
+  c->d_partial = nullptr;
+  c->image = nullptr;
+}
+
+// Builds the descriptor set of the regions `pick` selects. zero_src: segment sources point into
+// the zero buffer instead of the region (hashing DISCARD chunks as zeros).
+template <class Pick>
+static swap_status build_set(swap_ctx* c, DescSet* S, Pick pick, bool zero_src) {
+  const swp::Plan& P = c->plan;
+  const uint64_t seg = P.kind == SWAP_CHECKSUM_XXH64 ? P.C : std::min<uint64_t>(P.C, c->seg);
+  std::vector<swk::SegDesc> desc;
+  // group size: cfg.pipe_mib, or auto = payload / 32 clamped to [16 MiB, 256 MiB] (smaller groups cost
+  // more in per-copy and per-launch overhead than they gain in overlap)
+  uint64_t target = (uint64_t)c->cfg.pipe_mib << 20;
+  if (!target) target = std::min<uint64_t>(256ull << 20, std::max<uint64_t>(16ull << 20, c->plan.payload_bytes / 32));
+  Group cur{0, 0, {}};
+  uint64_t cur_bytes = 0;
+  for (size_t i = 0; i < P.regions.size(); ++i) {
+    const auto& r = P.regions[i];
+    if (!pick(i) || r.r.bytes == 0) continue;
+    S->region_spans.push_back(Span{r.r.dev_addr, c->image + r.off, r.r.bytes});
+    for (uint64_t j = 0; j < r.nchunks; ++j) {
+      const uint64_t lo = j * P.C, len = std::min<uint64_t>(P.C, r.r.bytes - lo);
+      const uint32_t nseg = (uint32_t)((len + seg - 1) / seg);
+      for (uint32_t s = 0; s < nseg; ++s) {
+        swk::SegDesc d;
+        d.dev = zero_src ? reinterpret_cast<uint64_t>(c->d_zero) + s * seg : r.r.dev_addr + lo + s * seg;
+        d.host = reinterpret_cast<uint64_t>(c->image_dev + r.off + lo + s * seg);
+        d.bytes = (uint32_t)std::min<uint64_t>(seg, len - s * seg);
+        d.chunk = (uint32_t)(r.first + j);
+        d.seg = s;
+        d.nseg = nseg;
+        desc.push_back(d);
+      }
+      S->ce_dev.push_back(reinterpret_cast<void*>(r.r.dev_addr + lo));
+      S->ce_host.push_back(c->image + r.off + lo);
+      S->ce_bytes.push_back(len);
+      // CE_PIPE groups: consecutive whole chunks up to ~pipe_mib MiB; spans merge contiguous chunks
+      Span sp{r.r.dev_addr + lo, c->image + r.off + lo, len};
+      if (!cur.spans.empty() && cur.spans.back().dev + cur.spans.back().bytes == sp.dev &&
+          cur.spans.back().host + cur.spans.back().bytes == sp.host)
+        cur.spans.back().bytes += len;
+      else
+        cur.spans.push_back(sp);
+      cur.d1 = (uint32_t)desc.size();
+      cur_bytes += len;
+      if (cur_bytes >= target) {
+        S->groups.push_back(std::move(cur));
+        cur = Group{(uint32_t)desc.size(), (uint32_t)desc.size(), {}};
+        cur_bytes = 0;
+      }
+    }
+  }
+  if (!cur.spans.empty()) S->groups.push_back(std::move(cur));
+  if (desc.size() > 0xFFFFFFFFull) {
+    c->err = "too many segments";
+    return SWAP_EUNSUPPORTED;
+  }
+  S->owned = true;
+  S->n_desc = (uint32_t)desc.size();
+  CUDA_TRY(c, cudaMalloc(&S->d_desc, std::max<size_t>(1, desc.size()) * sizeof(swk::SegDesc)));
+  if (!desc.empty())
+    CUDA_TRY(c, cudaMemcpy(S->d_desc, desc.data(), desc.size() * sizeof(swk::SegDesc), cudaMemcpyHostToDevice));
+  S->group_ev.assign(S->groups.size(), nullptr);
+  for (auto& e : S->group_ev) CUDA_TRY(c, cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  return SWAP_OK;
+}
+
+static DescSet alias_of(const DescSet& S) {
+  DescSet a = S;
+  a.owned = false;
+  return a;
+}
+
+// (Re)builds every set from the current policies.
+swap_status build_sets(swap_ctx* c) {
+  free_set(c->s_move);
+  free_set(c->s_save);
+  free_set(c->s_zero);
+  free_set(c->s_all);
+  if (c->d_zero) {
+    cudaFree(c->d_zero);
+    c->d_zero = nullptr;
+  }
+  const auto& pol = c->policy;
+  bool any_once = false, any_discard = false;
+  uint64_t zero_bytes = 0;
+  for (size_t i = 0; i < pol.size(); ++i) {
+    any_once |= pol[i] == SWAP_POLICY_SAVE_ONCE;
+    if (pol[i] == SWAP_POLICY_DISCARD) {
+      any_discard = true;
+      zero_bytes = std::max<uint64_t>(zero_bytes, std::min<uint64_t>(c->plan.C, c->plan.regions[i].r.bytes));
+    }
+  }
+  swap_status st = build_set(c, &c->s_all, [](size_t) { return true; }, false);
+  if (st != SWAP_OK) return st;
+  if (!any_once && !any_discard) {
+    c->s_move = alias_of(c->s_all);
+    c->s_save = alias_of(c->s_all);
+  } else {
+    st = build_set(c, &c->s_move, [&](size_t i) { return pol[i] != SWAP_POLICY_DISCARD; }, false);
+    if (st != SWAP_OK) return st;
+    if (any_once) {
+      st = build_set(c, &c->s_save, [&](size_t i) { return pol[i] == SWAP_POLICY_SAVE; }, false);
+      if (st != SWAP_OK) return st;
+    } else {
+      c->s_save = alias_of(c->s_move);
+    }
+  }
+  if (any_discard) {
+    CUDA_TRY(c, cudaMalloc(&c->d_zero, std::max<uint64_t>(16, (zero_bytes + 31) & ~31ull)));
+    CUDA_TRY(c, cudaMemset(c->d_zero, 0, std::max<uint64_t>(16, (zero_bytes + 31) & ~31ull)));
+    st = build_set(c, &c->s_zero, [&](size_t i) { return pol[i] == SWAP_POLICY_DISCARD; }, true);
+    if (st != SWAP_OK) return st;
+  }
+  if (c->d_partial) cudaFree(c->d_partial);
+  c->d_partial = nullptr;
+  CUDA_TRY(c, cudaMalloc(&c->d_partial, std::max<size_t>(1, c->s_all.n_desc) * 4));
+  return SWAP_OK;
+}
+
+}  // namespace swc
