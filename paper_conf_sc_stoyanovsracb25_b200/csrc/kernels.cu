@@ -493,7 +493,6 @@ template <bool AL32>
 __device__ __forceinline__ void ld32a(const uint8_t* p, uint32_t (&w)[8]) {
   if (AL32) ld32(p, w); else ld32_v4x2(p, w);
 }
-
 __device__ __forceinline__ uint32_t lds_at(uint32_t addr) {
   uint32_t v;
   asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
@@ -520,31 +519,52 @@ __device__ __forceinline__ uint32_t z96(uint32_t T, uint32_t lz) {
          lds_off<6 * 2048>(((T >> 17) & 0x780u) | lz) ^ lds_off<7 * 2048>(((T >> 21) & 0x780u) | lz);
 }
 
+// One 32-B piece: advance the register across the 96-B gap, then through the piece's 8 words.
+__device__ __forceinline__ uint32_t crc_piece32(uint32_t c, const uint32_t (&w)[8], uint32_t lb, uint32_t lz) {
+  c = z96(c, lz);
+#pragma unroll
+  for (int j = 0; j < 8; ++j) c = crc_word4(c, w[j], lb);
+  return c;
+}
+
 // Register of one lane over its pieces s0, s0+128, ... < send (send = min(strand end, len)).
+// A 4-deep software pipeline: each 256-bit load is consumed one loop iteration after it is issued,
+// so ptxas cannot sink it next to its use and four loads per lane stay in flight.
 template <bool AL32>
 __device__ __forceinline__ uint32_t lane_pieces_crc(const uint8_t* src, uint64_t s0, uint64_t send, uint32_t lb,
                                                     uint32_t lz) {
   uint32_t c = 0;
-  uint64_t s = s0;
-  // full pieces, HT_U at a time
-  for (; s + (HT_U - 1) * 128 + 32 <= send; s += HT_U * 128) {
-    uint32_t w[HT_U][8];
-#pragma unroll
-    for (int u = 0; u < HT_U; ++u) ld32a<AL32>(src + s + 128 * u, w[u]);
-#pragma unroll
-    for (int u = 0; u < HT_U; ++u) {
-      c = z96(c, lz);
-#pragma unroll
-      for (int j = 0; j < 8; ++j) c = crc_word4(c, w[u][j], lb);
+  const uint64_t n = s0 + 32 <= send ? (send - 32 - s0) / 128 + 1 : 0;  // whole 32-B pieces
+  uint64_t t = 0;
+  if (n >= 4) {
+    uint32_t a[8], b[8], d[8], e[8];
+    ld32a<AL32>(src + s0, a);
+    ld32a<AL32>(src + s0 + 128, b);
+    ld32a<AL32>(src + s0 + 256, d);
+    ld32a<AL32>(src + s0 + 384, e);
+    for (; t + 8 <= n; t += 4) {
+      const uint8_t* q = src + s0 + (t + 4) * 128;
+      c = crc_piece32(c, a, lb, lz);
+      ld32a<AL32>(q, a);
+      c = crc_piece32(c, b, lb, lz);
+      ld32a<AL32>(q + 128, b);
+      c = crc_piece32(c, d, lb, lz);
+      ld32a<AL32>(q + 256, d);
+      c = crc_piece32(c, e, lb, lz);
+      ld32a<AL32>(q + 384, e);
     }
+    c = crc_piece32(c, a, lb, lz);
+    c = crc_piece32(c, b, lb, lz);
+    c = crc_piece32(c, d, lb, lz);
+    c = crc_piece32(c, e, lb, lz);
+    t += 4;
   }
-  for (; s + 32 <= send; s += 128) {
+  for (; t < n; ++t) {
     uint32_t w[8];
-    ld32a<AL32>(src + s, w);
-    c = z96(c, lz);
-#pragma unroll
-    for (int j = 0; j < 8; ++j) c = crc_word4(c, w[j], lb);
+    ld32a<AL32>(src + s0 + t * 128, w);
+    c = crc_piece32(c, w, lb, lz);
   }
+  uint64_t s = s0 + n * 128;
   if (s < send) {  // a partial last piece (only at the end of the segment)
     c = z96(c, lz);
     for (; s < send; ++s) c = lds_at((((c ^ src[s]) & 0xFFu) << 7) | lb) ^ (c >> 8);  // table 0 = one byte
