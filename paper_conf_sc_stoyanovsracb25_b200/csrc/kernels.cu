@@ -807,23 +807,45 @@ __device__ __forceinline__ uint64_t w64(const uint32_t (&w)[8], int i) {
   return (uint64_t)w[2 * i] | ((uint64_t)w[2 * i + 1] << 32);
 }
 
+__device__ __forceinline__ void xxh_stripe(uint64_t (&v)[4], const uint32_t (&w)[8]) {
+#pragma unroll
+  for (int i = 0; i < 4; ++i) v[i] = xround(v[i], w64(w, i));
+}
+
+// Stripes [0, end) of one chunk into the four accumulators. A 4-deep software pipeline (each 256-bit
+// load consumed one loop iteration after issue) keeps four stripes per lane in flight; without it ptxas
+// sinks each load next to its use.
 template <bool AL32>
 __device__ __forceinline__ void xxh_stripes(const uint8_t* src, uint64_t end, uint64_t (&v)[4]) {
-  uint64_t o = 0;
-  for (; o + 32 * XK_U <= end; o += 32 * XK_U) {
-    uint32_t w[XK_U][8];
-#pragma unroll
-    for (int u = 0; u < XK_U; ++u) ld32a<AL32>(src + o + 32 * u, w[u]);
-#pragma unroll
-    for (int u = 0; u < XK_U; ++u)
-#pragma unroll
-      for (int i = 0; i < 4; ++i) v[i] = xround(v[i], w64(w[u], i));
+  const uint64_t n = end / 32;
+  uint64_t t = 0;
+  if (n >= 4) {
+    uint32_t a[8], b[8], d[8], e[8];
+    ld32a<AL32>(src, a);
+    ld32a<AL32>(src + 32, b);
+    ld32a<AL32>(src + 64, d);
+    ld32a<AL32>(src + 96, e);
+    for (; t + 8 <= n; t += 4) {
+      const uint8_t* q = src + (t + 4) * 32;
+      xxh_stripe(v, a);
+      ld32a<AL32>(q, a);
+      xxh_stripe(v, b);
+      ld32a<AL32>(q + 32, b);
+      xxh_stripe(v, d);
+      ld32a<AL32>(q + 64, d);
+      xxh_stripe(v, e);
+      ld32a<AL32>(q + 96, e);
+    }
+    xxh_stripe(v, a);
+    xxh_stripe(v, b);
+    xxh_stripe(v, d);
+    xxh_stripe(v, e);
+    t += 4;
   }
-  for (; o < end; o += 32) {
+  for (; t < n; ++t) {
     uint32_t w[8];
-    ld32a<AL32>(src + o, w);
-#pragma unroll
-    for (int i = 0; i < 4; ++i) v[i] = xround(v[i], w64(w, i));
+    ld32a<AL32>(src + t * 32, w);
+    xxh_stripe(v, w);
   }
 }
 
