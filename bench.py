@@ -46,6 +46,20 @@ VERIFY_KERNEL = {"crc32c": "hash_kernel<HASH_CHECK> (CRC-32C: quad-line 256-bit 
                  "xxh64": "xxh_lane_kernel<HASH_CHECK> (XXH64, one lane per chunk; TMA-ring kernel for few large chunks)"}
 PCIE_GEN5_X16_GBPS = 63.015  # 64 GB/s x 128/130 (nominal, per direction)
 MEASURED_PEAKS = os.path.join(ROOT, "MEASURED_PEAKS.json")
+NCU_TRAFFIC = os.path.join(ROOT, "profiles", "ncu_traffic.json")  # dram bytes per verify launch (ncu --set full)
+
+
+def ncu_traffic(workload: str, checksum: str, payload: int):
+    """DRAM bytes (read + write) of the HBM verify launch from the committed ncu capture of the
+    same workload (tools/ncu_verify.sh), or None when no capture matches this workload."""
+    try:
+        rec = json.load(open(NCU_TRAFFIC)).get(f"{workload}/{checksum}")
+    except (OSError, ValueError):
+        return None
+    if not rec or rec.get("payload_bytes") != payload:
+        return None
+    return {"bytes": rec["traffic_bytes"], "per_payload_byte": round(rec["traffic_bytes"] / payload, 5),
+            "source": rec["source"]}
 
 
 def parse():
@@ -432,11 +446,14 @@ def run_ours(args):
             "roofline": {"bound": "host_link", "kernel": RESTORE_KERNEL[eff_mech],
                          "achieved": round(achieved, 3), "peak": PCIE_GEN5_X16_GBPS, "unit": "GB/s",
                          "frac": round(achieved / PCIE_GEN5_X16_GBPS, 4), "traffic": None,
+                         "traffic_note": "copy-engine / link transfer: no kernel DRAM counters (see roofline_verify.traffic)",
                          "peak_source": "PCIe Gen5 x16 nominal per direction after 128b/130b (MEASURED_PEAKS.json has no host-link figure)",
                          "frac_of_measured_ce_h2d": round(achieved / ce["h2d"], 4) if ce else None},
             "roofline_verify": {"bound": "hbm", "kernel": VERIFY_KERNEL[args.checksum],
                                 "achieved": round(payload / (verify_ms * 1e-3) / GB, 1), "peak": hbm_peak,
                                 "unit": "GB/s", "frac": round(payload / (verify_ms * 1e-3) / GB / hbm_peak, 4),
+                                "traffic": (ncu_traffic(name, args.checksum, payload) or {}).get("bytes"),
+                                "traffic_detail": ncu_traffic(name, args.checksum, payload),
                                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)"},
             "measured_ce_GBps": {k: round(v, 2) for k, v in ce.items()},
             "mechanisms": compare,

@@ -15,12 +15,13 @@ from paper_conf_sc_stoyanovsracb25_b200.swap import Swapper  # noqa: E402
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--gib", type=float, default=8)
+ap.add_argument("--config", default="scaled", choices=["scaled", "B", "D"], help="B/D: the full bench workload")
 ap.add_argument("--mechanism", default="auto")
 ap.add_argument("--checksum", default="crc32c")
 ap.add_argument("--reps", type=int, default=2)
 ap.add_argument("--chunk", type=int, default=1 << 20)
 a = ap.parse_args()
-specs = W.scaled(W.config_b(), int(a.gib * (1 << 30)))
+specs = {"B": W.config_b, "D": lambda: W.config_d(0)}.get(a.config, lambda: W.scaled(W.config_b(), int(a.gib * (1 << 30))))()
 offs, total = W.place(specs)
 arena = torch.empty(total, dtype=torch.uint8, device="cuda")
 W.fill_device_arena(arena, specs, offs, seed=1)
