@@ -505,11 +505,17 @@ __device__ __forceinline__ uint32_t lds_off(uint32_t addr) {
   return v;
 }
 
-// slicing-by-4 word step; lb = B + 4*lane (B 32-KiB aligned): table k entry e at lb + k*32K + e*128
-__device__ __forceinline__ uint32_t crc_word4(uint32_t c, uint32_t w, uint32_t lb) {
+// slicing-by-4 word step; lb = B + 4*lane (B 32-KiB aligned): table k entry e at lb + k*32K + e*128.
+// Byte j of x = c ^ w indexes table 3-j at address (byte << 7) | lb. Bytes 0-2 take a shift + LOP3 on
+// the ALU pipe; byte 3's address is (x >> 24) * m128 + lb, an IMAD on the FMA pipe (m128 = 128 held in
+// a register so ptxas cannot fold it back into a shift). The ALU pipe limits this kernel (ncu: 80 %
+// busy); moving one address per word to the FMA pipe measured +6 % (interleaved A/B on config B; the
+// other splits tried — bytes 1-3 or all four via IMAD/IMAD.HI, byte-permute addressing with 64-KiB
+// table pairs — were slower: IMAD.HI and PRMT cost two ALU-equivalent issue slots).
+__device__ __forceinline__ uint32_t crc_word4(uint32_t c, uint32_t w, uint32_t lb, uint32_t m128) {
   c ^= w;
   return lds_off<3 * 32768>(((c << 7) & 0x7F80u) | lb) ^ lds_off<2 * 32768>(((c >> 1) & 0x7F80u) | lb) ^
-         lds_off<1 * 32768>(((c >> 9) & 0x7F80u) | lb) ^ lds_off<0>(((c >> 17) & 0x7F80u) | lb);
+         lds_off<1 * 32768>(((c >> 9) & 0x7F80u) | lb) ^ lds_off<0>((c >> 24) * m128 + lb);
 }
 // Z^96(T) from 8 nibble lookups; lz = B + 128K + 4*lane: nibble table k entry v at lz + k*2K + v*128
 __device__ __forceinline__ uint32_t z96(uint32_t T, uint32_t lz) {
@@ -520,10 +526,11 @@ __device__ __forceinline__ uint32_t z96(uint32_t T, uint32_t lz) {
 }
 
 // One 32-B piece: advance the register across the 96-B gap, then through the piece's 8 words.
-__device__ __forceinline__ uint32_t crc_piece32(uint32_t c, const uint32_t (&w)[8], uint32_t lb, uint32_t lz) {
+__device__ __forceinline__ uint32_t crc_piece32(uint32_t c, const uint32_t (&w)[8], uint32_t lb, uint32_t lz,
+                                                uint32_t m128) {
   c = z96(c, lz);
 #pragma unroll
-  for (int j = 0; j < 8; ++j) c = crc_word4(c, w[j], lb);
+  for (int j = 0; j < 8; ++j) c = crc_word4(c, w[j], lb, m128);
   return c;
 }
 
@@ -532,7 +539,7 @@ __device__ __forceinline__ uint32_t crc_piece32(uint32_t c, const uint32_t (&w)[
 // so ptxas cannot sink it next to its use and four loads per lane stay in flight.
 template <bool AL32>
 __device__ __forceinline__ uint32_t lane_pieces_crc(const uint8_t* src, uint64_t s0, uint64_t send, uint32_t lb,
-                                                    uint32_t lz) {
+                                                    uint32_t lz, uint32_t m128) {
   uint32_t c = 0;
   const uint64_t n = s0 + 32 <= send ? (send - 32 - s0) / 128 + 1 : 0;  // whole 32-B pieces
   uint64_t t = 0;
@@ -544,25 +551,25 @@ __device__ __forceinline__ uint32_t lane_pieces_crc(const uint8_t* src, uint64_t
     ld32a<AL32>(src + s0 + 384, e);
     for (; t + 8 <= n; t += 4) {
       const uint8_t* q = src + s0 + (t + 4) * 128;
-      c = crc_piece32(c, a, lb, lz);
+      c = crc_piece32(c, a, lb, lz, m128);
       ld32a<AL32>(q, a);
-      c = crc_piece32(c, b, lb, lz);
+      c = crc_piece32(c, b, lb, lz, m128);
       ld32a<AL32>(q + 128, b);
-      c = crc_piece32(c, d, lb, lz);
+      c = crc_piece32(c, d, lb, lz, m128);
       ld32a<AL32>(q + 256, d);
-      c = crc_piece32(c, e, lb, lz);
+      c = crc_piece32(c, e, lb, lz, m128);
       ld32a<AL32>(q + 384, e);
     }
-    c = crc_piece32(c, a, lb, lz);
-    c = crc_piece32(c, b, lb, lz);
-    c = crc_piece32(c, d, lb, lz);
-    c = crc_piece32(c, e, lb, lz);
+    c = crc_piece32(c, a, lb, lz, m128);
+    c = crc_piece32(c, b, lb, lz, m128);
+    c = crc_piece32(c, d, lb, lz, m128);
+    c = crc_piece32(c, e, lb, lz, m128);
     t += 4;
   }
   for (; t < n; ++t) {
     uint32_t w[8];
     ld32a<AL32>(src + s0 + t * 128, w);
-    c = crc_piece32(c, w, lb, lz);
+    c = crc_piece32(c, w, lb, lz, m128);
   }
   uint64_t s = s0 + n * 128;
   if (s < send) {  // a partial last piece (only at the end of the segment)
@@ -610,6 +617,7 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
   }
   __syncthreads();
   const uint32_t lb = B + 4u * lane, lz = B + HT_TAB_BYTES + 4u * lane;
+  const uint32_t m128 = blockDim.x >> 3;  // = 128 (HT_THREADS = 1024), opaque to ptxas
   const uint32_t* x2n = p.tables + TAB_X2N;
 
   for (uint32_t r = 0; r < rounds; ++r) {
@@ -626,8 +634,8 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
       const bool al32 = ((d.dev & 31) == 0);
       uint32_t X = 0;
       if (s0 < send) {
-        const uint32_t c = al32 ? lane_pieces_crc<true>(src, s0, send, lb, lz)
-                                : lane_pieces_crc<false>(src, s0, send, lb, lz);
+        const uint32_t c = al32 ? lane_pieces_crc<true>(src, s0, send, lb, lz, m128)
+                                : lane_pieces_crc<false>(src, s0, send, lb, lz, m128);
         const uint32_t k = (len == p.hlane_len) ? __ldg(p.tables + TAB_HLANE + lane)
                                                 : x2nmodp(len - hash_lane_end(len, lane), 3, x2n);
         X = multmodp(k, c);
