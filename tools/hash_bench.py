@@ -6,6 +6,7 @@ import argparse
 import json
 import os
 import statistics
+import time
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
@@ -21,6 +22,7 @@ ap.add_argument("--gib", type=float, default=0, help="0 = full config B")
 ap.add_argument("--checksum", default="crc32c")
 ap.add_argument("--chunk", type=int, default=1 << 20)
 ap.add_argument("--reps", type=int, default=10)
+ap.add_argument("--gap-ms", type=float, default=0, help="idle time before each verify (bench-like boost clocks)")
 ap.add_argument("--crc-variants", default="", help="comma list of SWAP_CRC_KERNEL values, interleaved in-process")
 a = ap.parse_args()
 specs = W.config_b() if not a.gib else W.scaled(W.config_b(), int(a.gib * (1 << 30)))
@@ -40,6 +42,9 @@ with Swapper(regions, mechanism="sm", checksum=1 if a.checksum == "crc32c" else 
         for v in variants:
             if v is not None:
                 os.environ["SWAP_CRC_KERNEL"] = v
+            if a.gap_ms:
+                torch.cuda.synchronize()
+                time.sleep(a.gap_ms * 1e-3)
             assert sw.verify(s)["status"] == 0
             if r >= 2:
                 ms[v].append(sw.timings()["verify_ms"])
