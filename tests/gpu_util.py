@@ -10,11 +10,11 @@ import workloads as W
 CHK = struct.Struct("<IIQQQ")
 
 
-def device_case(specs, seed):
+def device_case(specs, seed, skew=None):
     """Seeded arena on the GPU plus the region tables for the Swapper and for the oracle."""
     import torch
 
-    host, offs = W.host_arena(specs, seed)
+    host, offs = W.host_arena(specs, seed, skew)
     arena = torch.from_numpy(host).cuda()
     base = arena.data_ptr()
     sw_regions = [(base + o, r.nbytes, r.kind, 100 + i) for i, (r, o) in enumerate(zip(specs, offs))]

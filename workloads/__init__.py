@@ -192,12 +192,13 @@ def edge_tables(chunk: int) -> dict[str, list[RegionSpec]]:
 
 
 # ---------------------------------------------------------------- arena placement + contents
-def place(specs: list[RegionSpec]) -> tuple[list[int], int]:
-    """Offsets of each region inside one device arena: BASE_ALIGN-aligned, with GUARD_BYTES
-    of guard before the first region, between regions and after the last."""
+def place(specs: list[RegionSpec], skew: list[int] | None = None) -> tuple[list[int], int]:
+    """Offsets of each region inside one device arena: BASE_ALIGN-aligned (plus skew[i] bytes, a
+    multiple of 16, to exercise less-aligned device addresses), with GUARD_BYTES of guard before
+    the first region, between regions and after the last."""
     offs, pos = [], GUARD_BYTES
-    for r in specs:
-        pos = (pos + BASE_ALIGN - 1) // BASE_ALIGN * BASE_ALIGN
+    for i, r in enumerate(specs):
+        pos = (pos + BASE_ALIGN - 1) // BASE_ALIGN * BASE_ALIGN + (skew[i] if skew else 0)
         offs.append(pos)
         pos += r.nbytes + GUARD_BYTES
     return offs, pos
@@ -209,10 +210,10 @@ def random_bytes(seed: int, nbytes: int) -> np.ndarray:
     return rng.integers(0, 256, size=nbytes, dtype=np.uint8)
 
 
-def host_arena(specs: list[RegionSpec], seed: int) -> tuple[np.ndarray, list[int]]:
+def host_arena(specs: list[RegionSpec], seed: int, skew: list[int] | None = None) -> tuple[np.ndarray, list[int]]:
     """Arena bytes on the host: guard bytes everywhere, region contents seeded per region
     (uniform bytes; bf16 regions get N(0, 0.02) rounded to bf16)."""
-    offs, total = place(specs)
+    offs, total = place(specs, skew)
     arena = np.full(total, GUARD_BYTE, dtype=np.uint8)
     for i, (r, o) in enumerate(zip(specs, offs)):
         arena[o:o + r.nbytes] = region_bytes(r, seed * 1000003 + i)
