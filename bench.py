@@ -410,7 +410,7 @@ def run_ours(args):
         del h
 
     cpu = None
-    if rank == 0 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:  # the oracle beside N=1 only
         import oracle
 
         sample, _ = oracle_sample_specs(specs, args.sample_bytes)
