@@ -193,6 +193,19 @@ def time_oracle_restore(orc, specs, host, offs, threads: int, reps: int):
     return rates, payload
 
 
+def overhead(compare: dict, restore_gbps: float, ce: dict) -> dict | None:
+    """Fused-checksum overhead (BASELINE.json north_star target <= 5 %): the SM movers with vs without
+    the checksum compiled out, and the default restore vs the bare copy-engine H2D rate."""
+    out = {}
+    if "sm" in compare and "sm_nocheck" in compare:
+        for ph in ("restore", "checkpoint"):
+            a, b = compare["sm"][f"{ph}_GBps"], compare["sm_nocheck"][f"{ph}_GBps"]
+            out[f"sm_{ph}"] = round(b / a - 1, 4) if a else None
+    if ce.get("h2d"):
+        out["default_restore_vs_bare_ce_h2d"] = round(ce["h2d"] / restore_gbps - 1, 4)
+    return out or None
+
+
 def cpu_threads() -> int:
     try:
         return len(os.sched_getaffinity(0))
@@ -457,6 +470,7 @@ def run_ours(args):
                                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)"},
             "measured_ce_GBps": {k: round(v, 2) for k, v in ce.items()},
             "mechanisms": compare,
+            "fused_checksum_overhead": overhead(compare, achieved, ce),
             "setup_s": {"fill": round(t_fill, 2), "register_pin": round(t_register, 2)},
             "swap_in_with_hbm_reacquire_s": round(statistics.mean(x[1] for x in reacq), 4),
             "hbm_reacquire_s": round(statistics.mean(x[0] for x in reacq), 4),
