@@ -493,6 +493,26 @@ template <bool AL32>
 __device__ __forceinline__ void ld32a(const uint8_t* p, uint32_t (&w)[8]) {
   if (AL32) ld32(p, w); else ld32_v4x2(p, w);
 }
+// Streaming variants that do not allocate in L1 (every sector is consumed exactly once).
+__device__ __forceinline__ void ld32_na(const uint8_t* p, uint32_t (&w)[8]) {
+  asm("ld.global.nc.L1::no_allocate.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+      : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]), "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7])
+      : "l"(p));
+}
+__device__ __forceinline__ void ld32_v4x2_na(const uint8_t* p, uint32_t (&w)[8]) {
+  asm("ld.global.nc.L1::no_allocate.v4.b32 {%0,%1,%2,%3}, [%4];"
+      : "=r"(w[0]), "=r"(w[1]), "=r"(w[2]), "=r"(w[3]) : "l"(p));
+  asm("ld.global.nc.L1::no_allocate.v4.b32 {%0,%1,%2,%3}, [%4];"
+      : "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7]) : "l"(p + 16));
+}
+template <bool AL32, bool NA>
+__device__ __forceinline__ void ld32p(const uint8_t* p, uint32_t (&w)[8]) {
+  if (NA) {
+    if (AL32) ld32_na(p, w); else ld32_v4x2_na(p, w);
+  } else {
+    ld32a<AL32>(p, w);
+  }
+}
 __device__ __forceinline__ uint32_t lds_at(uint32_t addr) {
   uint32_t v;
   asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
@@ -804,10 +824,10 @@ static cudaError_t launch_xxh_ring(const Params& p, int sm_count, cudaStream_t s
 // ------------------------------------------------------------------ HBM hash kernel (XXH64, lane per chunk)
 // XXH64 consumes a chunk's 32-B stripes strictly in order, so parallelism comes from chunks:
 // one LANE per chunk, its four accumulators in registers, one 256-bit load per stripe (a full
-// sector), XK_U stripes in flight. Used for HASH_STORE / HASH_CHECK when there are enough chunks
-// to occupy the GPU (hash_xxh_lane_ok); otherwise the warp-per-chunk mover handles it.
+// sector), U stripes in flight (4 or 8), loads that do not allocate in L1. Used for HASH_STORE /
+// HASH_CHECK when there are enough chunks to occupy the GPU; launch_xxh_hash picks the launch shape.
 constexpr int XK_THREADS = 256;
-constexpr int XK_U = 4;  // 128 B in flight per lane (U = 8 with 2 CTAs/SM measured slower: 2.7 vs 3.6 TB/s)
+constexpr int XK_U = 4;  // 128 B in flight per lane
 constexpr size_t XK_OFF_BAR = 2 * XK_THREADS * sizeof(SegDesc);
 constexpr size_t XK_SMEM = XK_OFF_BAR + 16;
 
@@ -820,58 +840,52 @@ __device__ __forceinline__ void xxh_stripe(uint64_t (&v)[4], const uint32_t (&w)
   for (int i = 0; i < 4; ++i) v[i] = xround(v[i], w64(w, i));
 }
 
-// Stripes [0, end) of one chunk into the four accumulators. A 4-deep software pipeline (each 256-bit
-// load consumed one loop iteration after issue) keeps four stripes per lane in flight; without it ptxas
-// sinks each load next to its use.
-template <bool AL32>
+// Stripes [0, end) of one chunk into the four accumulators. A U-deep software pipeline (each 256-bit
+// load consumed U stripes after issue) keeps U stripes per lane in flight; without it ptxas sinks each
+// load next to its use.
+template <bool AL32, int U, bool NA>
 __device__ __forceinline__ void xxh_stripes(const uint8_t* src, uint64_t end, uint64_t (&v)[4]) {
   const uint64_t n = end / 32;
   uint64_t t = 0;
-  if (n >= 4) {
-    uint32_t a[8], b[8], d[8], e[8];
-    ld32a<AL32>(src, a);
-    ld32a<AL32>(src + 32, b);
-    ld32a<AL32>(src + 64, d);
-    ld32a<AL32>(src + 96, e);
-    for (; t + 8 <= n; t += 4) {
-      const uint8_t* q = src + (t + 4) * 32;
-      xxh_stripe(v, a);
-      ld32a<AL32>(q, a);
-      xxh_stripe(v, b);
-      ld32a<AL32>(q + 32, b);
-      xxh_stripe(v, d);
-      ld32a<AL32>(q + 64, d);
-      xxh_stripe(v, e);
-      ld32a<AL32>(q + 96, e);
+  if (n >= U) {
+    uint32_t buf[U][8];
+#pragma unroll
+    for (int u = 0; u < U; ++u) ld32p<AL32, NA>(src + u * 32, buf[u]);
+    for (; t + 2 * U <= n; t += U) {
+      const uint8_t* q = src + (t + U) * 32;
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        xxh_stripe(v, buf[u]);
+        ld32p<AL32, NA>(q + u * 32, buf[u]);
+      }
     }
-    xxh_stripe(v, a);
-    xxh_stripe(v, b);
-    xxh_stripe(v, d);
-    xxh_stripe(v, e);
-    t += 4;
+#pragma unroll
+    for (int u = 0; u < U; ++u) xxh_stripe(v, buf[u]);
+    t += U;
   }
   for (; t < n; ++t) {
     uint32_t w[8];
-    ld32a<AL32>(src + t * 32, w);
+    ld32p<AL32, NA>(src + t * 32, w);
     xxh_stripe(v, w);
   }
 }
 
-template <int MODE>
-__global__ void __launch_bounds__(XK_THREADS) xxh_lane_kernel(const Params p) {
+template <int MODE, int U, int MAXT, bool NA>
+__global__ void __launch_bounds__(MAXT) xxh_lane_kernel(const Params p) {
   extern __shared__ __align__(128) uint8_t smem[];
+  const uint32_t T = blockDim.x;
   SegDesc* sDesc = reinterpret_cast<SegDesc*>(smem);
-  uint64_t* sBar = reinterpret_cast<uint64_t*>(smem + XK_OFF_BAR);
+  uint64_t* sBar = reinterpret_cast<uint64_t*>(smem + 2 * T * sizeof(SegDesc));
   const int tid = threadIdx.x;
-  const uint32_t per_round = gridDim.x * XK_THREADS;
-  const uint32_t first0 = blockIdx.x * XK_THREADS;
+  const uint32_t per_round = gridDim.x * T;
+  const uint32_t first0 = blockIdx.x * T;
   const uint32_t rounds = p.n_desc > first0 ? (p.n_desc - first0 + per_round - 1) / per_round : 0u;
   auto issue = [&](uint32_t r) {
     const uint32_t first = r * per_round + first0;
-    const uint32_t cnt = min((uint32_t)XK_THREADS, p.n_desc - first);
+    const uint32_t cnt = min(T, p.n_desc - first);
     uint64_t* bar = sBar + (r & 1);
     mbar_expect_tx(bar, cnt * (uint32_t)sizeof(SegDesc));
-    bulk_g2s(sDesc + (r & 1) * XK_THREADS, p.desc + first, cnt * (uint32_t)sizeof(SegDesc), bar);
+    bulk_g2s(sDesc + (r & 1) * T, p.desc + first, cnt * (uint32_t)sizeof(SegDesc), bar);
   };
   if (tid == 0) {
     mbar_init(sBar, 1);
@@ -886,13 +900,13 @@ __global__ void __launch_bounds__(XK_THREADS) xxh_lane_kernel(const Params p) {
     mbar_wait(sBar + (r & 1), (r >> 1) & 1u);
     const uint32_t idx = r * per_round + first0 + tid;
     if (idx < p.n_desc) {
-      const SegDesc d = sDesc[(r & 1) * XK_THREADS + tid];
+      const SegDesc d = sDesc[(r & 1) * T + tid];
       const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
       const uint64_t len = d.bytes;
       const bool al32 = ((d.dev & 31) == 0);
       uint64_t v[4] = {P1 + P2, P2, 0, 0ull - P1};
       const uint64_t stripes_end = len / 32 * 32;
-      if (al32) xxh_stripes<true>(src, stripes_end, v); else xxh_stripes<false>(src, stripes_end, v);
+      if (al32) xxh_stripes<true, U, NA>(src, stripes_end, v); else xxh_stripes<false, U, NA>(src, stripes_end, v);
       const uint64_t v1 = v[0], v2 = v[1], v3 = v[2], v4 = v[3];
       uint64_t o = stripes_end;
       uint64_t h;
@@ -936,18 +950,43 @@ __global__ void __launch_bounds__(XK_THREADS) xxh_lane_kernel(const Params p) {
   }
 }
 
-template <int MODE>
+template <int MODE, int U, bool NA = false>
 static cudaError_t launch_xxh_lane(const Params& p, int sm_count, cudaStream_t s) {
   const uint32_t blocks = (p.n_desc + XK_THREADS - 1) / XK_THREADS;
   const int grid = (int)std::max<uint32_t>(1, std::min<uint32_t>(blocks, (uint32_t)sm_count * 4));
-  xxh_lane_kernel<MODE><<<grid, XK_THREADS, XK_SMEM, s>>>(p);
+  xxh_lane_kernel<MODE, U, XK_THREADS, NA><<<grid, XK_THREADS, XK_SMEM, s>>>(p);
   return cudaGetLastError();
 }
 
+// Balanced lane launch: exactly one CTA per SM (the dynamic shared-memory request admits only one, so
+// the block scheduler cannot stack CTAs on some SMs and leave others idle — with the 4-CTA/SM launch
+// above, config B's 197 CTAs ran at 11.2 ms or 20.7 ms depending on placement), chunks spread evenly:
+// T = ceil(n / SMs) lanes per SM, rounded to whole warps, capped by the register file.
+constexpr size_t XB_SMEM = 116 * 1024;
+template <int MODE, int U, bool NA = false>
+static cudaError_t launch_xxh_lane_bal(const Params& p, int sm_count, cudaStream_t s) {
+  constexpr int MAXT = U >= 8 ? 640 : 1024;
+  static unsigned long long attr_set = 0;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (!((attr_set >> (dev & 63)) & 1ull)) {
+    e = cudaFuncSetAttribute(xxh_lane_kernel<MODE, U, MAXT, NA>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)XB_SMEM);
+    if (e != cudaSuccess) return e;
+    attr_set |= 1ull << (dev & 63);
+  }
+  // R full rounds of T lanes per SM (a last round a third full would leave two thirds of the lanes idle)
+  const uint32_t per_sm = (p.n_desc + sm_count - 1) / sm_count;
+  const uint32_t R = std::max<uint32_t>(1, (per_sm + MAXT - 1) / MAXT);
+  const uint32_t T = std::min<uint32_t>(MAXT, std::max<uint32_t>(32, ((per_sm + R - 1) / R + 31) / 32 * 32));
+  const int grid = (int)std::min<uint32_t>((uint32_t)sm_count, (p.n_desc + T - 1) / T);
+  xxh_lane_kernel<MODE, U, MAXT, NA><<<grid, T, XB_SMEM, s>>>(p);
+  return cudaGetLastError();
+}
 
-// Many chunks: one lane per chunk keeps all 32 lanes issuing rounds (5+ TB/s measured); few
-// (large) chunks: the TMA ring keeps the memory pipe full with one warp per chunk.
-bool hash_xxh_lane_ok(int sm_count, uint32_t n_desc) { return n_desc >= (uint32_t)sm_count * 192u; }
+// Enough chunks for the lane-per-chunk kernels (below this the TMA ring, one warp per chunk, wins).
+bool hash_xxh_lane_ok(int sm_count, uint32_t n_desc) { return n_desc >= (uint32_t)sm_count * 27u; }
 
 int mover_threads() { return THREADS; }
 size_t mover_smem_bytes(int kind) {
@@ -970,24 +1009,57 @@ static cudaError_t launch_t(const Params& p, int grid, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-// Kernel choice for XXH64 hash passes: 0 = automatic, 1 = lane per chunk, 3 = TMA ring
-// (SWAP_XXH_KERNEL=lane|ring forces one, for measurements and tests).
+// Kernel choice for XXH64 hash passes: 0 = automatic, 1 = lane per chunk (XK_U deep, up to 4 CTAs/SM),
+// 2 = the same 8 deep, 3 = TMA ring, 4/5 = balanced lane launch 4/8 deep (SWAP_XXH_KERNEL=lane|lane8|
+// ring|bal|bal8 forces one, for measurements and tests; read at every launch so one process can
+// interleave variants).
 static int xxh_variant() {
-  static int v = [] {
-    const char* e = getenv("SWAP_XXH_KERNEL");
-    if (!e) return 0;
-    if (!strcmp(e, "lane")) return 1;
-    if (!strcmp(e, "ring")) return 3;
-    return 0;
-  }();
-  return v;
+  const char* e = getenv("SWAP_XXH_KERNEL");
+  if (!e) return 0;
+  if (!strcmp(e, "lane")) return 1;
+  if (!strcmp(e, "lane8")) return 2;
+  if (!strcmp(e, "ring")) return 3;
+  if (!strcmp(e, "bal")) return 4;
+  if (!strcmp(e, "bal8")) return 5;
+  if (!strcmp(e, "lanena")) return 6;
+  if (!strcmp(e, "lane8na")) return 7;
+  if (!strcmp(e, "balna")) return 8;
+  if (!strcmp(e, "bal8na")) return 9;
+  return 0;
 }
 
 cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_t s) {
   if (p.n_desc == 0) return cudaSuccess;
-  if (xxh_variant() == 1 || (xxh_variant() == 0 && hash_xxh_lane_ok(sm_count, p.n_desc)))
-    return mode == HASH_STORE ? launch_xxh_lane<HASH_STORE>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK>(p, sm_count, s);
-  return mode == HASH_STORE ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
+  const bool st = mode == HASH_STORE;
+  switch (xxh_variant()) {
+    case 2: return st ? launch_xxh_lane<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8>(p, sm_count, s);
+    case 4: return st ? launch_xxh_lane_bal<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 4>(p, sm_count, s);
+    case 5: return st ? launch_xxh_lane_bal<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8>(p, sm_count, s);
+    case 6: return st ? launch_xxh_lane<HASH_STORE, 4, true>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 4, true>(p, sm_count, s);
+    case 7: return st ? launch_xxh_lane<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8, true>(p, sm_count, s);
+    case 8: return st ? launch_xxh_lane_bal<HASH_STORE, 4, true>(p, sm_count, s)
+                      : launch_xxh_lane_bal<HASH_CHECK, 4, true>(p, sm_count, s);
+    case 9: return st ? launch_xxh_lane_bal<HASH_STORE, 8, true>(p, sm_count, s)
+                      : launch_xxh_lane_bal<HASH_CHECK, 8, true>(p, sm_count, s);
+    case 3: return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
+    case 1: return st ? launch_xxh_lane<HASH_STORE, XK_U>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, XK_U>(p, sm_count, s);
+    default: break;
+  }
+  // Measured on config B and an 8-GiB cut of it (profiles/r01_xxh_variants.md): up to
+  // 256 KiB chunks the 8-deep lane kernel wins (5.6-6.0 TB/s); from 1 MiB with many chunks the
+  // balanced 4-deep launch (5.2 TB/s; 8 deep falls to 2.7-2.9 TB/s at 1 MiB), with fewer chunks the
+  // balanced 8-deep launch (per-lane rate = bytes in flight / latency), and with only a few thousand
+  // chunks the warp-per-chunk TMA ring.
+  const uint32_t n = p.n_desc, many = (uint32_t)sm_count * 192u;
+  if (p.chunk_bytes <= (256u << 10)) {
+    if (n >= many) return st ? launch_xxh_lane<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8, true>(p, sm_count, s);
+    return st ? launch_xxh_lane_bal<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8, true>(p, sm_count, s);
+  }
+  if (n >= many)
+    return st ? launch_xxh_lane_bal<HASH_STORE, 4, true>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 4, true>(p, sm_count, s);
+  if (hash_xxh_lane_ok(sm_count, n))
+    return st ? launch_xxh_lane_bal<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8, true>(p, sm_count, s);
+  return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
 }
 
 cudaError_t launch_mover(int mode, int kind, const Params& p, int grid, cudaStream_t s) {

@@ -23,7 +23,9 @@ ap.add_argument("--checksum", default="crc32c")
 ap.add_argument("--chunk", type=int, default=1 << 20)
 ap.add_argument("--reps", type=int, default=10)
 ap.add_argument("--gap-ms", type=float, default=0, help="idle time before each verify (bench-like boost clocks)")
-ap.add_argument("--crc-variants", default="", help="comma list of SWAP_CRC_KERNEL values, interleaved in-process")
+ap.add_argument("--variants", default="", help="comma list of kernel variants (SWAP_XXH_KERNEL for xxh64, "
+                "SWAP_CRC_KERNEL for crc32c), interleaved in-process")
+ap.add_argument("--all", action="store_true", help="print every rep's time")
 a = ap.parse_args()
 specs = W.config_b() if not a.gib else W.scaled(W.config_b(), int(a.gib * (1 << 30)))
 offs, total = W.place(specs)
@@ -36,12 +38,13 @@ with Swapper(regions, mechanism="sm", checksum=1 if a.checksum == "crc32c" else 
         torch.cuda.stream(s):
     sw.checkpoint(s)
     sw.restore(s)
-    variants = a.crc_variants.split(",") if a.crc_variants else [None]
+    variants = a.variants.split(",") if a.variants else [None]
+    env_key = "SWAP_XXH_KERNEL" if a.checksum == "xxh64" else "SWAP_CRC_KERNEL"
     ms = {v: [] for v in variants}
     for r in range(a.reps + 2):
         for v in variants:
             if v is not None:
-                os.environ["SWAP_CRC_KERNEL"] = v
+                os.environ[env_key] = v
             if a.gap_ms:
                 torch.cuda.synchronize()
                 time.sleep(a.gap_ms * 1e-3)
@@ -53,4 +56,5 @@ for v in variants:
     print(json.dumps({"checksum": a.checksum, "chunk": a.chunk, "payload": payload,
                       "variant": v if v is not None else os.environ.get("SWAP_XXH_KERNEL", "") + os.environ.get("SWAP_CRC_KERNEL", ""),
                       "verify_ms": round(med, 3), "min_ms": round(min(ms[v]), 3), "max_ms": round(max(ms[v]), 3),
-                      "TBps": round(payload / (med * 1e-3) / 1e12, 3)}), flush=True)
+                      "TBps": round(payload / (med * 1e-3) / 1e12, 3),
+                      "all_ms": [round(x, 2) for x in ms[v]] if a.all else None}), flush=True)
