@@ -11,6 +11,7 @@
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "ctx.h"
@@ -76,6 +77,25 @@ swap_status swap_create(const swap_config_t* cfg_in, swap_ctx_t** out) {
   return SWAP_OK;
 }
 
+// Faults the image's pages in (the kernel zero-fills them) from several threads before pinning:
+// cudaHostRegister would otherwise fault and zero every page from the calling thread alone.
+static void prefault(uint8_t* p, size_t n) {
+  const size_t page = 2u << 20;
+  const unsigned hw = std::thread::hardware_concurrency();
+  const size_t k = std::max<size_t>(1, std::min<size_t>({hw ? hw : 1u, 32u, n / page}));
+  const size_t per = (n / k + page - 1) / page * page;
+  std::vector<std::thread> th;
+  for (size_t t = 0; t < k; ++t) {
+    const size_t lo = t * per, hi = std::min(n, lo + per);
+    if (lo >= hi) break;
+    th.emplace_back([p, lo, hi] {
+      volatile uint8_t* q = p;
+      for (size_t o = lo; o < hi; o += 4096) q[o] = 0;  // a write: a read would map the shared zero page
+    });
+  }
+  for (auto& x : th) x.join();
+}
+
 swap_status swap_register_regions(swap_ctx_t* c, const swap_region_t* regions, size_t n) {
   if (!c) return SWAP_EINVAL;
   swp::Plan plan;
@@ -101,6 +121,7 @@ swap_status swap_register_regions(swap_ctx_t* c, const swap_region_t* regions, s
   }
   c->image = static_cast<uint8_t*>(m);
   madvise(m, c->map_bytes, MADV_HUGEPAGE);
+  prefault(c->image, c->map_bytes);
   cudaError_t e = cudaHostRegister(m, c->map_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
   if (e != cudaSuccess) {
     cudaGetLastError();
