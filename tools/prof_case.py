@@ -15,13 +15,14 @@ from paper_conf_sc_stoyanovsracb25_b200.swap import Swapper  # noqa: E402
 
 ap = argparse.ArgumentParser()
 ap.add_argument("--gib", type=float, default=8)
-ap.add_argument("--config", default="scaled", choices=["scaled", "B", "D"], help="B/D: the full bench workload")
+ap.add_argument("--config", default="scaled", choices=["scaled", "A", "B", "D"],
+                help="A: the 64-MiB parity/bench case (seed 0); B/D: the full bench workloads")
 ap.add_argument("--mechanism", default="auto")
 ap.add_argument("--checksum", default="crc32c")
 ap.add_argument("--reps", type=int, default=2)
 ap.add_argument("--chunk", type=int, default=1 << 20)
 a = ap.parse_args()
-specs = {"B": W.config_b, "D": lambda: W.config_d(0)}.get(a.config, lambda: W.scaled(W.config_b(), int(a.gib * (1 << 30))))()
+specs = {"A": lambda: W.config_a(0), "B": W.config_b, "D": lambda: W.config_d(0)}.get(a.config, lambda: W.scaled(W.config_b(), int(a.gib * (1 << 30))))()
 offs, total = W.place(specs)
 arena = torch.empty(total, dtype=torch.uint8, device="cuda")
 W.fill_device_arena(arena, specs, offs, seed=1)
