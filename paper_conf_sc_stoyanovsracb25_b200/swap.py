@@ -264,9 +264,16 @@ class Swapper:
                 table.append((addr, nb, r[3] if len(r) > 3 else i, kind))
         if isinstance(mechanism, str):
             mechanism = MECHANISMS[mechanism]
+        if device is None:  # raw addresses: the caller's current device (torch's, when torch is in use)
+            try:
+                import torch
+
+                device = torch.cuda.current_device() if torch.cuda.is_available() else 0
+            except ImportError:
+                device = 0
         cfg = swap_config_default()
         cfg.chunk_bytes, cfg.checksum, cfg.mechanism, cfg.align = chunk_bytes, checksum, mechanism, align
-        cfg.device, cfg.rank, cfg.world = device or 0, rank, world
+        cfg.device, cfg.rank, cfg.world = device, rank, world
         cfg.grid_ctas, cfg.seg_bytes, cfg.pipe_mib = grid_ctas, seg_bytes, pipe_mib
         st, h = swap_create(cfg)
         if st:
