@@ -49,12 +49,16 @@ uint32_t host_multmodp(uint32_t a, uint32_t b) {  // a*b mod P, reflected (bit 3
   return p;
 }
 
-uint32_t host_x2nmodp(uint64_t n, unsigned k, const uint32_t* x2n) {  // x^(n*2^k) mod P
+// x^(n*2^k) mod P. For the Castagnoli polynomial x^(2^31) = x (mod P), so x^(2^k) repeats with period
+// 31, not 32 as zlib's CRC-32 table indexing `k & 31` assumes: k is reduced mod 31 (lengths of
+// 512 MiB and more reach k >= 32).
+uint32_t host_x2nmodp(uint64_t n, unsigned k, const uint32_t* x2n) {
   uint32_t p = 1u << 31;
+  k %= 31;
   while (n) {
-    if (n & 1) p = host_multmodp(x2n[k & 31], p);
+    if (n & 1) p = host_multmodp(x2n[k], p);
     n >>= 1;
-    ++k;
+    if (++k == 31) k = 0;
   }
   return p;
 }
@@ -143,12 +147,13 @@ __device__ __forceinline__ uint32_t multmodp(uint32_t a, uint32_t b) {
   }
   return p;
 }
-__device__ uint32_t x2nmodp(uint64_t n, unsigned k, const uint32_t* __restrict__ x2n) {
+__device__ uint32_t x2nmodp(uint64_t n, unsigned k, const uint32_t* __restrict__ x2n) {  // see host_x2nmodp
   uint32_t p = 1u << 31;
+  k %= 31;
   while (n) {
-    if (n & 1) p = multmodp(__ldg(x2n + (k & 31)), p);
+    if (n & 1) p = multmodp(__ldg(x2n + k), p);
     n >>= 1;
-    ++k;
+    if (++k == 31) k = 0;
   }
   return p;
 }
