@@ -80,3 +80,54 @@ def test_random_configuration(seed):
             res = sw.verify(s, hbm_pass=True, raise_on_corrupt=False)
             img[plan.off[i] + byte] ^= 1 << (flip & 7)
             assert (res["n_bad"], res["first_bad_chunk"]) == (1, want), (k, res, want)
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_random_policies_and_sequences(seed):
+    """Random per-region SAVE / SAVE_ONCE / DISCARD policies (reading 24) over a random
+    configuration, through a sequence: checkpoint, the engine mutates memory, checkpoint again, restore
+    twice (restore-many), mutate, checkpoint a third time, restore. Every image and every
+    restored arena equals the oracle applied to oracle.policy_view."""
+    import oracle as orc
+    from paper_conf_sc_stoyanovsracb25_b200 import swap
+
+    specs, skew, k, flip = draw(10_000 + seed)
+    rng = np.random.Generator(np.random.PCG64(flip))
+    arena, host, base, offs, sw_regions, or_regions = device_case(specs, seed, skew)
+    pol = [int(rng.choice([orc.SAVE, orc.SAVE_ONCE, orc.DISCARD], p=[0.5, 0.3, 0.2])) for _ in specs]
+    C, A, kind = k["C"], k["A"], k["kind"]
+
+    def mutate(mem):
+        out = mem.copy()
+        for r, o in zip(specs, offs):
+            if r.nbytes and rng.random() < 0.6:
+                lo = int(rng.integers(0, r.nbytes))
+                out[o + lo:o + min(r.nbytes, lo + 1 + int(rng.integers(0, 5000)))] ^= np.uint8(rng.integers(1, 256))
+        return out
+
+    s = torch.cuda.Stream()
+    with swap.Swapper(sw_regions, chunk_bytes=C, checksum=kind, mechanism=k["mech"], align=A, seg_bytes=k["seg"],
+                      grid_ctas=k["grid"], pipe_mib=k["pipe"]) as sw, torch.cuda.stream(s):
+        for i, p in enumerate(pol):
+            sw.set_region_policy(i, p)
+        first = host.copy()
+        now = host
+        for step in range(3):
+            if step:
+                now = mutate(now)
+                arena.copy_(torch.from_numpy(now).cuda())
+                torch.cuda.synchronize()
+            sw.checkpoint(s)
+            view = orc.policy_view(or_regions, pol, now, first, base)
+            rc, ref, _ = orc.checkpoint(or_regions, view, base, kind, C, A, threads=8)
+            assert rc == 0
+            diff = np.flatnonzero(sw.image() != ref)
+            assert diff.size == 0, f"step {step} {k} pol={pol}: image differs at {diff[:8]}"
+            for _ in range(2 if step == 1 else 1):
+                poison(arena, specs, offs)
+                sw.restore(s)
+                res = sw.verify(s, hbm_pass=True)
+                assert res["status"] == 0 and res["n_bad"] == 0 and res["hbm_n_bad"] == 0, (step, k, res)
+                torch.cuda.synchronize()
+                back = arena.cpu().numpy()
+                assert np.array_equal(back, view), f"step {step} {k}: restored arena differs at {np.flatnonzero(back != view)[:8]}"
