@@ -101,8 +101,8 @@ typedef struct {
   uint32_t grid_ctas;   /* SM mover grid; 0 -> auto (2 CTAs per SM) */
   uint32_t seg_bytes;   /* CRC32C work split inside a chunk: power of 2, >= 4096; 0 -> auto (at registration:
                            one segment per warp slot of the GPU, 4 KiB .. 256 KiB) */
-  uint32_t pipe_mib;    /* SWAP_MECH_CE_PIPE group size in MiB (rounded to whole chunks); 0 -> auto: payload/32
-                           clamped to [2, 256] MiB */
+  uint32_t pipe_mib;    /* SWAP_MECH_CE_PIPE group size in MiB (rounded up to whole chunks); 0 -> auto: payload/32
+                           clamped to [16, 256] MiB */
 } swap_config_t;
 
 typedef struct {
