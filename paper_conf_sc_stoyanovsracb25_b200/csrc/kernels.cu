@@ -875,6 +875,52 @@ __device__ __forceinline__ void xxh_stripes(const uint8_t* src, uint64_t end, ui
   }
 }
 
+// One whole chunk (descriptor d) by one lane: stripes, merge, tail, avalanche (xxHash spec), then
+// store / compare its c_g.
+template <int MODE, int U, bool NA>
+__device__ __forceinline__ void xxh_chunk(const Params& p, const SegDesc& d) {
+  const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
+  const uint64_t len = d.bytes;
+  const bool al32 = ((d.dev & 31) == 0);
+  uint64_t v[4] = {P1 + P2, P2, 0, 0ull - P1};
+  const uint64_t stripes_end = len / 32 * 32;
+  if (al32) xxh_stripes<true, U, NA>(src, stripes_end, v); else xxh_stripes<false, U, NA>(src, stripes_end, v);
+  const uint64_t v1 = v[0], v2 = v[1], v3 = v[2], v4 = v[3];
+  uint64_t o = stripes_end;
+  uint64_t h;
+  if (len >= 32) {
+    h = rotl64(v1, 1) + rotl64(v2, 7) + rotl64(v3, 12) + rotl64(v4, 18);
+    h = xmerge(h, v1);
+    h = xmerge(h, v2);
+    h = xmerge(h, v3);
+    h = xmerge(h, v4);
+  } else {
+    h = P5;
+  }
+  h += len;
+  for (; o + 8 <= len; o += 8) {
+    h ^= xround(0, ld_u64_smem(src + o));  // bytewise little-endian read (tail is unaligned)
+    h = rotl64(h, 27) * P1 + P4;
+  }
+  if (o + 4 <= len) {
+    const uint32_t w = (uint32_t)src[o] | ((uint32_t)src[o + 1] << 8) | ((uint32_t)src[o + 2] << 16) |
+                       ((uint32_t)src[o + 3] << 24);
+    h ^= (uint64_t)w * P1;
+    h = rotl64(h, 23) * P2 + P3;
+    o += 4;
+  }
+  for (; o < len; ++o) {
+    h ^= (uint64_t)src[o] * P5;
+    h = rotl64(h, 11) * P1;
+  }
+  h ^= h >> 33;
+  h *= P2;
+  h ^= h >> 29;
+  h *= P3;
+  h ^= h >> 32;
+  chunk_result<MODE>(p, d.chunk, h);
+}
+
 template <int MODE, int U, int MAXT, bool NA>
 __global__ void __launch_bounds__(MAXT) xxh_lane_kernel(const Params p) {
   extern __shared__ __align__(128) uint8_t smem[];
@@ -906,52 +952,30 @@ __global__ void __launch_bounds__(MAXT) xxh_lane_kernel(const Params p) {
     const uint32_t idx = r * per_round + first0 + tid;
     if (idx < p.n_desc) {
       const SegDesc d = sDesc[(r & 1) * T + tid];
-      const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
-      const uint64_t len = d.bytes;
-      const bool al32 = ((d.dev & 31) == 0);
-      uint64_t v[4] = {P1 + P2, P2, 0, 0ull - P1};
-      const uint64_t stripes_end = len / 32 * 32;
-      if (al32) xxh_stripes<true, U, NA>(src, stripes_end, v); else xxh_stripes<false, U, NA>(src, stripes_end, v);
-      const uint64_t v1 = v[0], v2 = v[1], v3 = v[2], v4 = v[3];
-      uint64_t o = stripes_end;
-      uint64_t h;
-      if (len >= 32) {
-        h = rotl64(v1, 1) + rotl64(v2, 7) + rotl64(v3, 12) + rotl64(v4, 18);
-        h = xmerge(h, v1);
-        h = xmerge(h, v2);
-        h = xmerge(h, v3);
-        h = xmerge(h, v4);
-      } else {
-        h = P5;
-      }
-      h += len;
-      for (; o + 8 <= len; o += 8) {
-        h ^= xround(0, ld_u64_smem(src + o));  // bytewise little-endian read (tail is unaligned)
-        h = rotl64(h, 27) * P1 + P4;
-      }
-      if (o + 4 <= len) {
-        const uint32_t w = (uint32_t)src[o] | ((uint32_t)src[o + 1] << 8) | ((uint32_t)src[o + 2] << 16) |
-                           ((uint32_t)src[o + 3] << 24);
-        h ^= (uint64_t)w * P1;
-        h = rotl64(h, 23) * P2 + P3;
-        o += 4;
-      }
-      for (; o < len; ++o) {
-        h ^= (uint64_t)src[o] * P5;
-        h = rotl64(h, 11) * P1;
-      }
-      h ^= h >> 33;
-      h *= P2;
-      h ^= h >> 29;
-      h *= P3;
-      h ^= h >> 32;
-      chunk_result<MODE>(p, d.chunk, h);
+      xxh_chunk<MODE, U, NA>(p, d);
     }
     __syncthreads();
     if (tid == 0 && r + 2 < rounds) {
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       issue(r + 2);
     }
+  }
+}
+
+// Dynamic lane kernel: every lane starts on chunk (its global index) and then takes the next unclaimed
+// chunk from a ticket counter (claimed at the start of the current chunk, so the atomic's latency hides
+// behind it). The static launches hand every lane its chunks up front, and under load some SMs are
+// served more slowly than others: ncu on config B showed SMs idle for 8 % (4 deep) / 26 % (8 deep) of
+// the kernel waiting for the slowest one. Here fast lanes simply hash more chunks.
+template <int MODE, int U, int MAXT, bool NA>
+__global__ void __launch_bounds__(MAXT) xxh_dyn_kernel(const Params p) {
+  const uint32_t lanes = gridDim.x * blockDim.x;
+  uint32_t idx = blockIdx.x * blockDim.x + threadIdx.x;
+  while (idx < p.n_desc) {
+    const SegDesc d = p.desc[idx];
+    const uint32_t next = lanes + atomicAdd(p.ticket, 1u);
+    xxh_chunk<MODE, U, NA>(p, d);
+    idx = next;
   }
 }
 
@@ -989,6 +1013,23 @@ static cudaError_t launch_xxh_lane_bal(const Params& p, int sm_count, cudaStream
   const uint32_t T = std::min<uint32_t>(MAXT, std::max<uint32_t>(32, ((per_sm + R - 1) / R + 31) / 32 * 32));
   const int grid = (int)std::min<uint32_t>((uint32_t)sm_count, (p.n_desc + T - 1) / T);
   xxh_lane_kernel<MODE, U, MAXT, NA><<<grid, T, XB_SMEM, s>>>(p);
+  return cudaGetLastError();
+}
+
+// Dynamic lane launch: one CTA of T lanes per SM (SWAP_XXH_DYN_T overrides T, for measurements), the
+// ticket zeroed on the launching stream first.
+template <int MODE, int U, bool NA = true>
+static cudaError_t launch_xxh_dyn(const Params& p, int sm_count, cudaStream_t s) {
+  constexpr int MAXT = U >= 8 ? 640 : 1024;
+  if (!p.ticket) return launch_xxh_lane_bal<MODE, U, NA>(p, sm_count, s);
+  uint32_t T = U >= 8 ? 192 : 352;
+  if (const char* e = getenv("SWAP_XXH_DYN_T")) T = std::max(32, std::min(MAXT, atoi(e)));
+  const uint32_t per_sm = (p.n_desc + sm_count - 1) / sm_count;
+  T = std::min<uint32_t>(T, std::max<uint32_t>(32, (per_sm + 31) / 32 * 32));
+  const int grid = (int)std::min<uint32_t>((uint32_t)sm_count, (p.n_desc + T - 1) / T);
+  cudaError_t e = cudaMemsetAsync(p.ticket, 0, sizeof(unsigned int), s);
+  if (e != cudaSuccess) return e;
+  xxh_dyn_kernel<MODE, U, MAXT, NA><<<grid, T, 0, s>>>(p);
   return cudaGetLastError();
 }
 
@@ -1032,6 +1073,8 @@ static int xxh_variant() {
   if (!strcmp(e, "lane8na")) return 7;
   if (!strcmp(e, "balna")) return 8;
   if (!strcmp(e, "bal8na")) return 9;
+  if (!strcmp(e, "dyn")) return 10;
+  if (!strcmp(e, "dyn8")) return 11;
   return 0;
 }
 
@@ -1048,13 +1091,16 @@ cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_
                       : launch_xxh_lane_bal<HASH_CHECK, 4, true>(p, sm_count, s);
     case 9: return st ? launch_xxh_lane_bal<HASH_STORE, 8, true>(p, sm_count, s)
                       : launch_xxh_lane_bal<HASH_CHECK, 8, true>(p, sm_count, s);
+    case 10: return st ? launch_xxh_dyn<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 4>(p, sm_count, s);
+    case 11: return st ? launch_xxh_dyn<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 8>(p, sm_count, s);
     case 3: return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
     case 1: return st ? launch_xxh_lane<HASH_STORE, XK_U>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, XK_U>(p, sm_count, s);
     default: break;
   }
   // Measured on config B and an 8-GiB cut of it (profiles/r01_xxh_variants.md): up to
   // 256 KiB chunks the 8-deep lane kernel wins (5.6-6.0 TB/s); from 1 MiB with many chunks the
-  // balanced 4-deep launch (5.2 TB/s; 8 deep falls to 2.7-2.9 TB/s at 1 MiB), with fewer chunks the
+  // dynamic 4-deep launch (5.2 TB/s, 2 % above the balanced one; 8 deep falls to 2.7-2.9 TB/s at 1 MiB
+  // once more than ~7 MB are in flight), with fewer chunks the
   // balanced 8-deep launch (per-lane rate = bytes in flight / latency), and with only a few thousand
   // chunks the warp-per-chunk TMA ring.
   const uint32_t n = p.n_desc, many = (uint32_t)sm_count * 192u;
@@ -1062,8 +1108,7 @@ cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_
     if (n >= many) return st ? launch_xxh_lane<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8, true>(p, sm_count, s);
     return st ? launch_xxh_lane_bal<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8, true>(p, sm_count, s);
   }
-  if (n >= many)
-    return st ? launch_xxh_lane_bal<HASH_STORE, 4, true>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 4, true>(p, sm_count, s);
+  if (n >= many) return st ? launch_xxh_dyn<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 4>(p, sm_count, s);
   if (hash_xxh_lane_ok(sm_count, n))
     return st ? launch_xxh_lane_bal<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8, true>(p, sm_count, s);
   return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);

@@ -29,6 +29,7 @@ static_assert(sizeof(SegDesc) == 32, "descriptor is 32 B");
 struct DevStatus {
   unsigned long long n_bad, first_bad;          // fused check of the last restore
   unsigned long long hbm_n_bad, hbm_first_bad;  // HBM verify pass
+  unsigned int ticket, pad;                     // work counter of the dynamic XXH64 lane kernel
 };
 
 enum Mode : int { GATHER = 0, SCATTER = 1, HASH_STORE = 2, HASH_CHECK = 3 };
@@ -61,6 +62,7 @@ struct Params {
   uint32_t zinit_c;              // Z^C(0xFFFFFFFF): the init term of a full chunk
   uint32_t xseg;                 // x^(8*seg_bytes) mod P
   uint32_t hlane_len;            // L1: the segment length TAB_HLANE was built for
+  unsigned int* ticket;          // dynamic XXH64 lane kernel: chunk counter, zeroed before each launch
 };
 
 void build_tables(uint32_t* tab /* TAB_WORDS */, uint64_t common_seg_len, uint64_t seg_bytes);

@@ -34,6 +34,7 @@ swk::Params base_params(swap_ctx* c, const DescSet& S) {
   p.zinit_c = c->zinit_c;
   p.xseg = c->xseg;
   p.hlane_len = (uint32_t)std::min<uint64_t>(c->plan.C, c->seg);
+  p.ticket = &c->d_status->ticket;
   return p;
 }
 
