@@ -43,7 +43,8 @@ RESTORE_KERNEL = {
     "ce_batch": "restore phase: cudaMemcpyBatchAsync + HBM hash pass",
 }
 VERIFY_KERNEL = {"crc32c": "hash_kernel<HASH_CHECK> (CRC-32C: quad-line 256-bit loads, per-lane replicated slice-by-4 + Z^96 tables)",
-                 "xxh64": "xxh_lane_kernel<HASH_CHECK> (XXH64, one lane per chunk; TMA-ring kernel for few large chunks)"}
+                 "xxh64": "xxh_dyn_kernel<HASH_CHECK> (XXH64, one lane per chunk, chunks claimed from a ticket; "
+                           "lane / TMA-ring kernels for other chunk sizes and counts)"}
 PCIE_GEN5_X16_GBPS = 63.015  # 64 GB/s x 128/130 (nominal, per direction)
 MEASURED_PEAKS = os.path.join(ROOT, "MEASURED_PEAKS.json")
 NCU_TRAFFIC = os.path.join(ROOT, "profiles", "ncu_traffic.json")  # dram bytes per verify launch (ncu --set full)
