@@ -875,25 +875,20 @@ __device__ __forceinline__ void xxh_stripes(const uint8_t* src, uint64_t end, ui
   }
 }
 
-// One whole chunk (descriptor d) by one lane: stripes, merge, tail, avalanche (xxHash spec), then
-// store / compare its c_g.
-template <int MODE, int U, bool NA>
-__device__ __forceinline__ void xxh_chunk(const Params& p, const SegDesc& d) {
+// The end of one chunk's XXH64 once its whole 32-B stripes are in v (xxHash spec): merge, the tail
+// [stripes_end, len) read from device memory at src, avalanche; then store / compare its c_g.
+template <int MODE>
+__device__ __forceinline__ void xxh_finish(const Params& p, const SegDesc& d, const uint64_t (&v)[4]) {
   const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
   const uint64_t len = d.bytes;
-  const bool al32 = ((d.dev & 31) == 0);
-  uint64_t v[4] = {P1 + P2, P2, 0, 0ull - P1};
-  const uint64_t stripes_end = len / 32 * 32;
-  if (al32) xxh_stripes<true, U, NA>(src, stripes_end, v); else xxh_stripes<false, U, NA>(src, stripes_end, v);
-  const uint64_t v1 = v[0], v2 = v[1], v3 = v[2], v4 = v[3];
-  uint64_t o = stripes_end;
+  uint64_t o = len / 32 * 32;
   uint64_t h;
   if (len >= 32) {
-    h = rotl64(v1, 1) + rotl64(v2, 7) + rotl64(v3, 12) + rotl64(v4, 18);
-    h = xmerge(h, v1);
-    h = xmerge(h, v2);
-    h = xmerge(h, v3);
-    h = xmerge(h, v4);
+    h = rotl64(v[0], 1) + rotl64(v[1], 7) + rotl64(v[2], 12) + rotl64(v[3], 18);
+    h = xmerge(h, v[0]);
+    h = xmerge(h, v[1]);
+    h = xmerge(h, v[2]);
+    h = xmerge(h, v[3]);
   } else {
     h = P5;
   }
@@ -919,6 +914,16 @@ __device__ __forceinline__ void xxh_chunk(const Params& p, const SegDesc& d) {
   h *= P3;
   h ^= h >> 32;
   chunk_result<MODE>(p, d.chunk, h);
+}
+
+// One whole chunk (descriptor d) by one lane.
+template <int MODE, int U, bool NA>
+__device__ __forceinline__ void xxh_chunk(const Params& p, const SegDesc& d) {
+  const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
+  uint64_t v[4] = {P1 + P2, P2, 0, 0ull - P1};
+  const uint64_t stripes_end = (uint64_t)d.bytes / 32 * 32;
+  if ((d.dev & 31) == 0) xxh_stripes<true, U, NA>(src, stripes_end, v); else xxh_stripes<false, U, NA>(src, stripes_end, v);
+  xxh_finish<MODE>(p, d, v);
 }
 
 template <int MODE, int U, int MAXT, bool NA>
@@ -979,6 +984,85 @@ __global__ void __launch_bounds__(MAXT) xxh_dyn_kernel(const Params p) {
   }
 }
 
+// Warp-cooperative XXH64 (one lane still owns one chunk and its four accumulators, but the warp moves
+// the data): a warp takes a batch of 32 consecutive chunks from the ticket counter and walks them in
+// 512-B blocks; for each of the 32 chunks the warp copies the block into a shared-memory row with one
+// coalesced 16-B-per-lane cp.async (512 contiguous bytes, one page per instruction, where the lane
+// kernels touch 32 pages per load), S stages in flight; then every lane hashes its own row's stripes
+// with LDS.128 (rows padded to 528 B: conflict-free). No registers hold in-flight data, so the depth
+// per chunk is S x 512 B instead of U x 32 B.
+constexpr int XC_ROW = 512 + 16;
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, uint32_t n) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(n) : "memory");
+}
+template <int MODE, int W, int S>
+__global__ void __launch_bounds__(W * 32) xxh_coop_kernel(const Params p) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  uint8_t* rows = smem + (size_t)warp * S * 32 * XC_ROW;
+  const uint32_t rows_s = smem_u32(rows);
+  const uint32_t n_batches = (p.n_desc + 31) / 32;
+  const uint32_t warps = gridDim.x * W;
+  uint32_t batch = blockIdx.x * W + warp;
+  while (batch < n_batches) {
+    uint32_t next = 0;
+    if (lane == 0) next = warps + atomicAdd(p.ticket, 1u);
+    next = __shfl_sync(0xffffffffu, next, 0);
+    const uint32_t idx = batch * 32 + lane;
+    SegDesc d{};
+    if (idx < p.n_desc) d = p.desc[idx];
+    const uint64_t len = idx < p.n_desc ? d.bytes : 0;
+    uint64_t maxlen = len;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) maxlen = max(maxlen, __shfl_xor_sync(0xffffffffu, maxlen, o));
+    const uint32_t nblk = (uint32_t)((maxlen + 511) / 512);
+    auto issue = [&](uint32_t b) {  // block b of every chunk of the batch into stage b % S
+      const uint32_t st = rows_s + (b % S) * 32 * XC_ROW;
+#pragma unroll 4
+      for (int c = 0; c < 32; ++c) {
+        const uint64_t cl = __shfl_sync(0xffffffffu, len, c);
+        const uint64_t cb = __shfl_sync(0xffffffffu, d.dev, c);
+        const uint64_t off = (uint64_t)b * 512 + lane * 16;
+        if (off < cl) {
+          const uint32_t nb = (uint32_t)(cl - off < 16 ? cl - off : 16);
+          cp_async16(st + c * XC_ROW + lane * 16, reinterpret_cast<const void*>(cb + off), nb);
+        }
+      }
+      asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+#pragma unroll
+    for (int b = 0; b < S - 1; ++b) {
+      if ((uint32_t)b < nblk) issue(b);
+      else asm volatile("cp.async.commit_group;" ::: "memory");
+    }
+    uint64_t v[4] = {P1 + P2, P2, 0, 0ull - P1};
+    const uint64_t stripes = len / 32;
+    for (uint32_t b = 0; b < nblk; ++b) {
+      __syncwarp();  // every lane is done reading the stage block b + S - 1 overwrites
+      if (b + S - 1 < nblk) issue(b + S - 1);
+      else asm volatile("cp.async.commit_group;" ::: "memory");
+      asm volatile("cp.async.wait_group %0;" ::"n"(S - 1) : "memory");
+      __syncwarp();
+      const uint64_t s0 = (uint64_t)b * 16;
+      if (s0 < stripes) {
+        const uint32_t ns = (uint32_t)(stripes - s0 < 16 ? stripes - s0 : 16);
+        const uint4* row = reinterpret_cast<const uint4*>(rows + ((b % S) * 32 + lane) * XC_ROW);
+        for (uint32_t t = 0; t < ns; ++t) {
+          const uint4 a = row[2 * t], c = row[2 * t + 1];
+          v[0] = xround(v[0], ((uint64_t)a.y << 32) | a.x);
+          v[1] = xround(v[1], ((uint64_t)a.w << 32) | a.z);
+          v[2] = xround(v[2], ((uint64_t)c.y << 32) | c.x);
+          v[3] = xround(v[3], ((uint64_t)c.w << 32) | c.z);
+        }
+      }
+    }
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    __syncwarp();
+    if (idx < p.n_desc) xxh_finish<MODE>(p, d, v);
+    batch = next;
+  }
+}
+
 template <int MODE, int U, bool NA = false>
 static cudaError_t launch_xxh_lane(const Params& p, int sm_count, cudaStream_t s) {
   const uint32_t blocks = (p.n_desc + XK_THREADS - 1) / XK_THREADS;
@@ -1033,6 +1117,27 @@ static cudaError_t launch_xxh_dyn(const Params& p, int sm_count, cudaStream_t s)
   return cudaGetLastError();
 }
 
+template <int MODE, int W, int S>
+static cudaError_t launch_xxh_coop(const Params& p, int sm_count, cudaStream_t s) {
+  constexpr size_t smem = (size_t)W * S * 32 * XC_ROW;
+  if (!p.ticket) return cudaErrorInvalidValue;
+  static unsigned long long attr_set = 0;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (!((attr_set >> (dev & 63)) & 1ull)) {
+    e = cudaFuncSetAttribute(xxh_coop_kernel<MODE, W, S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr_set |= 1ull << (dev & 63);
+  }
+  const uint32_t n_batches = (p.n_desc + 31) / 32;
+  const int grid = (int)std::max<uint32_t>(1, std::min<uint32_t>((uint32_t)sm_count, (n_batches + W - 1) / W));
+  e = cudaMemsetAsync(p.ticket, 0, sizeof(unsigned int), s);
+  if (e != cudaSuccess) return e;
+  xxh_coop_kernel<MODE, W, S><<<grid, W * 32, smem, s>>>(p);
+  return cudaGetLastError();
+}
+
 // Enough chunks for the lane-per-chunk kernels (below this the TMA ring, one warp per chunk, wins).
 bool hash_xxh_lane_ok(int sm_count, uint32_t n_desc) { return n_desc >= (uint32_t)sm_count * 27u; }
 
@@ -1075,6 +1180,9 @@ static int xxh_variant() {
   if (!strcmp(e, "bal8na")) return 9;
   if (!strcmp(e, "dyn")) return 10;
   if (!strcmp(e, "dyn8")) return 11;
+  if (!strcmp(e, "coop")) return 12;   // 6 warps x 2 stages
+  if (!strcmp(e, "coop3")) return 13;  // 4 warps x 3 stages
+  if (!strcmp(e, "coop4")) return 14;  // 3 warps x 4 stages
   return 0;
 }
 
@@ -1093,6 +1201,9 @@ cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_
                       : launch_xxh_lane_bal<HASH_CHECK, 8, true>(p, sm_count, s);
     case 10: return st ? launch_xxh_dyn<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 4>(p, sm_count, s);
     case 11: return st ? launch_xxh_dyn<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 8>(p, sm_count, s);
+    case 12: return st ? launch_xxh_coop<HASH_STORE, 6, 2>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2>(p, sm_count, s);
+    case 13: return st ? launch_xxh_coop<HASH_STORE, 4, 3>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 4, 3>(p, sm_count, s);
+    case 14: return st ? launch_xxh_coop<HASH_STORE, 3, 4>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 3, 4>(p, sm_count, s);
     case 3: return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
     case 1: return st ? launch_xxh_lane<HASH_STORE, XK_U>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, XK_U>(p, sm_count, s);
     default: break;
@@ -1102,11 +1213,20 @@ cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_
   // dynamic 4-deep launch (5.2 TB/s, 2 % above the balanced one; 8 deep falls to 2.7-2.9 TB/s at 1 MiB
   // once more than ~7 MB are in flight), with fewer chunks the
   // balanced 8-deep launch (per-lane rate = bytes in flight / latency), and with only a few thousand
-  // chunks the warp-per-chunk TMA ring.
+  // chunks the warp-per-chunk TMA ring. From 2 MiB chunks the warp-cooperative kernel while there are
+  // enough 32-chunk batches for its warps (2 MiB: 3.9 vs 2.0 TB/s; 4 MiB: 2.5 vs 1.5), else the ring.
   const uint32_t n = p.n_desc, many = (uint32_t)sm_count * 192u;
   if (p.chunk_bytes <= (256u << 10)) {
     if (n >= many) return st ? launch_xxh_lane<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8, true>(p, sm_count, s);
     return st ? launch_xxh_lane_bal<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8, true>(p, sm_count, s);
+  }
+  if (p.chunk_bytes >= (2u << 20) && p.ticket) {  // big chunks: the warp-cooperative kernel while batches last
+    const uint32_t batches = (n + 31) / 32;
+    if (batches >= (uint32_t)sm_count * 5)
+      return st ? launch_xxh_coop<HASH_STORE, 6, 2>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2>(p, sm_count, s);
+    if (batches >= (uint32_t)sm_count * 2)
+      return st ? launch_xxh_coop<HASH_STORE, 4, 3>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 4, 3>(p, sm_count, s);
+    return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
   }
   if (n >= many) return st ? launch_xxh_dyn<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 4>(p, sm_count, s);
   if (hash_xxh_lane_ok(sm_count, n))
