@@ -1047,12 +1047,31 @@ __global__ void __launch_bounds__(W * 32) xxh_coop_kernel(const Params p) {
       if (s0 < stripes) {
         const uint32_t ns = (uint32_t)(stripes - s0 < 16 ? stripes - s0 : 16);
         const uint4* row = reinterpret_cast<const uint4*>(rows + ((b % S) * 32 + lane) * XC_ROW);
-        for (uint32_t t = 0; t < ns; ++t) {
-          const uint4 a = row[2 * t], c = row[2 * t + 1];
-          v[0] = xround(v[0], ((uint64_t)a.y << 32) | a.x);
-          v[1] = xround(v[1], ((uint64_t)a.w << 32) | a.z);
-          v[2] = xround(v[2], ((uint64_t)c.y << 32) | c.x);
-          v[3] = xround(v[3], ((uint64_t)c.w << 32) | c.z);
+        if (ns == 16) {  // a whole block: shared-memory loads four stripes ahead of the rounds
+#pragma unroll
+          for (int t0 = 0; t0 < 16; t0 += 4) {
+            uint4 a[4], c[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+              a[u] = row[2 * (t0 + u)];
+              c[u] = row[2 * (t0 + u) + 1];
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+              v[0] = xround(v[0], ((uint64_t)a[u].y << 32) | a[u].x);
+              v[1] = xround(v[1], ((uint64_t)a[u].w << 32) | a[u].z);
+              v[2] = xround(v[2], ((uint64_t)c[u].y << 32) | c[u].x);
+              v[3] = xround(v[3], ((uint64_t)c[u].w << 32) | c[u].z);
+            }
+          }
+        } else {
+          for (uint32_t t = 0; t < ns; ++t) {
+            const uint4 a = row[2 * t], c = row[2 * t + 1];
+            v[0] = xround(v[0], ((uint64_t)a.y << 32) | a.x);
+            v[1] = xround(v[1], ((uint64_t)a.w << 32) | a.z);
+            v[2] = xround(v[2], ((uint64_t)c.y << 32) | c.x);
+            v[3] = xround(v[3], ((uint64_t)c.w << 32) | c.z);
+          }
         }
       }
     }
