@@ -991,41 +991,45 @@ __global__ void __launch_bounds__(MAXT) xxh_dyn_kernel(const Params p) {
 // kernels touch 32 pages per load), S stages in flight; then every lane hashes its own row's stripes
 // with LDS.128 (rows padded to 528 B: conflict-free). No registers hold in-flight data, so the depth
 // per chunk is S x 512 B instead of U x 32 B.
-constexpr int XC_ROW = 512 + 16;
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, uint32_t n) {
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src), "r"(n) : "memory");
 }
-template <int MODE, int W, int S>
+template <int MODE, int W, int S, int K>
 __global__ void __launch_bounds__(W * 32) xxh_coop_kernel(const Params p) {
+  constexpr int BLK = 16384 / K, ROW = BLK + 16, SPB = BLK / 32;  // block bytes per chunk, row, stripes
   extern __shared__ __align__(128) uint8_t smem[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  uint8_t* rows = smem + (size_t)warp * S * 32 * XC_ROW;
+  uint8_t* rows = smem + (size_t)warp * S * K * ROW;
   const uint32_t rows_s = smem_u32(rows);
-  const uint32_t n_batches = (p.n_desc + 31) / 32;
+  const uint32_t n_batches = (p.n_desc + K - 1) / K;
   const uint32_t warps = gridDim.x * W;
   uint32_t batch = blockIdx.x * W + warp;
   while (batch < n_batches) {
     uint32_t next = 0;
     if (lane == 0) next = warps + atomicAdd(p.ticket, 1u);
     next = __shfl_sync(0xffffffffu, next, 0);
-    const uint32_t idx = batch * 32 + lane;
+    const uint32_t idx = batch * K + lane;
+    const bool mine = lane < K && idx < p.n_desc;
     SegDesc d{};
-    if (idx < p.n_desc) d = p.desc[idx];
-    const uint64_t len = idx < p.n_desc ? d.bytes : 0;
+    if (mine) d = p.desc[idx];
+    const uint64_t len = mine ? d.bytes : 0;
     uint64_t maxlen = len;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) maxlen = max(maxlen, __shfl_xor_sync(0xffffffffu, maxlen, o));
-    const uint32_t nblk = (uint32_t)((maxlen + 511) / 512);
+    const uint32_t nblk = (uint32_t)((maxlen + BLK - 1) / BLK);
     auto issue = [&](uint32_t b) {  // block b of every chunk of the batch into stage b % S
-      const uint32_t st = rows_s + (b % S) * 32 * XC_ROW;
+      const uint32_t st = rows_s + (b % S) * K * ROW;
 #pragma unroll 4
-      for (int c = 0; c < 32; ++c) {
+      for (int c = 0; c < K; ++c) {
         const uint64_t cl = __shfl_sync(0xffffffffu, len, c);
         const uint64_t cb = __shfl_sync(0xffffffffu, d.dev, c);
-        const uint64_t off = (uint64_t)b * 512 + lane * 16;
-        if (off < cl) {
-          const uint32_t nb = (uint32_t)(cl - off < 16 ? cl - off : 16);
-          cp_async16(st + c * XC_ROW + lane * 16, reinterpret_cast<const void*>(cb + off), nb);
+#pragma unroll
+        for (int j = 0; j < BLK / 512; ++j) {
+          const uint64_t off = (uint64_t)b * BLK + j * 512 + lane * 16;
+          if (off < cl) {
+            const uint32_t nb = (uint32_t)(cl - off < 16 ? cl - off : 16);
+            cp_async16(st + c * ROW + j * 512 + lane * 16, reinterpret_cast<const void*>(cb + off), nb);
+          }
         }
       }
       asm volatile("cp.async.commit_group;" ::: "memory");
@@ -1043,13 +1047,13 @@ __global__ void __launch_bounds__(W * 32) xxh_coop_kernel(const Params p) {
       else asm volatile("cp.async.commit_group;" ::: "memory");
       asm volatile("cp.async.wait_group %0;" ::"n"(S - 1) : "memory");
       __syncwarp();
-      const uint64_t s0 = (uint64_t)b * 16;
+      const uint64_t s0 = (uint64_t)b * SPB;
       if (s0 < stripes) {
-        const uint32_t ns = (uint32_t)(stripes - s0 < 16 ? stripes - s0 : 16);
-        const uint4* row = reinterpret_cast<const uint4*>(rows + ((b % S) * 32 + lane) * XC_ROW);
-        if (ns == 16) {  // a whole block: shared-memory loads four stripes ahead of the rounds
-#pragma unroll
-          for (int t0 = 0; t0 < 16; t0 += 4) {
+        const uint32_t ns = (uint32_t)(stripes - s0 < SPB ? stripes - s0 : SPB);
+        const uint4* row = reinterpret_cast<const uint4*>(rows + ((b % S) * K + lane) * ROW);
+        if (ns == SPB) {  // a whole block: shared-memory loads four stripes ahead of the rounds
+#pragma unroll 2
+          for (int t0 = 0; t0 < SPB; t0 += 4) {
             uint4 a[4], c[4];
 #pragma unroll
             for (int u = 0; u < 4; ++u) {
@@ -1077,7 +1081,7 @@ __global__ void __launch_bounds__(W * 32) xxh_coop_kernel(const Params p) {
     }
     asm volatile("cp.async.wait_group 0;" ::: "memory");
     __syncwarp();
-    if (idx < p.n_desc) xxh_finish<MODE>(p, d, v);
+    if (mine) xxh_finish<MODE>(p, d, v);
     batch = next;
   }
 }
@@ -1136,24 +1140,24 @@ static cudaError_t launch_xxh_dyn(const Params& p, int sm_count, cudaStream_t s)
   return cudaGetLastError();
 }
 
-template <int MODE, int W, int S>
+template <int MODE, int W, int S, int K = 32>
 static cudaError_t launch_xxh_coop(const Params& p, int sm_count, cudaStream_t s) {
-  constexpr size_t smem = (size_t)W * S * 32 * XC_ROW;
+  constexpr size_t smem = (size_t)W * S * K * (16384 / K + 16);
   if (!p.ticket) return cudaErrorInvalidValue;
   static unsigned long long attr_set = 0;
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
   if (!((attr_set >> (dev & 63)) & 1ull)) {
-    e = cudaFuncSetAttribute(xxh_coop_kernel<MODE, W, S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    e = cudaFuncSetAttribute(xxh_coop_kernel<MODE, W, S, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr_set |= 1ull << (dev & 63);
   }
-  const uint32_t n_batches = (p.n_desc + 31) / 32;
+  const uint32_t n_batches = (p.n_desc + K - 1) / K;
   const int grid = (int)std::max<uint32_t>(1, std::min<uint32_t>((uint32_t)sm_count, (n_batches + W - 1) / W));
   e = cudaMemsetAsync(p.ticket, 0, sizeof(unsigned int), s);
   if (e != cudaSuccess) return e;
-  xxh_coop_kernel<MODE, W, S><<<grid, W * 32, smem, s>>>(p);
+  xxh_coop_kernel<MODE, W, S, K><<<grid, W * 32, smem, s>>>(p);
   return cudaGetLastError();
 }
 
@@ -1202,6 +1206,8 @@ static int xxh_variant() {
   if (!strcmp(e, "coop")) return 12;   // 6 warps x 2 stages
   if (!strcmp(e, "coop3")) return 13;  // 4 warps x 3 stages
   if (!strcmp(e, "coop4")) return 14;  // 3 warps x 4 stages
+  if (!strcmp(e, "coopk16")) return 15;  // 6 warps x 2 stages, 16 chunks per warp (1-KiB runs)
+  if (!strcmp(e, "coopk8")) return 16;   // 6 warps x 2 stages, 8 chunks per warp (2-KiB runs)
   return 0;
 }
 
@@ -1223,6 +1229,8 @@ cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_
     case 12: return st ? launch_xxh_coop<HASH_STORE, 6, 2>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2>(p, sm_count, s);
     case 13: return st ? launch_xxh_coop<HASH_STORE, 4, 3>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 4, 3>(p, sm_count, s);
     case 14: return st ? launch_xxh_coop<HASH_STORE, 3, 4>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 3, 4>(p, sm_count, s);
+    case 15: return st ? launch_xxh_coop<HASH_STORE, 6, 2, 16>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 16>(p, sm_count, s);
+    case 16: return st ? launch_xxh_coop<HASH_STORE, 6, 2, 8>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 8>(p, sm_count, s);
     case 3: return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
     case 1: return st ? launch_xxh_lane<HASH_STORE, XK_U>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, XK_U>(p, sm_count, s);
     default: break;
@@ -1233,18 +1241,23 @@ cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_
   // once more than ~7 MB are in flight), with fewer chunks the
   // balanced 8-deep launch (per-lane rate = bytes in flight / latency), and with only a few thousand
   // chunks the warp-per-chunk TMA ring. From 2 MiB chunks the warp-cooperative kernel while there are
-  // enough 32-chunk batches for its warps (2 MiB: 3.9 vs 2.0 TB/s; 4 MiB: 2.5 vs 1.5), else the ring.
+  // enough batches for its warps (2 MiB: 4.3 vs 2.0 TB/s; 4 MiB: 3.1 vs 1.5; 8 MiB: 1.7 vs 1.0), else
+  // the ring.
   const uint32_t n = p.n_desc, many = (uint32_t)sm_count * 192u;
   if (p.chunk_bytes <= (256u << 10)) {
     if (n >= many) return st ? launch_xxh_lane<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8, true>(p, sm_count, s);
     return st ? launch_xxh_lane_bal<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8, true>(p, sm_count, s);
   }
-  if (p.chunk_bytes >= (2u << 20) && p.ticket) {  // big chunks: the warp-cooperative kernel while batches last
-    const uint32_t batches = (n + 31) / 32;
-    if (batches >= (uint32_t)sm_count * 5)
-      return st ? launch_xxh_coop<HASH_STORE, 6, 2>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2>(p, sm_count, s);
-    if (batches >= (uint32_t)sm_count * 2)
-      return st ? launch_xxh_coop<HASH_STORE, 4, 3>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 4, 3>(p, sm_count, s);
+  if (p.chunk_bytes >= (2u << 20) && p.ticket) {
+    // big chunks: the warp-cooperative kernel with as many chunks per warp (32 / 16 / 8: 4.9 / 3.6 /
+    // 2.4 GB/s per warp) as still keeps ~all 6 x SMs warps busy, else the ring
+    const uint32_t need = (uint32_t)sm_count * 6 * 85 / 100;
+    if (n / 32 >= need)
+      return st ? launch_xxh_coop<HASH_STORE, 6, 2, 32>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 32>(p, sm_count, s);
+    if (n / 16 >= need)
+      return st ? launch_xxh_coop<HASH_STORE, 6, 2, 16>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 16>(p, sm_count, s);
+    if (n / 8 >= need)
+      return st ? launch_xxh_coop<HASH_STORE, 6, 2, 8>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 8>(p, sm_count, s);
     return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
   }
   if (n >= many) return st ? launch_xxh_dyn<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 4>(p, sm_count, s);

@@ -35,7 +35,7 @@ print("variant ok")
 '''
 
 
-@pytest.mark.parametrize("variant", ["lane", "lane8", "ring", "bal", "bal8", "lanena", "lane8na", "balna", "bal8na", "dyn", "dyn8", "coop", "coop3", "coop4"])
+@pytest.mark.parametrize("variant", ["lane", "lane8", "ring", "bal", "bal8", "lanena", "lane8na", "balna", "bal8na", "dyn", "dyn8", "coop", "coop3", "coop4", "coopk16", "coopk8"])
 def test_xxh64_kernel_variant(variant):
     env = dict(os.environ, SWAP_XXH_KERNEL=variant)
     out = subprocess.run([sys.executable, "-c", SCRIPT, ROOT], capture_output=True, text=True, env=env, timeout=600)
