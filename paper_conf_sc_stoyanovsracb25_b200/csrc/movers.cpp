@@ -45,12 +45,15 @@ int grid_of(swap_ctx* c) { return c->cfg.grid_ctas ? (int)c->cfg.grid_ctas : 2 *
 // per-copy and per-launch costs make the single fused SM pass faster for small images.
 //   restore:    < 128 MiB SM;  < 2 GiB CE_BATCH (needs a non-default stream, else SM);  else CE_PIPE
 //   checkpoint: < 1 GiB SM;    else CE_PIPE
-// XXH64 is not combinable: with chunks > 1 MiB a pipeline group holds too few chunks for the side-stream
-// hash to keep up with the link, while the fused SM pass hashes every chunk in flight — SM then.
+// XXH64 is not combinable: with chunks > 4 MiB a pipeline group holds too few chunks for the side-stream
+// hash to keep up with the link (config B, 16 MiB: CE_PIPE swap-in 15 GB/s), so restores take one batch
+// copy plus one hash pass (CE_BATCH 50.7 GB/s vs SM 48.6) and checkpoints the fused SM pass (51.6 vs
+// 49.7). Up to 4 MiB the rule is the CRC one (config B, 2 / 4 MiB: CE_PIPE 54.6 / 54.2 vs SM 50.8 / 50.6).
 uint32_t resolve_mech(const swap_ctx* c, int dir, bool default_stream) {
   if (c->cfg.mechanism != SWAP_MECH_AUTO) return c->cfg.mechanism;
   const uint64_t S = c->plan.payload_bytes;
-  if (c->plan.kind == SWAP_CHECKSUM_XXH64 && c->plan.C > (1ull << 20)) return SWAP_MECH_SM;
+  if (c->plan.kind == SWAP_CHECKSUM_XXH64 && c->plan.C > (4ull << 20))
+    return (dir == 1 && S >= (128ull << 20) && !default_stream) ? SWAP_MECH_CE_BATCH : SWAP_MECH_SM;
   if (dir == 0) return S < (1ull << 30) ? SWAP_MECH_SM : SWAP_MECH_CE_PIPE;
   if (S < (128ull << 20)) return SWAP_MECH_SM;
   if (S < (2ull << 30)) return default_stream ? SWAP_MECH_SM : SWAP_MECH_CE_BATCH;
