@@ -510,13 +510,9 @@ __device__ __forceinline__ void ld32_v4x2_na(const uint8_t* p, uint32_t (&w)[8])
   asm("ld.global.nc.L1::no_allocate.v4.b32 {%0,%1,%2,%3}, [%4];"
       : "=r"(w[4]), "=r"(w[5]), "=r"(w[6]), "=r"(w[7]) : "l"(p + 16));
 }
-template <bool AL32, bool NA>
-__device__ __forceinline__ void ld32p(const uint8_t* p, uint32_t (&w)[8]) {
-  if (NA) {
-    if (AL32) ld32_na(p, w); else ld32_v4x2_na(p, w);
-  } else {
-    ld32a<AL32>(p, w);
-  }
+template <bool AL32>
+__device__ __forceinline__ void ld32na(const uint8_t* p, uint32_t (&w)[8]) {
+  if (AL32) ld32_na(p, w); else ld32_v4x2_na(p, w);
 }
 __device__ __forceinline__ uint32_t lds_at(uint32_t addr) {
   uint32_t v;
@@ -832,7 +828,6 @@ static cudaError_t launch_xxh_ring(const Params& p, int sm_count, cudaStream_t s
 // sector), U stripes in flight (4 or 8), loads that do not allocate in L1. Used for HASH_STORE /
 // HASH_CHECK when there are enough chunks to occupy the GPU; launch_xxh_hash picks the launch shape.
 constexpr int XK_THREADS = 256;
-constexpr int XK_U = 4;  // 128 B in flight per lane
 constexpr size_t XK_OFF_BAR = 2 * XK_THREADS * sizeof(SegDesc);
 constexpr size_t XK_SMEM = XK_OFF_BAR + 16;
 
@@ -848,20 +843,20 @@ __device__ __forceinline__ void xxh_stripe(uint64_t (&v)[4], const uint32_t (&w)
 // Stripes [0, end) of one chunk into the four accumulators. A U-deep software pipeline (each 256-bit
 // load consumed U stripes after issue) keeps U stripes per lane in flight; without it ptxas sinks each
 // load next to its use.
-template <bool AL32, int U, bool NA>
+template <bool AL32, int U>
 __device__ __forceinline__ void xxh_stripes(const uint8_t* src, uint64_t end, uint64_t (&v)[4]) {
   const uint64_t n = end / 32;
   uint64_t t = 0;
   if (n >= U) {
     uint32_t buf[U][8];
 #pragma unroll
-    for (int u = 0; u < U; ++u) ld32p<AL32, NA>(src + u * 32, buf[u]);
+    for (int u = 0; u < U; ++u) ld32na<AL32>(src + u * 32, buf[u]);
     for (; t + 2 * U <= n; t += U) {
       const uint8_t* q = src + (t + U) * 32;
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         xxh_stripe(v, buf[u]);
-        ld32p<AL32, NA>(q + u * 32, buf[u]);
+        ld32na<AL32>(q + u * 32, buf[u]);
       }
     }
 #pragma unroll
@@ -870,7 +865,7 @@ __device__ __forceinline__ void xxh_stripes(const uint8_t* src, uint64_t end, ui
   }
   for (; t < n; ++t) {
     uint32_t w[8];
-    ld32p<AL32, NA>(src + t * 32, w);
+    ld32na<AL32>(src + t * 32, w);
     xxh_stripe(v, w);
   }
 }
@@ -917,16 +912,16 @@ __device__ __forceinline__ void xxh_finish(const Params& p, const SegDesc& d, co
 }
 
 // One whole chunk (descriptor d) by one lane.
-template <int MODE, int U, bool NA>
+template <int MODE, int U>
 __device__ __forceinline__ void xxh_chunk(const Params& p, const SegDesc& d) {
   const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
   uint64_t v[4] = {P1 + P2, P2, 0, 0ull - P1};
   const uint64_t stripes_end = (uint64_t)d.bytes / 32 * 32;
-  if ((d.dev & 31) == 0) xxh_stripes<true, U, NA>(src, stripes_end, v); else xxh_stripes<false, U, NA>(src, stripes_end, v);
+  if ((d.dev & 31) == 0) xxh_stripes<true, U>(src, stripes_end, v); else xxh_stripes<false, U>(src, stripes_end, v);
   xxh_finish<MODE>(p, d, v);
 }
 
-template <int MODE, int U, int MAXT, bool NA>
+template <int MODE, int U, int MAXT>
 __global__ void __launch_bounds__(MAXT) xxh_lane_kernel(const Params p) {
   extern __shared__ __align__(128) uint8_t smem[];
   const uint32_t T = blockDim.x;
@@ -957,7 +952,7 @@ __global__ void __launch_bounds__(MAXT) xxh_lane_kernel(const Params p) {
     const uint32_t idx = r * per_round + first0 + tid;
     if (idx < p.n_desc) {
       const SegDesc d = sDesc[(r & 1) * T + tid];
-      xxh_chunk<MODE, U, NA>(p, d);
+      xxh_chunk<MODE, U>(p, d);
     }
     __syncthreads();
     if (tid == 0 && r + 2 < rounds) {
@@ -972,14 +967,14 @@ __global__ void __launch_bounds__(MAXT) xxh_lane_kernel(const Params p) {
 // behind it). The static launches hand every lane its chunks up front, and under load some SMs are
 // served more slowly than others: ncu on config B showed SMs idle for 8 % (4 deep) / 26 % (8 deep) of
 // the kernel waiting for the slowest one. Here fast lanes simply hash more chunks.
-template <int MODE, int U, int MAXT, bool NA>
+template <int MODE, int U, int MAXT>
 __global__ void __launch_bounds__(MAXT) xxh_dyn_kernel(const Params p) {
   const uint32_t lanes = gridDim.x * blockDim.x;
   uint32_t idx = blockIdx.x * blockDim.x + threadIdx.x;
   while (idx < p.n_desc) {
     const SegDesc d = p.desc[idx];
     const uint32_t next = lanes + atomicAdd(p.ticket, 1u);
-    xxh_chunk<MODE, U, NA>(p, d);
+    xxh_chunk<MODE, U>(p, d);
     idx = next;
   }
 }
@@ -1086,11 +1081,11 @@ __global__ void __launch_bounds__(W * 32) xxh_coop_kernel(const Params p) {
   }
 }
 
-template <int MODE, int U, bool NA = false>
+template <int MODE, int U>
 static cudaError_t launch_xxh_lane(const Params& p, int sm_count, cudaStream_t s) {
   const uint32_t blocks = (p.n_desc + XK_THREADS - 1) / XK_THREADS;
   const int grid = (int)std::max<uint32_t>(1, std::min<uint32_t>(blocks, (uint32_t)sm_count * 4));
-  xxh_lane_kernel<MODE, U, XK_THREADS, NA><<<grid, XK_THREADS, XK_SMEM, s>>>(p);
+  xxh_lane_kernel<MODE, U, XK_THREADS><<<grid, XK_THREADS, XK_SMEM, s>>>(p);
   return cudaGetLastError();
 }
 
@@ -1099,7 +1094,7 @@ static cudaError_t launch_xxh_lane(const Params& p, int sm_count, cudaStream_t s
 // above, config B's 197 CTAs ran at 11.2 ms or 20.7 ms depending on placement), chunks spread evenly:
 // T = ceil(n / SMs) lanes per SM, rounded to whole warps, capped by the register file.
 constexpr size_t XB_SMEM = 116 * 1024;
-template <int MODE, int U, bool NA = false>
+template <int MODE, int U>
 static cudaError_t launch_xxh_lane_bal(const Params& p, int sm_count, cudaStream_t s) {
   constexpr int MAXT = U >= 8 ? 640 : 1024;
   static unsigned long long attr_set = 0;
@@ -1107,8 +1102,7 @@ static cudaError_t launch_xxh_lane_bal(const Params& p, int sm_count, cudaStream
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
   if (!((attr_set >> (dev & 63)) & 1ull)) {
-    e = cudaFuncSetAttribute(xxh_lane_kernel<MODE, U, MAXT, NA>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)XB_SMEM);
+    e = cudaFuncSetAttribute(xxh_lane_kernel<MODE, U, MAXT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)XB_SMEM);
     if (e != cudaSuccess) return e;
     attr_set |= 1ull << (dev & 63);
   }
@@ -1119,16 +1113,16 @@ static cudaError_t launch_xxh_lane_bal(const Params& p, int sm_count, cudaStream
   // 148 CTAs of 341 lanes (every SM busy, a partial last warp) in 11.06 ms (in-process A/B, 8 reps)
   const uint32_t T = std::min<uint32_t>(MAXT, std::max<uint32_t>(32, ((per_sm + R - 1) / R + 31) / 32 * 32));
   const int grid = (int)std::min<uint32_t>((uint32_t)sm_count, (p.n_desc + T - 1) / T);
-  xxh_lane_kernel<MODE, U, MAXT, NA><<<grid, T, XB_SMEM, s>>>(p);
+  xxh_lane_kernel<MODE, U, MAXT><<<grid, T, XB_SMEM, s>>>(p);
   return cudaGetLastError();
 }
 
 // Dynamic lane launch: one CTA of T lanes per SM (SWAP_XXH_DYN_T overrides T, for measurements), the
 // ticket zeroed on the launching stream first.
-template <int MODE, int U, bool NA = true>
+template <int MODE, int U>
 static cudaError_t launch_xxh_dyn(const Params& p, int sm_count, cudaStream_t s) {
   constexpr int MAXT = U >= 8 ? 640 : 1024;
-  if (!p.ticket) return launch_xxh_lane_bal<MODE, U, NA>(p, sm_count, s);
+  if (!p.ticket) return launch_xxh_lane_bal<MODE, U>(p, sm_count, s);
   uint32_t T = U >= 8 ? 192 : 352;
   if (const char* e = getenv("SWAP_XXH_DYN_T")) T = std::max(32, std::min(MAXT, atoi(e)));
   const uint32_t per_sm = (p.n_desc + sm_count - 1) / sm_count;
@@ -1136,7 +1130,7 @@ static cudaError_t launch_xxh_dyn(const Params& p, int sm_count, cudaStream_t s)
   const int grid = (int)std::min<uint32_t>((uint32_t)sm_count, (p.n_desc + T - 1) / T);
   cudaError_t e = cudaMemsetAsync(p.ticket, 0, sizeof(unsigned int), s);
   if (e != cudaSuccess) return e;
-  xxh_dyn_kernel<MODE, U, MAXT, NA><<<grid, T, 0, s>>>(p);
+  xxh_dyn_kernel<MODE, U, MAXT><<<grid, T, 0, s>>>(p);
   return cudaGetLastError();
 }
 
@@ -1185,54 +1179,29 @@ static cudaError_t launch_t(const Params& p, int grid, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-// Kernel choice for XXH64 hash passes: 0 = automatic, 1 = lane per chunk (XK_U deep, up to 4 CTAs/SM),
-// 2 = the same 8 deep, 3 = TMA ring, 4/5 = balanced lane launch 4/8 deep (SWAP_XXH_KERNEL=lane|lane8|
-// ring|bal|bal8 forces one, for measurements and tests; read at every launch so one process can
-// interleave variants).
+// Kernel choice for XXH64 hash passes: automatic (below), or forced with SWAP_XXH_KERNEL for
+// measurements and tests (read at every launch, so one process can interleave variants).
 static int xxh_variant() {
   const char* e = getenv("SWAP_XXH_KERNEL");
   if (!e) return 0;
-  if (!strcmp(e, "lane")) return 1;
-  if (!strcmp(e, "lane8")) return 2;
-  if (!strcmp(e, "ring")) return 3;
-  if (!strcmp(e, "bal")) return 4;
-  if (!strcmp(e, "bal8")) return 5;
-  if (!strcmp(e, "lanena")) return 6;
-  if (!strcmp(e, "lane8na")) return 7;
-  if (!strcmp(e, "balna")) return 8;
-  if (!strcmp(e, "bal8na")) return 9;
-  if (!strcmp(e, "dyn")) return 10;
-  if (!strcmp(e, "dyn8")) return 11;
-  if (!strcmp(e, "coop")) return 12;   // 6 warps x 2 stages
-  if (!strcmp(e, "coop3")) return 13;  // 4 warps x 3 stages
-  if (!strcmp(e, "coop4")) return 14;  // 3 warps x 4 stages
-  if (!strcmp(e, "coopk16")) return 15;  // 6 warps x 2 stages, 16 chunks per warp (1-KiB runs)
-  if (!strcmp(e, "coopk8")) return 16;   // 6 warps x 2 stages, 8 chunks per warp (2-KiB runs)
+  const char* names[] = {"lane8", "bal", "bal8", "dyn", "coop", "coop16", "coop8", "ring"};
+  for (int i = 0; i < 8; ++i)
+    if (!strcmp(e, names[i])) return i + 1;
   return 0;
 }
 
 cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_t s) {
   if (p.n_desc == 0) return cudaSuccess;
   const bool st = mode == HASH_STORE;
-  switch (xxh_variant()) {
-    case 2: return st ? launch_xxh_lane<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8>(p, sm_count, s);
-    case 4: return st ? launch_xxh_lane_bal<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 4>(p, sm_count, s);
-    case 5: return st ? launch_xxh_lane_bal<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8>(p, sm_count, s);
-    case 6: return st ? launch_xxh_lane<HASH_STORE, 4, true>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 4, true>(p, sm_count, s);
-    case 7: return st ? launch_xxh_lane<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8, true>(p, sm_count, s);
-    case 8: return st ? launch_xxh_lane_bal<HASH_STORE, 4, true>(p, sm_count, s)
-                      : launch_xxh_lane_bal<HASH_CHECK, 4, true>(p, sm_count, s);
-    case 9: return st ? launch_xxh_lane_bal<HASH_STORE, 8, true>(p, sm_count, s)
-                      : launch_xxh_lane_bal<HASH_CHECK, 8, true>(p, sm_count, s);
-    case 10: return st ? launch_xxh_dyn<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 4>(p, sm_count, s);
-    case 11: return st ? launch_xxh_dyn<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 8>(p, sm_count, s);
-    case 12: return st ? launch_xxh_coop<HASH_STORE, 6, 2>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2>(p, sm_count, s);
-    case 13: return st ? launch_xxh_coop<HASH_STORE, 4, 3>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 4, 3>(p, sm_count, s);
-    case 14: return st ? launch_xxh_coop<HASH_STORE, 3, 4>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 3, 4>(p, sm_count, s);
-    case 15: return st ? launch_xxh_coop<HASH_STORE, 6, 2, 16>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 16>(p, sm_count, s);
-    case 16: return st ? launch_xxh_coop<HASH_STORE, 6, 2, 8>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 8>(p, sm_count, s);
-    case 3: return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
-    case 1: return st ? launch_xxh_lane<HASH_STORE, XK_U>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, XK_U>(p, sm_count, s);
+  switch (xxh_variant()) {  // forced: lane8 | bal | bal8 | dyn | coop | coop16 | coop8 | ring
+    case 1: return st ? launch_xxh_lane<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8>(p, sm_count, s);
+    case 2: return st ? launch_xxh_lane_bal<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 4>(p, sm_count, s);
+    case 3: return st ? launch_xxh_lane_bal<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8>(p, sm_count, s);
+    case 4: return st ? launch_xxh_dyn<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 4>(p, sm_count, s);
+    case 5: return st ? launch_xxh_coop<HASH_STORE, 6, 2, 32>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 32>(p, sm_count, s);
+    case 6: return st ? launch_xxh_coop<HASH_STORE, 6, 2, 16>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 16>(p, sm_count, s);
+    case 7: return st ? launch_xxh_coop<HASH_STORE, 6, 2, 8>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 8>(p, sm_count, s);
+    case 8: return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
     default: break;
   }
   // Measured on config B and an 8-GiB cut of it (profiles/r01_xxh_variants.md): up to
@@ -1245,8 +1214,8 @@ cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_
   // the ring.
   const uint32_t n = p.n_desc, many = (uint32_t)sm_count * 192u;
   if (p.chunk_bytes <= (256u << 10)) {
-    if (n >= many) return st ? launch_xxh_lane<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8, true>(p, sm_count, s);
-    return st ? launch_xxh_lane_bal<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8, true>(p, sm_count, s);
+    if (n >= many) return st ? launch_xxh_lane<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8>(p, sm_count, s);
+    return st ? launch_xxh_lane_bal<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8>(p, sm_count, s);
   }
   if (p.chunk_bytes >= (2u << 20) && p.ticket) {
     // big chunks: the warp-cooperative kernel with as many chunks per warp (32 / 16 / 8: 4.9 / 3.6 /
@@ -1262,7 +1231,7 @@ cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_
   }
   if (n >= many) return st ? launch_xxh_dyn<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 4>(p, sm_count, s);
   if (hash_xxh_lane_ok(sm_count, n))
-    return st ? launch_xxh_lane_bal<HASH_STORE, 8, true>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8, true>(p, sm_count, s);
+    return st ? launch_xxh_lane_bal<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8>(p, sm_count, s);
   return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
 }
 

@@ -95,7 +95,7 @@ print("skew ok")
 '''
 
 
-@pytest.mark.parametrize("variant", ["lane", "ring"])
+@pytest.mark.parametrize("variant", ["lane8", "bal", "dyn", "coop", "coop16", "coop8", "ring"])
 def test_skewed_xxh64_hash_kernels(variant):
     """The XXH64 HBM hash kernels forced in turn (SWAP_XXH_KERNEL) on 16-B-aligned chunk starts."""
     env = dict(os.environ, SWAP_XXH_KERNEL=variant)

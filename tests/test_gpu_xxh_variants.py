@@ -1,4 +1,5 @@
-"""Each XXH64 HBM hash kernel (lane-per-chunk 4 or 8 deep, balanced lane launch, TMA ring) forced in turn through
+"""Each XXH64 HBM hash kernel (lane per chunk 8 deep; balanced 4 / 8 deep; dynamic; warp-cooperative with
+32 / 16 / 8 chunks per warp; TMA ring) forced in turn through
 SWAP_XXH_KERNEL, in a subprocess, on many small chunks and on few large ones: images and verify
 results bit-exact against the oracle."""
 import os
@@ -35,7 +36,7 @@ print("variant ok")
 '''
 
 
-@pytest.mark.parametrize("variant", ["lane", "lane8", "ring", "bal", "bal8", "lanena", "lane8na", "balna", "bal8na", "dyn", "dyn8", "coop", "coop3", "coop4", "coopk16", "coopk8"])
+@pytest.mark.parametrize("variant", ["lane8", "bal", "bal8", "dyn", "coop", "coop16", "coop8", "ring"])
 def test_xxh64_kernel_variant(variant):
     env = dict(os.environ, SWAP_XXH_KERNEL=variant)
     out = subprocess.run([sys.executable, "-c", SCRIPT, ROOT], capture_output=True, text=True, env=env, timeout=600)

@@ -33,6 +33,15 @@ with swap.Swapper(regions, chunk_bytes=1024, checksum=2, mechanism="ce_region") 
     sw.checkpoint(s)
     sw.restore(s)
     assert sw.verify(s)["status"] == 0
+# every XXH64 hash kernel, forced per launch through SWAP_XXH_KERNEL (the CE movers hash from HBM)
+for v in ("lane8", "bal", "bal8", "dyn", "coop", "coop16", "coop8", "ring"):
+    os.environ["SWAP_XXH_KERNEL"] = v
+    with swap.Swapper(regions, chunk_bytes=1024, checksum=2, mechanism="ce_region") as sw, torch.cuda.stream(s):
+        sw.checkpoint(s)
+        poison(arena, specs, offs)
+        sw.restore(s)
+        assert sw.verify(s)["status"] == 0, v
+os.environ.pop("SWAP_XXH_KERNEL")
 # VMM arenas + full-duplex exchange
 def engine(seed):
     sp = W.scaled(W.config_b(), 48 << 20)
