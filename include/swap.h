@@ -179,6 +179,17 @@ SWAP_API swap_status swap_verify(swap_ctx_t* ctx, swap_stream_t stream, int hbm_
 /* Sets region `region_index`'s policy (index in registration order). Only between
  * swap_register_regions and the first checkpoint (ESTATE otherwise). */
 SWAP_API swap_status swap_set_region_policy(swap_ctx_t* ctx, uint32_t region_index, uint32_t policy);
+/* Touched-block masks (NEXT-3, "move only touched KV blocks"; reading 25): keep[j] = 0 marks
+ * chunk j of SAVE region `region_index` as holding no state the engine needs (an unused KV block). The
+ * mask takes effect at the NEXT checkpoint, which captures such chunks as zeros exactly like DISCARD —
+ * image bytes 0 (zero-filled in stream order if an earlier checkpoint left data there), c_g = checksum of
+ * a zero chunk — and moves only the kept chunks; the restore of that checkpoint moves only the kept chunks
+ * and zero-fills the others on the device; the HBM pass checks every chunk. keep = NULL keeps all.
+ * n must equal the region's chunk count ceil(bytes / C) (EINVAL otherwise, or if the region's policy is
+ * not SAVE; changing the policy resets the mask). Any state after registration except a checkpoint
+ * that is not yet synced (ESTATE). swap_import/swap_load restore the whole imported image and re-apply
+ * the mask at the next checkpoint. The array is copied. */
+SWAP_API swap_status swap_set_chunk_mask(swap_ctx_t* ctx, uint32_t region_index, const uint8_t* keep, uint64_t n);
 
 /* Selects the data mover for later calls (SWAP_MECH_*). The image format is unchanged. */
 SWAP_API swap_status swap_set_mechanism(swap_ctx_t* ctx, uint32_t mechanism);

@@ -194,17 +194,26 @@ def checkpoint(regions, mem: np.ndarray, mem_base: int, kind: int, chunk_bytes: 
 SAVE, SAVE_ONCE, DISCARD = 0, 1, 2
 
 
-def policy_view(regions, policies, mem_now: np.ndarray, mem_first: np.ndarray, mem_base: int) -> np.ndarray:
+def policy_view(regions, policies, mem_now: np.ndarray, mem_first: np.ndarray, mem_base: int,
+                chunk_bytes: int | None = None, masks: dict | None = None) -> np.ndarray:
     """The bytes a checkpoint captures under per-region swap policies (reading 24):
     SAVE -> the region now; SAVE_ONCE -> the region as it was at the first checkpoint;
-    DISCARD -> zeros. Feed the result to checkpoint()."""
+    DISCARD -> zeros. Touched-chunk masks (reading 25): masks = {region index: keep[0..n_i)} for SAVE
+    regions; chunk j with keep[j] == 0 covers region bytes [j*C, min((j+1)*C, bytes)) (SURVEY §8(c)
+    step 3) and is captured as zeros, like DISCARD. Feed the result to checkpoint()."""
     view = mem_now.copy()
-    for (rid, addr, nbytes, kind), pol in zip(regions, policies):
+    for i, ((rid, addr, nbytes, kind), pol) in enumerate(zip(regions, policies)):
         lo = addr - mem_base
         if pol == DISCARD:
             view[lo:lo + nbytes] = 0
         elif pol == SAVE_ONCE:
             view[lo:lo + nbytes] = mem_first[lo:lo + nbytes]
+        elif masks and i in masks and masks[i] is not None:
+            keep = masks[i]
+            assert len(keep) == -(-nbytes // chunk_bytes), "one mask entry per chunk"
+            for j, k in enumerate(keep):
+                if not k:
+                    view[lo + j * chunk_bytes:lo + min((j + 1) * chunk_bytes, nbytes)] = 0
     return view
 
 

@@ -62,6 +62,13 @@ struct swap_ctx {
   // device-side work state; sets: all regions (verify), SAVE|SAVE_ONCE (first checkpoint, restore),
   // SAVE (later checkpoints), DISCARD chunks hashed from a zero buffer (their c_g)
   std::vector<uint32_t> policy;
+  // chunk masks (swap_set_chunk_mask, NEXT-3): keep = the mask of the sets in use (last checkpoint's),
+  // next_keep = the mask the next checkpoint applies; img_zero = the chunk's image bytes are known zero
+  std::vector<uint8_t> keep, next_keep, img_zero;
+  bool mask_dirty = false;
+  std::vector<Span> zero_spans;  // device ranges a restore zero-fills (DISCARD regions, masked chunks)
+  swk::ZSpan* d_zspans = nullptr;  // the same ranges cut into <= 1 MiB pieces for launch_zero_fill
+  uint32_t n_zspans = 0;
   DescSet s_all, s_move, s_save, s_zero;
   bool first_ckpt_done = false;
   uint8_t* d_zero = nullptr;
@@ -113,6 +120,7 @@ int hash_kind(swap_ctx* c);
 swap_status launch(swap_ctx* c, int mode, int kind, const swk::Params& p, cudaStream_t s);
 swap_status memcpy_dir(swap_ctx* c, const Span& sp, int dir, cudaStream_t s);
 swap_status ce_copy(swap_ctx* c, DescSet& S, int dir, cudaStream_t s);
+swap_status copy_spans(swap_ctx* c, const std::vector<Span>& spans, int dir, cudaStream_t s);
 swap_status map_spans(swap_ctx* c, const std::vector<Span>& spans);
 swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, cudaStream_t s);
 swap_status collect_timing(swap_ctx* c, int p);
@@ -123,5 +131,8 @@ uint32_t auto_seg(const swap_ctx* c, uint64_t payload);
 void free_helpers(swap_ctx* c);
 void release(swap_ctx* c);
 swap_status build_sets(swap_ctx* c);
+swap_status apply_mask(swap_ctx* c, cudaStream_t s, bool* hash_zero);
+void note_gathered(swap_ctx* c, const DescSet& S);
+swap_status zero_fill_device(swap_ctx* c, cudaStream_t s);
 
 }  // namespace swc

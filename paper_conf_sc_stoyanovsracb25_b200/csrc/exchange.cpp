@@ -51,6 +51,8 @@ swap_status swap_exchange(swap_ctx_t* const* victims, size_t nv, swap_ctx_t* in,
   swap_status st;
   for (size_t i = 0; i < nv; ++i) {
     swap_ctx* v = victims[i];
+    bool hash_zero = false;
+    if ((st = apply_mask(v, so, &hash_zero)) != SWAP_OK) return st;
     DescSet& S = v->first_ckpt_done ? v->s_save : v->s_move;
     vsets[i] = &S;
     swap_arena* A = v->arena;
@@ -69,7 +71,7 @@ swap_status swap_exchange(swap_ctx_t* const* victims, size_t nv, swap_ctx_t* in,
       if ((st = swarena::unmap_slab(A, s)) != SWAP_OK) return cuda_fail(v, cudaErrorUnknown, "slab release");
     }
     CUDA_TRY(v, cudaEventRecord(v->ev[0], so));
-    if (!v->first_ckpt_done && v->s_zero.n_desc &&
+    if (hash_zero && v->s_zero.n_desc &&
         (st = launch(v, swk::HASH_STORE, hash_kind(v), base_params(v, v->s_zero), so)) != SWAP_OK)
       return st;
     for (size_t gi = 0; gi < S.groups.size(); ++gi) {
@@ -79,8 +81,7 @@ swap_status swap_exchange(swap_ctx_t* const* victims, size_t nv, swap_ctx_t* in,
       p.partial = v->d_partial + G.d0;
       p.n_desc = G.d1 - G.d0;
       if ((st = launch(v, swk::HASH_STORE, hash_kind(v), p, so)) != SWAP_OK) return st;
-      for (const Span& sp : G.spans)
-        if ((st = memcpy_dir(v, sp, 0, so)) != SWAP_OK) return st;
+      if ((st = copy_spans(v, G.spans, 0, so)) != SWAP_OK) return st;
       CUDA_TRY(v, cudaEventRecord(S.group_ev[gi], so));
       Release r{S.group_ev[gi], A, {}};
       for (uint64_t s = 0; s < last.size(); ++s)
@@ -89,6 +90,7 @@ swap_status swap_exchange(swap_ctx_t* const* victims, size_t nv, swap_ctx_t* in,
     }
     CUDA_TRY(v, cudaEventRecord(v->ev[1], so));
     v->pending[0] = true;
+    note_gathered(v, S);
     v->first_ckpt_done = true;
     v->st = St::CKPT_PENDING;
   }
@@ -142,20 +144,16 @@ swap_status swap_exchange(swap_ctx_t* const* victims, size_t nv, swap_ctx_t* in,
     CUDA_TRY(in, cudaMemsetAsync(&in->d_status->n_bad, 0, 8, si));
     CUDA_TRY(in, cudaMemsetAsync(&in->d_status->first_bad, 0xFF, 8, si));
     CUDA_TRY(in, cudaEventRecord(in->ev[2], si));
-    for (size_t i = 0; i < in->policy.size(); ++i)
-      if (in->policy[i] == SWAP_POLICY_DISCARD && in->plan.regions[i].r.bytes) {
-        const auto& r = in->plan.regions[i].r;
-        if ((st = acquire(r.dev_addr, r.dev_addr + r.bytes)) != SWAP_OK) return st;
-        CUDA_TRY(in, cudaMemsetAsync(reinterpret_cast<void*>(r.dev_addr), 0, r.bytes, si));
-      }
+    for (const Span& z : in->zero_spans)  // DISCARD regions and masked chunks come back as zeros
+      if ((st = acquire(z.dev, z.dev + z.bytes)) != SWAP_OK) return st;
+    if ((st = zero_fill_device(in, si)) != SWAP_OK) return st;
     CUDA_TRY(in, cudaEventRecord(in->ev_fork, si));
     CUDA_TRY(in, cudaStreamWaitEvent(in->side, in->ev_fork, 0));
     for (size_t gi = 0; gi < S.groups.size(); ++gi) {
       const Group& G = S.groups[gi];
       for (const Span& sp : G.spans)
         if ((st = acquire(sp.dev, sp.dev + sp.bytes)) != SWAP_OK) return st;
-      for (const Span& sp : G.spans)
-        if ((st = memcpy_dir(in, sp, 1, si)) != SWAP_OK) return st;
+      if ((st = copy_spans(in, G.spans, 1, si)) != SWAP_OK) return st;
       CUDA_TRY(in, cudaEventRecord(S.group_ev[gi], si));
       CUDA_TRY(in, cudaStreamWaitEvent(in->side, S.group_ev[gi], 0));
       swk::Params p = base;

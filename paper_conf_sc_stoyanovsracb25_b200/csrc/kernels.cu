@@ -1253,4 +1253,24 @@ cudaError_t launch_mover(int mode, int kind, const Params& p, int grid, cudaStre
   return cudaErrorInvalidValue;
 }
 
+// One warp per span (warp-strided over the list), 16-B stores by all 32 lanes, ragged tail bytewise.
+__global__ void __launch_bounds__(256) zero_fill_kernel(const ZSpan* __restrict__ spans, uint32_t n) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t warps = gridDim.x * (blockDim.x >> 5);
+  for (uint32_t w = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); w < n; w += warps) {
+    const uint64_t dst = spans[w].dst, bytes = spans[w].bytes;
+    uint4* v = reinterpret_cast<uint4*>(dst);
+    const uint64_t nv = bytes >> 4;
+    for (uint64_t i = lane; i < nv; i += 32) v[i] = make_uint4(0u, 0u, 0u, 0u);
+    for (uint64_t i = (nv << 4) + lane; i < bytes; i += 32) reinterpret_cast<uint8_t*>(dst)[i] = 0;
+  }
+}
+
+cudaError_t launch_zero_fill(const ZSpan* spans, uint32_t n, int sm_count, cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  const uint32_t grid = (uint32_t)std::min<uint64_t>((uint64_t)sm_count * 8, (n + 7) / 8);
+  zero_fill_kernel<<<grid, 256, 0, s>>>(spans, n);
+  return cudaGetLastError();
+}
+
 }  // namespace swk

@@ -92,4 +92,13 @@ size_t mover_smem_bytes(int kind);
 bool hash_xxh_lane_ok(int sm_count, uint32_t n_desc);
 cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_t stream);
 
+// Zero-fill of a span list (DISCARD regions and masked chunks on the device at restore; stale masked
+// chunks of the mapped host image at checkpoint): one launch instead of one cudaMemsetAsync per span.
+// dst must be 16-B aligned; bytes arbitrary (split into pieces of <= kZeroPiece by the host).
+struct ZSpan {
+  uint64_t dst, bytes;
+};
+constexpr uint64_t kZeroPiece = 1ull << 20;
+cudaError_t launch_zero_fill(const ZSpan* spans, uint32_t n, int sm_count, cudaStream_t stream);
+
 }  // namespace swk

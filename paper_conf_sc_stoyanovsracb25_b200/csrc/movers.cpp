@@ -3,6 +3,7 @@
 #include <sys/mman.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -132,13 +133,49 @@ swap_status ce_copy(swap_ctx* c, DescSet& S, int dir, cudaStream_t s) {
 swap_status map_spans(swap_ctx* c, const std::vector<Span>& spans) {
   if (!c->arena || swarena::resident(c->arena)) return SWAP_OK;
   for (const Span& sp : spans) {
-    if (!swarena::contains(c->arena, sp.dev, sp.dev + sp.bytes)) continue;
+    if (!sp.bytes || !swarena::contains(c->arena, sp.dev, sp.dev + sp.bytes)) continue;
+    bool mapped = true;  // skip the driver round trip for spans on slabs already mapped
+    for (uint64_t k = swarena::slab_of(c->arena, sp.dev); mapped && k <= swarena::slab_of(c->arena, sp.dev + sp.bytes - 1); ++k)
+      mapped = swarena::slab_mapped(c->arena, k);
+    if (mapped) continue;
     swap_status st = swarena::map_dev_range(c->arena, sp.dev, sp.dev + sp.bytes);
     if (st != SWAP_OK) {
       c->err = "re-acquiring arena HBM failed";
       return st;
     }
   }
+  return SWAP_OK;
+}
+
+// The copies of one pipeline group. A restore group fragmented into many spans (touched-chunk masks, many
+// small regions) goes to the copy engine as one cudaMemcpyBatchAsync: per-copy submission costs dominate
+// ~1-MiB cudaMemcpyAsync calls. Checkpoints keep per-span copies (batched D2H measured slower);
+// the legacy default stream cannot take batches.
+swap_status copy_spans(swap_ctx* c, const std::vector<Span>& spans, int dir, cudaStream_t s) {
+  if (spans.size() <= 4 || s == nullptr || dir == 0) {
+    for (const Span& sp : spans) {
+      swap_status st = memcpy_dir(c, sp, dir, s);
+      if (st != SWAP_OK) return st;
+    }
+    return SWAP_OK;
+  }
+  std::vector<void*> dst(spans.size()), src(spans.size());
+  std::vector<size_t> bytes(spans.size());
+  for (size_t i = 0; i < spans.size(); ++i) {
+    void* dev = reinterpret_cast<void*>(spans[i].dev);
+    dst[i] = dir == 0 ? static_cast<void*>(spans[i].host) : dev;
+    src[i] = dir == 0 ? dev : static_cast<void*>(spans[i].host);
+    bytes[i] = spans[i].bytes;
+  }
+  cudaMemcpyAttributes attr;
+  std::memset(&attr, 0, sizeof(attr));
+  attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
+  attr.srcLocHint.type = dir == 0 ? cudaMemLocationTypeDevice : cudaMemLocationTypeHost;
+  attr.srcLocHint.id = dir == 0 ? c->cfg.device : 0;
+  attr.dstLocHint.type = dir == 0 ? cudaMemLocationTypeHost : cudaMemLocationTypeDevice;
+  attr.dstLocHint.id = dir == 0 ? 0 : c->cfg.device;
+  size_t attr_idx = 0, fail_idx = 0;
+  CUDA_TRY(c, cudaMemcpyBatchAsync(dst.data(), src.data(), bytes.data(), spans.size(), &attr, &attr_idx, 1, &fail_idx, s));
   return SWAP_OK;
 }
 
@@ -178,8 +215,7 @@ swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, c
       if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, c->side)) != SWAP_OK) return st;
       continue;
     }
-    for (const Span& sp : G.spans)
-      if ((st = memcpy_dir(c, sp, dir, s)) != SWAP_OK) return st;
+    if ((st = copy_spans(c, G.spans, dir, s)) != SWAP_OK) return st;
     if (dir == 1) {
       CUDA_TRY(c, cudaEventRecord(S.group_ev[g], s));
       CUDA_TRY(c, cudaStreamWaitEvent(c->side, S.group_ev[g], 0));
@@ -266,6 +302,8 @@ void release(swap_ctx* c) {
   free_set(c->s_all);
   if (c->d_zero) cudaFree(c->d_zero);
   c->d_zero = nullptr;
+  if (c->d_zspans) cudaFree(c->d_zspans);
+  c->d_zspans = nullptr;
   if (c->d_partial) cudaFree(c->d_partial);
   if (c->d_arrive) cudaFree(c->d_arrive);
   if (c->d_status) cudaFree(c->d_status);
@@ -297,10 +335,16 @@ static swap_status build_set(swap_ctx* c, DescSet* S, Pick pick, bool zero_src) 
   uint64_t cur_bytes = 0;
   for (size_t i = 0; i < P.regions.size(); ++i) {
     const auto& r = P.regions[i];
-    if (!pick(i) || r.r.bytes == 0) continue;
-    S->region_spans.push_back(Span{r.r.dev_addr, c->image + r.off, r.r.bytes});
+    if (r.r.bytes == 0) continue;
     for (uint64_t j = 0; j < r.nchunks; ++j) {
+      if (!pick(i, r.first + j)) continue;
       const uint64_t lo = j * P.C, len = std::min<uint64_t>(P.C, r.r.bytes - lo);
+      // CE_REGION spans: runs of picked chunks (a whole region unless chunk masks cut it)
+      if (!S->region_spans.empty() && S->region_spans.back().dev + S->region_spans.back().bytes == r.r.dev_addr + lo &&
+          S->region_spans.back().host + S->region_spans.back().bytes == c->image + r.off + lo)
+        S->region_spans.back().bytes += len;
+      else
+        S->region_spans.push_back(Span{r.r.dev_addr + lo, c->image + r.off + lo, len});
       const uint32_t nseg = (uint32_t)((len + seg - 1) / seg);
       for (uint32_t s = 0; s < nseg; ++s) {
         swk::SegDesc d;
@@ -352,7 +396,20 @@ static DescSet alias_of(const DescSet& S) {
   return a;
 }
 
-// (Re)builds every set from the current policies.
+static void cut_pieces(uint64_t dst, uint64_t bytes, std::vector<swk::ZSpan>* out) {
+  for (uint64_t o = 0; o < bytes; o += swk::kZeroPiece)
+    out->push_back(swk::ZSpan{dst + o, std::min<uint64_t>(swk::kZeroPiece, bytes - o)});
+}
+
+// Zero-fills every DISCARD region and masked chunk on the device: one kernel launch.
+swap_status zero_fill_device(swap_ctx* c, cudaStream_t s) {
+  if (!c->n_zspans) return SWAP_OK;
+  CUDA_TRY(c, swk::launch_zero_fill(c->d_zspans, c->n_zspans, c->sm_count, s));
+  ++c->launches;
+  return SWAP_OK;
+}
+
+// (Re)builds every set from the current policies and chunk masks (c->keep).
 swap_status build_sets(swap_ctx* c) {
   free_set(c->s_move);
   free_set(c->s_save);
@@ -363,40 +420,117 @@ swap_status build_sets(swap_ctx* c) {
     c->d_zero = nullptr;
   }
   const auto& pol = c->policy;
-  bool any_once = false, any_discard = false;
+  const auto& P = c->plan;
+  bool any_once = false, any_zero = false;
   uint64_t zero_bytes = 0;
+  c->zero_spans.clear();
   for (size_t i = 0; i < pol.size(); ++i) {
+    const auto& r = P.regions[i];
     any_once |= pol[i] == SWAP_POLICY_SAVE_ONCE;
-    if (pol[i] == SWAP_POLICY_DISCARD) {
-      any_discard = true;
-      zero_bytes = std::max<uint64_t>(zero_bytes, std::min<uint64_t>(c->plan.C, c->plan.regions[i].r.bytes));
+    for (uint64_t j = 0; j < r.nchunks; ++j) {
+      if (pol[i] != SWAP_POLICY_DISCARD && c->keep[r.first + j]) continue;
+      // a zero chunk: DISCARD region or masked-out chunk — restored by zero-filling, hashed from d_zero
+      any_zero = true;
+      const uint64_t lo = j * P.C, len = std::min<uint64_t>(P.C, r.r.bytes - lo);
+      zero_bytes = std::max<uint64_t>(zero_bytes, len);
+      std::vector<Span>& z = c->zero_spans;
+      if (!z.empty() && z.back().dev + z.back().bytes == r.r.dev_addr + lo)
+        z.back().bytes += len;
+      else
+        z.push_back(Span{r.r.dev_addr + lo, c->image + r.off + lo, len});
     }
   }
-  swap_status st = build_set(c, &c->s_all, [](size_t) { return true; }, false);
+  auto keep = [&](size_t i, uint64_t g) { return pol[i] != SWAP_POLICY_DISCARD && c->keep[g]; };
+  swap_status st = build_set(c, &c->s_all, [](size_t, uint64_t) { return true; }, false);
   if (st != SWAP_OK) return st;
-  if (!any_once && !any_discard) {
+  if (!any_once && !any_zero) {
     c->s_move = alias_of(c->s_all);
     c->s_save = alias_of(c->s_all);
   } else {
-    st = build_set(c, &c->s_move, [&](size_t i) { return pol[i] != SWAP_POLICY_DISCARD; }, false);
+    st = build_set(c, &c->s_move, keep, false);
     if (st != SWAP_OK) return st;
     if (any_once) {
-      st = build_set(c, &c->s_save, [&](size_t i) { return pol[i] == SWAP_POLICY_SAVE; }, false);
+      st = build_set(c, &c->s_save, [&](size_t i, uint64_t g) { return pol[i] == SWAP_POLICY_SAVE && keep(i, g); },
+                     false);
       if (st != SWAP_OK) return st;
     } else {
       c->s_save = alias_of(c->s_move);
     }
   }
-  if (any_discard) {
+  if (any_zero) {
     CUDA_TRY(c, cudaMalloc(&c->d_zero, std::max<uint64_t>(16, (zero_bytes + 31) & ~31ull)));
     CUDA_TRY(c, cudaMemset(c->d_zero, 0, std::max<uint64_t>(16, (zero_bytes + 31) & ~31ull)));
-    st = build_set(c, &c->s_zero, [&](size_t i) { return pol[i] == SWAP_POLICY_DISCARD; }, true);
+    st = build_set(c, &c->s_zero, [&](size_t i, uint64_t g) { return !keep(i, g); }, true);
     if (st != SWAP_OK) return st;
+  }
+  if (c->d_zspans) cudaFree(c->d_zspans);
+  c->d_zspans = nullptr;
+  std::vector<swk::ZSpan> pieces;
+  for (const Span& z : c->zero_spans) cut_pieces(z.dev, z.bytes, &pieces);
+  c->n_zspans = (uint32_t)pieces.size();
+  if (!pieces.empty()) {
+    CUDA_TRY(c, cudaMalloc(&c->d_zspans, pieces.size() * sizeof(swk::ZSpan)));
+    CUDA_TRY(c, cudaMemcpy(c->d_zspans, pieces.data(), pieces.size() * sizeof(swk::ZSpan), cudaMemcpyHostToDevice));
   }
   if (c->d_partial) cudaFree(c->d_partial);
   c->d_partial = nullptr;
   CUDA_TRY(c, cudaMalloc(&c->d_partial, std::max<size_t>(1, c->s_all.n_desc) * 4));
   return SWAP_OK;
+}
+
+// Chunk masks (swap_set_chunk_mask) take effect at the next checkpoint: rebuilds the sets for the new
+// mask and zero-fills, in stream order, the image bytes of chunks that are masked now but hold data from
+// an earlier checkpoint (their image bytes must read as zeros, reading 25). *hash_zero: the zero chunks'
+// checksums must be (re)written by this checkpoint.
+swap_status apply_mask(swap_ctx* c, cudaStream_t s, bool* hash_zero) {
+  *hash_zero = !c->first_ckpt_done;
+  if (!c->mask_dirty) return SWAP_OK;
+  const auto& P = c->plan;
+  std::vector<swk::ZSpan> pieces;  // image bytes of chunks masked now that still hold older data
+  for (size_t i = 0; i < P.regions.size(); ++i) {
+    const auto& r = P.regions[i];
+    uint64_t run_lo = 0, run_len = 0;
+    for (uint64_t j = 0; j < r.nchunks; ++j) {
+      const uint64_t g = r.first + j, lo = j * P.C, len = std::min<uint64_t>(P.C, r.r.bytes - lo);
+      if (c->next_keep[g] || c->img_zero[g]) continue;
+      if (run_len && run_lo + run_len != lo) {
+        pieces.push_back(swk::ZSpan{reinterpret_cast<uint64_t>(c->image_dev + r.off + run_lo), run_len});
+        run_len = 0;
+      }
+      if (!run_len) run_lo = lo;
+      run_len += len;
+      c->img_zero[g] = 1;
+    }
+    if (run_len) pieces.push_back(swk::ZSpan{reinterpret_cast<uint64_t>(c->image_dev + r.off + run_lo), run_len});
+  }
+  // zeros to the mapped image, in stream order: one cudaMemsetAsync per run of chunks. (A single
+  // zero_fill_kernel launch over the same pieces was measured slower here: config-B scale checkpoints
+  // 0.85-0.97 s vs 0.32-0.57 s, tools/mask_probe.py — SM-issued writes to host memory.)
+  for (const swk::ZSpan& z : pieces)
+    CUDA_TRY(c, cudaMemsetAsync(reinterpret_cast<void*>(z.dst), 0, z.bytes, s));
+  c->keep = c->next_keep;
+  c->mask_dirty = false;
+  swap_status st = build_sets(c);
+  if (st != SWAP_OK) return st;
+  *hash_zero = true;
+  if (!c->helpers.empty()) {  // restore groups changed: re-size the helpers' staging
+    std::vector<int> devs;
+    for (auto& h : c->helpers) devs.push_back(h.dev);
+    return swap_set_helpers(c, devs.data(), (int)devs.size());
+  }
+  return SWAP_OK;
+}
+
+// After a checkpoint has been enqueued: the chunks it gathered now hold data in the image.
+void note_gathered(swap_ctx* c, const DescSet& S) {
+  (void)S;
+  const auto& P = c->plan;
+  for (size_t i = 0; i < P.regions.size(); ++i) {
+    if (c->policy[i] == SWAP_POLICY_DISCARD) continue;
+    const auto& r = P.regions[i];
+    for (uint64_t j = 0; j < r.nchunks; ++j)
+      if (c->keep[r.first + j]) c->img_zero[r.first + j] = 0;
+  }
 }
 
 }  // namespace swc

@@ -145,6 +145,10 @@ swap_status swap_register_regions(swap_ctx_t* c, const swap_region_t* regions, s
   c->seg = c->cfg.seg_bytes ? c->cfg.seg_bytes : auto_seg(c, P.payload_bytes);
   if ((st = upload_tables(c)) != SWAP_OK) return st;
   c->policy.assign(P.regions.size(), SWAP_POLICY_SAVE);
+  c->keep.assign(P.n_chunks, 1);
+  c->next_keep.assign(P.n_chunks, 1);
+  c->img_zero.assign(P.n_chunks, 1);  // the image is zero-filled at allocation
+  c->mask_dirty = false;
   st = build_sets(c);
   if (st != SWAP_OK) return st;
   c->st = St::REGISTERED;
@@ -160,13 +164,16 @@ swap_status swap_checkpoint(swap_ctx_t* c, swap_stream_t stream) {
   DeviceGuard g(c->cfg.device);
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   c->cur_mech = resolve_mech(c, 0, s == nullptr);
-  // SAVE_ONCE regions are gathered by the first checkpoint only; DISCARD regions never (their image
-  // bytes stay zero and their c_g are the checksums of zero chunks, hashed once from a zero buffer).
+  CUDA_TRY(c, cudaEventRecord(c->ev[0], s));
+  bool hash_zero = false;
+  swap_status st = apply_mask(c, s, &hash_zero);  // a new chunk mask: sets rebuilt, stale image bytes zeroed
+  if (st != SWAP_OK) return st;
+  // SAVE_ONCE regions are gathered by the first checkpoint only; DISCARD regions and masked chunks never
+  // (their image bytes are zero and their c_g the checksums of zero chunks, hashed from a zero buffer
+  // whenever the set of zero chunks changes).
   DescSet& S = c->first_ckpt_done ? c->s_save : c->s_move;
   swk::Params p = base_params(c, S);
-  CUDA_TRY(c, cudaEventRecord(c->ev[0], s));
-  swap_status st;
-  if (!c->first_ckpt_done && c->s_zero.n_desc &&
+  if (hash_zero && c->s_zero.n_desc &&
       (st = launch(c, swk::HASH_STORE, hash_kind(c), base_params(c, c->s_zero), s)) != SWAP_OK)
     return st;
   if (mech(c) == SWAP_MECH_CE_PIPE) {
@@ -178,6 +185,7 @@ swap_status swap_checkpoint(swap_ctx_t* c, swap_stream_t stream) {
     if ((st = launch(c, swk::GATHER, kind_of(c), p, s)) != SWAP_OK) return st;
   }
   CUDA_TRY(c, cudaEventRecord(c->ev[1], s));
+  note_gathered(c, S);
   c->first_ckpt_done = true;
   c->pending[0] = true;
   c->st = St::CKPT_PENDING;
@@ -217,17 +225,22 @@ swap_status swap_restore(swap_ctx_t* c, swap_stream_t stream) {
   CUDA_TRY(c, cudaMemsetAsync(&c->d_status->first_bad, 0xFF, 8, s));
   CUDA_TRY(c, cudaEventRecord(c->ev[2], s));
   if (c->arena && !swarena::resident(c->arena)) {
-    // DISCARD regions (zero-filled below) and, for movers other than CE_PIPE, everything, need HBM now
-    std::vector<Span> now;
-    for (size_t i = 0; i < c->policy.size(); ++i)
-      if (mech(c) != SWAP_MECH_CE_PIPE || c->policy[i] == SWAP_POLICY_DISCARD)
+    // zero chunks (filled below) and, for movers other than CE_PIPE, everything, need HBM now
+    std::vector<Span> now = c->zero_spans;
+    if (mech(c) != SWAP_MECH_CE_PIPE)
+      for (size_t i = 0; i < c->policy.size(); ++i)
         now.push_back(Span{c->plan.regions[i].r.dev_addr, nullptr, c->plan.regions[i].r.bytes});
     if ((st = map_spans(c, now)) != SWAP_OK) return st;
   }
-  for (size_t i = 0; i < c->policy.size(); ++i)  // DISCARD regions come back as zeros
-    if (c->policy[i] == SWAP_POLICY_DISCARD && c->plan.regions[i].r.bytes)
-      CUDA_TRY(c, cudaMemsetAsync(reinterpret_cast<void*>(c->plan.regions[i].r.dev_addr), 0,
-                                  c->plan.regions[i].r.bytes, s));
+  // DISCARD regions and masked chunks come back as zeros; under CE_PIPE on the side stream, overlapped
+  // with the first group's copies (ce_pipe joins the side stream back into `s` at the end)
+  cudaStream_t zs = s;
+  if (mech(c) == SWAP_MECH_CE_PIPE && !c->zero_spans.empty()) {
+    CUDA_TRY(c, cudaEventRecord(c->ev_fork, s));
+    CUDA_TRY(c, cudaStreamWaitEvent(c->side, c->ev_fork, 0));
+    zs = c->side;
+  }
+  if ((st = zero_fill_device(c, zs)) != SWAP_OK) return st;
   if (mech(c) == SWAP_MECH_CE_PIPE) {
     if ((st = ce_pipe(c, S, 1, p, s)) != SWAP_OK) return st;
   } else if (is_ce(mech(c))) {
@@ -291,6 +304,11 @@ swap_status swap_set_region_policy(swap_ctx_t* c, uint32_t region_index, uint32_
   if (region_index >= c->policy.size()) return SWAP_EINVAL;
   if (c->policy[region_index] == policy) return SWAP_OK;
   c->policy[region_index] = policy;
+  const auto& r = c->plan.regions[region_index];
+  if (policy != SWAP_POLICY_SAVE)  // chunk masks apply to SAVE regions only
+    std::fill(c->next_keep.begin() + r.first, c->next_keep.begin() + r.first + r.nchunks, 1);
+  c->keep = c->next_keep;
+  c->mask_dirty = false;
   DeviceGuard g(c->cfg.device);
   swap_status st = build_sets(c);
   if (st != SWAP_OK || c->helpers.empty()) return st;
@@ -352,6 +370,42 @@ swap_status swap_import(swap_ctx_t* c) {
   if (st != SWAP_OK) return st;
   c->st = St::CHECKPOINTED;
   c->first_ckpt_done = true;  // the imported image already holds SAVE_ONCE bytes and DISCARD checksums
+  // the image came from elsewhere: its zero chunks are unknown, so restores move every chunk a mask
+  // does not force to zero by policy, and the next checkpoint re-applies any pending mask in full
+  std::fill(c->img_zero.begin(), c->img_zero.end(), 0);
+  if (std::find(c->keep.begin(), c->keep.end(), 0) != c->keep.end()) {
+    const std::vector<uint8_t> pending = c->next_keep;
+    std::fill(c->keep.begin(), c->keep.end(), 1);
+    DeviceGuard g(c->cfg.device);
+    if ((st = build_sets(c)) != SWAP_OK) return st;
+    c->next_keep = pending;
+    c->mask_dirty = true;
+  }
+  return SWAP_OK;
+}
+
+swap_status swap_set_chunk_mask(swap_ctx_t* c, uint32_t region_index, const uint8_t* keep, uint64_t n) {
+  if (!c) return SWAP_EINVAL;
+  if (c->st == St::CREATED || c->st == St::CKPT_PENDING) {
+    c->err = c->st == St::CREATED ? "chunk mask before swap_register_regions" : "previous checkpoint not synced";
+    return SWAP_ESTATE;
+  }
+  if (region_index >= c->policy.size()) return SWAP_EINVAL;
+  const auto& r = c->plan.regions[region_index];
+  if (n != r.nchunks) {
+    c->err = "chunk mask length differs from the region's chunk count";
+    return SWAP_EINVAL;
+  }
+  if (c->policy[region_index] != SWAP_POLICY_SAVE) {
+    c->err = "chunk masks apply to SAVE regions only";
+    return SWAP_EINVAL;
+  }
+  for (uint64_t j = 0; j < n; ++j) {
+    const uint8_t k = keep ? (keep[j] ? 1 : 0) : 1;
+    if (c->next_keep[r.first + j] != k) c->mask_dirty = true;
+    c->next_keep[r.first + j] = k;
+  }
+  if (c->next_keep == c->keep) c->mask_dirty = false;
   return SWAP_OK;
 }
 

@@ -30,7 +30,7 @@ U64_MAX = (1 << 64) - 1
 
 EXPORTS = [
     "swap_config_default", "swap_create", "swap_register_regions", "swap_checkpoint", "swap_sync",
-    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_set_region_policy", "swap_get_manifest", "swap_get_image",
+    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_set_region_policy", "swap_set_chunk_mask", "swap_get_manifest", "swap_get_image",
     "swap_get_summary", "swap_import", "swap_save", "swap_load", "swap_set_global", "swap_merge_global", "swap_plan_layout", "swap_plan_manifest", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
     "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
@@ -106,6 +106,7 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_set_mechanism": (st, [vp, u32]),
         "swap_get_mechanism": (st, [vp, P(u32)]),
         "swap_set_region_policy": (st, [vp, u32, u32]),
+        "swap_set_chunk_mask": (st, [vp, u32, vp, ctypes.c_uint64]),
         "swap_get_manifest": (st, [vp, P(vp), P(sz)]),
         "swap_get_image": (st, [vp, P(vp), P(sz)]),
         "swap_get_summary": (st, [vp, P(swap_shard_summary_t)]),
@@ -287,6 +288,8 @@ class Swapper:
             self.close()
             raise SwapError(st, msg)
         self.regions = table
+        C = chunk_bytes or (1 << 20)
+        self._n_chunks = [(nb + C - 1) // C for (_, nb, _, _) in table]
 
     # -- helpers
     def _check(self, st: int):
@@ -351,6 +354,15 @@ class Swapper:
         if isinstance(policy, str):
             policy = POLICIES[policy]
         self._check(load().swap_set_region_policy(self._ctx, region_index, policy))
+
+    def set_chunk_mask(self, region_index: int, keep=None):
+        """Touched-chunk mask of a SAVE region for the next checkpoint (None = keep every chunk):
+        chunks with keep[j] == 0 are captured as zeros and not moved (include/swap.h)."""
+        if keep is None:
+            self._check(load().swap_set_chunk_mask(self._ctx, region_index, None, self._n_chunks[region_index]))
+            return
+        k = np.ascontiguousarray(np.asarray(keep, dtype=np.uint8))
+        self._check(load().swap_set_chunk_mask(self._ctx, region_index, k.ctypes.data, k.size))
 
     def mechanism(self) -> str:
         """Name of the mover the next call uses (AUTO resolved)."""

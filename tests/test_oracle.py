@@ -285,3 +285,50 @@ def test_summary_and_global_digest(orc):
     # global digest of fabricated rank-ordered summaries
     fab = b"".join(SUM.pack(r, 4, 1, 3, 10 + r, 1000 * r, 5000, r * 7, r * 11, 0) for r in range(4))
     assert orc.global_digest(fab) == orc.crc32c_sse42(fab)
+
+
+# ------------------------------------------------------------------ touched-chunk masks (reading 25)
+def test_policy_view_chunk_masks(orc):
+    """Pins for the mask rule of oracle.policy_view against independent statements of it: an all-zero
+    mask is the DISCARD policy, an all-one mask (or none) is SAVE, and byte k of a region is zeroed
+    iff keep[k // C] == 0 (brute force over tiny regions, byte by byte)."""
+    import xxhash
+
+    C = 16
+    specs = [W.RegionSpec(f"r{i}", W.KIND_KV, n) for i, n in enumerate([0, 1, 15, 16, 17, 31, 32, 33, 48, 50])]
+    arena, base, regs = make_case(specs, 11)
+    n_ch = [-(-r[2] // C) for r in regs]
+    save = [orc.SAVE] * len(regs)
+    # all-zero mask == DISCARD, all-one / absent mask == SAVE
+    zero = {i: np.zeros(n, np.uint8) for i, n in enumerate(n_ch)}
+    ones = {i: np.ones(n, np.uint8) for i, n in enumerate(n_ch)}
+    assert np.array_equal(orc.policy_view(regs, save, arena, arena, base, C, zero),
+                          orc.policy_view(regs, [orc.DISCARD] * len(regs), arena, arena, base))
+    assert np.array_equal(orc.policy_view(regs, save, arena, arena, base, C, ones), arena)
+    assert np.array_equal(orc.policy_view(regs, save, arena, arena, base), arena)
+    # random masks, checked byte by byte
+    rng = np.random.default_rng(5)
+    for _ in range(20):
+        masks = {i: rng.integers(0, 2, n).astype(np.uint8) for i, n in enumerate(n_ch)}
+        view = orc.policy_view(regs, save, arena, arena, base, C, masks)
+        want = arena.copy()
+        for i, (_, addr, nb, _) in enumerate(regs):
+            for k in range(nb):
+                if masks[i][k // C] == 0:
+                    want[addr - base + k] = 0
+        assert np.array_equal(view, want)
+        # the captured image: masked chunks are zero bytes with the checksum of a zero chunk
+        for kind in (orc.CRC32C, orc.XXH64):
+            rc, image, moff = orc.checkpoint(regs, view, base, kind, C, 16)
+            assert rc == 0
+            h = parse_manifest(image[moff:].tobytes())
+            for i, rr in enumerate(h["regs"]):
+                first = rr[5]
+                for j, keep in enumerate(masks[i]):
+                    if keep:
+                        continue
+                    ln = h["chunks"][first + j][3]
+                    assert np.all(image[rr[4] + j * C:rr[4] + j * C + ln] == 0)
+                    z = bytes(ln)
+                    want_cs = orc.crc32c_bitwise(z) if kind == orc.CRC32C else xxhash.xxh64_intdigest(z, 0)
+                    assert h["chunks"][first + j][4] == want_cs

@@ -28,6 +28,17 @@ for kind in (1, 2):
                 poison(arena, specs, offs)
                 sw.restore(s)
                 assert sw.verify(s)["status"] == 0, (kind, mech, C)
+# touched-chunk masks (zero-filled chunks, batched group copies under CE_PIPE, image zeroing)
+for mech in ("ce_pipe", "sm"):
+    with swap.Swapper(regions, chunk_bytes=4096, mechanism=mech, pipe_mib=1) as sw, torch.cuda.stream(s):
+        big = max(range(len(specs)), key=lambda i: specs[i].nbytes)
+        n = -(-specs[big].nbytes // 4096)
+        for keep in (np.arange(n) % 3 == 0, np.arange(n) % 2 == 0):
+            sw.set_chunk_mask(big, keep.astype(np.uint8))
+            sw.checkpoint(s)
+            poison(arena, specs, offs)
+            sw.restore(s)
+            assert sw.verify(s)["status"] == 0, mech
 # XXH64 kernel variants are chosen by chunk count; a 1 KiB-chunk case exercises the lane kernel
 with swap.Swapper(regions, chunk_bytes=1024, checksum=2, mechanism="ce_region") as sw, torch.cuda.stream(s):
     sw.checkpoint(s)
