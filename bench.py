@@ -40,7 +40,7 @@ RESTORE_KERNEL = {
     "ce_pipe": "restore phase: cudaMemcpyAsync H2D groups (copy engine) + hash_kernel<HASH_CHECK> per group on a side stream",
     "ce_region": "restore phase: cudaMemcpyAsync per region + HBM hash pass",
     "ce_chunk": "restore phase: cudaMemcpyAsync per chunk + HBM hash pass",
-    "ce_batch": "restore phase: cudaMemcpyBatchAsync + HBM hash pass",
+    "ce_batch": "restore phase: coalesced cudaMemcpyAsync runs + HBM hash pass",
 }
 VERIFY_KERNEL = {"crc32c": "hash_kernel<HASH_CHECK> (CRC-32C: quad-line 256-bit loads, per-lane replicated slice-by-4 + Z^96 tables)",
                  "xxh64": "xxh_dyn_kernel<HASH_CHECK> (XXH64, one lane per chunk, chunks claimed from a ticket; "

@@ -67,7 +67,8 @@ typedef int32_t swap_status;
                                     chunk checksum fused from the same registers (one pass, bytes checked in flight) */
 #define SWAP_MECH_CE_REGION 2u   /* copy engine: cudaMemcpyAsync per region + separate HBM hash pass */
 #define SWAP_MECH_CE_CHUNK 3u    /* copy engine: cudaMemcpyAsync per chunk + HBM hash pass */
-#define SWAP_MECH_CE_BATCH 4u    /* copy engine: one cudaMemcpyBatchAsync per call + HBM hash pass */
+#define SWAP_MECH_CE_BATCH 4u    /* copy engine: the per-chunk copies coalesced into maximal runs contiguous on
+                                    both sides, one cudaMemcpyAsync per run, + HBM hash pass */
 #define SWAP_MECH_CE_PIPE 5u     /* copy engine moves the image in groups of ~pipe_mib MiB on the caller's stream
                                     while the hash kernel checks (restore) / hashes (checkpoint) each group from
                                     HBM on a second, library-owned stream; the caller's stream joins at the end */

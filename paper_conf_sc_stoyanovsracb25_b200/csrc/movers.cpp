@@ -44,11 +44,11 @@ int grid_of(swap_ctx* c) { return c->cfg.grid_ctas ? (int)c->cfg.grid_ctas : 2 *
 // The mechanism a call uses. AUTO resolves per direction from the measured crossover (DESIGN.md §6,
 // `profiles/r01_crossover.md`): the copy engines reach a higher link rate than SM-issued accesses, but
 // per-copy and per-launch costs make the single fused SM pass faster for small images.
-//   restore:    < 128 MiB SM;  < 2 GiB CE_BATCH (needs a non-default stream, else SM);  else CE_PIPE
+//   restore:    < 128 MiB SM;  < 2 GiB CE_BATCH (SM on the legacy default stream);  else CE_PIPE
 //   checkpoint: < 1 GiB SM;    else CE_PIPE
 // XXH64 is not combinable: with chunks > 4 MiB a pipeline group holds too few chunks for the side-stream
-// hash to keep up with the link (config B, 16 MiB: CE_PIPE swap-in 15 GB/s), so restores take one batch
-// copy plus one hash pass (CE_BATCH 50.7 GB/s vs SM 48.6) and checkpoints the fused SM pass (51.6 vs
+// hash to keep up with the link (config B, 16 MiB: CE_PIPE swap-in 15 GB/s), so restores take the coalesced
+// copies plus one hash pass (CE_BATCH 50.7 GB/s vs SM 48.6) and checkpoints the fused SM pass (51.6 vs
 // 49.7). Up to 4 MiB the rule is the CRC one (config B, 2 / 4 MiB: CE_PIPE 54.6 / 54.2 vs SM 50.8 / 50.6).
 uint32_t resolve_mech(const swap_ctx* c, int dir, bool default_stream) {
   if (c->cfg.mechanism != SWAP_MECH_AUTO) return c->cfg.mechanism;
@@ -83,6 +83,24 @@ swap_status launch(swap_ctx* c, int mode, int kind, const swk::Params& p, cudaSt
   return SWAP_OK;
 }
 
+// Merges consecutive spans whose device and image ranges both continue where the previous one ends.
+std::vector<Span> coalesce(const std::vector<Span>& spans) {
+  std::vector<Span> out;
+  out.reserve(spans.size());
+  for (const Span& sp : spans) {
+    if (!sp.bytes) continue;
+    if (!out.empty()) {
+      Span& b = out.back();
+      if (b.dev + b.bytes == sp.dev && b.host + b.bytes == sp.host) {
+        b.bytes += sp.bytes;
+        continue;
+      }
+    }
+    out.push_back(sp);
+  }
+  return out;
+}
+
 swap_status memcpy_dir(swap_ctx* c, const Span& sp, int dir, cudaStream_t s) {
   void* dev = reinterpret_cast<void*>(sp.dev);
   CUDA_TRY(c, dir == 0 ? cudaMemcpyAsync(sp.host, dev, sp.bytes, cudaMemcpyDeviceToHost, s)
@@ -108,24 +126,16 @@ swap_status ce_copy(swap_ctx* c, DescSet& S, int dir, cudaStream_t s) {
     }
     return SWAP_OK;
   }
-  // CE_BATCH: one cudaMemcpyBatchAsync over every chunk.
-  if (s == nullptr) {
-    c->err = "SWAP_MECH_CE_BATCH needs a non-default stream (cudaMemcpyBatchAsync restriction)";
-    return SWAP_EUNSUPPORTED;
+  // CE_BATCH: the per-chunk copies coalesced into maximal runs contiguous on both sides, one
+  // cudaMemcpyAsync per run (a masked chunk or a region boundary with padding ends a run).
+  std::vector<Span> runs;
+  runs.reserve(S.ce_bytes.size());
+  for (size_t i = 0; i < S.ce_bytes.size(); ++i)
+    runs.push_back(Span{reinterpret_cast<uint64_t>(S.ce_dev[i]), static_cast<uint8_t*>(S.ce_host[i]), S.ce_bytes[i]});
+  for (const Span& sp : coalesce(runs)) {
+    swap_status st = memcpy_dir(c, sp, dir, s);
+    if (st != SWAP_OK) return st;
   }
-  if (S.ce_bytes.empty()) return SWAP_OK;
-  cudaMemcpyAttributes attr;
-  std::memset(&attr, 0, sizeof(attr));
-  attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-  attr.srcLocHint.type = dir == 0 ? cudaMemLocationTypeDevice : cudaMemLocationTypeHost;
-  attr.srcLocHint.id = dir == 0 ? c->cfg.device : 0;
-  attr.dstLocHint.type = dir == 0 ? cudaMemLocationTypeHost : cudaMemLocationTypeDevice;
-  attr.dstLocHint.id = dir == 0 ? 0 : c->cfg.device;
-  size_t attr_idx = 0, fail_idx = 0;
-  std::vector<void*>& dst = dir == 0 ? S.ce_host : S.ce_dev;
-  std::vector<void*>& src = dir == 0 ? S.ce_dev : S.ce_host;
-  CUDA_TRY(c, cudaMemcpyBatchAsync(dst.data(), src.data(), S.ce_bytes.data(), S.ce_bytes.size(), &attr, &attr_idx, 1,
-                                   &fail_idx, s));
   return SWAP_OK;
 }
 
@@ -147,35 +157,13 @@ swap_status map_spans(swap_ctx* c, const std::vector<Span>& spans) {
   return SWAP_OK;
 }
 
-// The copies of one pipeline group. A restore group fragmented into many spans (touched-chunk masks, many
-// small regions) goes to the copy engine as one cudaMemcpyBatchAsync: per-copy submission costs dominate
-// ~1-MiB cudaMemcpyAsync calls. Checkpoints keep per-span copies (batched D2H measured slower);
-// the legacy default stream cannot take batches.
+// The copies of one pipeline group: spans contiguous on both sides (consecutive chunks of a region, a
+// region and its successor with no padding between) are coalesced, one cudaMemcpyAsync per run.
 swap_status copy_spans(swap_ctx* c, const std::vector<Span>& spans, int dir, cudaStream_t s) {
-  if (spans.size() <= 4 || s == nullptr || dir == 0) {
-    for (const Span& sp : spans) {
-      swap_status st = memcpy_dir(c, sp, dir, s);
-      if (st != SWAP_OK) return st;
-    }
-    return SWAP_OK;
+  for (const Span& sp : coalesce(spans)) {
+    swap_status st = memcpy_dir(c, sp, dir, s);
+    if (st != SWAP_OK) return st;
   }
-  std::vector<void*> dst(spans.size()), src(spans.size());
-  std::vector<size_t> bytes(spans.size());
-  for (size_t i = 0; i < spans.size(); ++i) {
-    void* dev = reinterpret_cast<void*>(spans[i].dev);
-    dst[i] = dir == 0 ? static_cast<void*>(spans[i].host) : dev;
-    src[i] = dir == 0 ? dev : static_cast<void*>(spans[i].host);
-    bytes[i] = spans[i].bytes;
-  }
-  cudaMemcpyAttributes attr;
-  std::memset(&attr, 0, sizeof(attr));
-  attr.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-  attr.srcLocHint.type = dir == 0 ? cudaMemLocationTypeDevice : cudaMemLocationTypeHost;
-  attr.srcLocHint.id = dir == 0 ? c->cfg.device : 0;
-  attr.dstLocHint.type = dir == 0 ? cudaMemLocationTypeHost : cudaMemLocationTypeDevice;
-  attr.dstLocHint.id = dir == 0 ? 0 : c->cfg.device;
-  size_t attr_idx = 0, fail_idx = 0;
-  CUDA_TRY(c, cudaMemcpyBatchAsync(dst.data(), src.data(), bytes.data(), spans.size(), &attr, &attr_idx, 1, &fail_idx, s));
   return SWAP_OK;
 }
 
