@@ -28,7 +28,7 @@ for kind in (1, 2):
                 poison(arena, specs, offs)
                 sw.restore(s)
                 assert sw.verify(s)["status"] == 0, (kind, mech, C)
-# touched-chunk masks (zero-filled chunks, batched group copies under CE_PIPE, image zeroing)
+# touched-chunk masks (zero-filled chunks, fragmented group copies under CE_PIPE, image zeroing)
 for mech in ("ce_pipe", "sm"):
     with swap.Swapper(regions, chunk_bytes=4096, mechanism=mech, pipe_mib=1) as sw, torch.cuda.stream(s):
         big = max(range(len(specs)), key=lambda i: specs[i].nbytes)
