@@ -59,10 +59,8 @@ typedef int32_t swap_status;
 
 /* Data mover for checkpoint/restore (the image bytes are identical for all of them): */
 #define SWAP_MECH_AUTO 0u        /* default, resolved per call from the measured crossover: restore
-                                    SM < 128 MiB, CE_BATCH < 2 GiB (SM on the legacy default stream), else
-                                    CE_PIPE; checkpoint SM < 1 GiB, else CE_PIPE; XXH64 with chunks > 4 MiB:
-                                    restore CE_BATCH from 128 MiB (SM below / on the default stream),
-                                    checkpoint SM */
+                                    SM < 2 GiB, else CE_PIPE; checkpoint SM < 1 GiB, else CE_PIPE; XXH64 with
+                                    chunks > 4 MiB: restore CE_BATCH from 2 GiB (SM below), checkpoint SM */
 #define SWAP_MECH_SM 1u          /* one SM kernel: 16-B vector loads/stores to mapped pinned host memory with the
                                     chunk checksum fused from the same registers (one pass, bytes checked in flight) */
 #define SWAP_MECH_CE_REGION 2u   /* copy engine: cudaMemcpyAsync per region + separate HBM hash pass */
@@ -194,7 +192,7 @@ SWAP_API swap_status swap_set_chunk_mask(swap_ctx_t* ctx, uint32_t region_index,
 
 /* Selects the data mover for later calls (SWAP_MECH_*). The image format is unchanged. */
 SWAP_API swap_status swap_set_mechanism(swap_ctx_t* ctx, uint32_t mechanism);
-/* The mechanism the next restore on a non-default stream will use (SWAP_MECH_AUTO resolved; REGISTERED+). */
+/* The mechanism the next restore will use (SWAP_MECH_AUTO resolved; REGISTERED+). */
 SWAP_API swap_status swap_get_mechanism(const swap_ctx_t* ctx, uint32_t* effective);
 
 /* Borrowed views, valid until swap_destroy. The manifest is final only after swap_sync.

@@ -113,7 +113,7 @@ swap_status cuda_fail(swap_ctx* c, cudaError_t e, const char* what);
 uint8_t* manifest_ptr(swap_ctx* c);
 swk::Params base_params(swap_ctx* c, const DescSet& S);
 int grid_of(swap_ctx* c);
-uint32_t resolve_mech(const swap_ctx* c, int dir, bool default_stream);
+uint32_t resolve_mech(const swap_ctx* c, int dir);
 uint32_t mech(const swap_ctx* c);
 int kind_of(swap_ctx* c);
 int hash_kind(swap_ctx* c);

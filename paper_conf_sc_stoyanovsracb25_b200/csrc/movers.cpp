@@ -42,23 +42,22 @@ swk::Params base_params(swap_ctx* c, const DescSet& S) {
 int grid_of(swap_ctx* c) { return c->cfg.grid_ctas ? (int)c->cfg.grid_ctas : 2 * c->sm_count; }
 
 // The mechanism a call uses. AUTO resolves per direction from the measured crossover (DESIGN.md §6,
-// `profiles/r01_crossover.md`): the copy engines reach a higher link rate than SM-issued accesses, but
-// per-copy and per-launch costs make the single fused SM pass faster for small images.
-//   restore:    < 128 MiB SM;  < 2 GiB CE_BATCH (SM on the legacy default stream);  else CE_PIPE
-//   checkpoint: < 1 GiB SM;    else CE_PIPE
+// `profiles/r01_crossover_v2.md`): the copy engines reach a higher link rate than SM-issued accesses, but
+// per-copy and per-launch costs make the single fused SM pass faster for small images (swap-in GB/s,
+// SM / CE_PIPE: 256 MiB 50.2 / 41.2, 1 GiB 50.7 / 50.6, 4 GiB 50.9 / 53.7).
+//   restore:    < 2 GiB SM;  else CE_PIPE
+//   checkpoint: < 1 GiB SM;  else CE_PIPE
 // XXH64 is not combinable: with chunks > 4 MiB a pipeline group holds too few chunks for the side-stream
-// hash to keep up with the link (config B, 16 MiB: CE_PIPE swap-in 15 GB/s), so restores take the coalesced
-// copies plus one hash pass (CE_BATCH 50.7 GB/s vs SM 48.6) and checkpoints the fused SM pass (51.6 vs
-// 49.7). Up to 4 MiB the rule is the CRC one (config B, 2 / 4 MiB: CE_PIPE 54.6 / 54.2 vs SM 50.8 / 50.6).
-uint32_t resolve_mech(const swap_ctx* c, int dir, bool default_stream) {
+// hash to keep up with the link (config B, 16 MiB: CE_PIPE swap-in 15 GB/s), so restores from 2 GiB take
+// the coalesced CE_BATCH copies plus one hash pass and checkpoints the fused SM pass (51.6 vs 49.7). Up to
+// 4 MiB the rule is the CRC one (config B, 2 / 4 MiB: CE_PIPE 54.6 / 54.2 vs SM 50.8 / 50.6).
+uint32_t resolve_mech(const swap_ctx* c, int dir) {
   if (c->cfg.mechanism != SWAP_MECH_AUTO) return c->cfg.mechanism;
   const uint64_t S = c->plan.payload_bytes;
   if (c->plan.kind == SWAP_CHECKSUM_XXH64 && c->plan.C > (4ull << 20))
-    return (dir == 1 && S >= (128ull << 20) && !default_stream) ? SWAP_MECH_CE_BATCH : SWAP_MECH_SM;
+    return (dir == 1 && S >= (2ull << 30)) ? SWAP_MECH_CE_BATCH : SWAP_MECH_SM;
   if (dir == 0) return S < (1ull << 30) ? SWAP_MECH_SM : SWAP_MECH_CE_PIPE;
-  if (S < (128ull << 20)) return SWAP_MECH_SM;
-  if (S < (2ull << 30)) return default_stream ? SWAP_MECH_SM : SWAP_MECH_CE_BATCH;
-  return SWAP_MECH_CE_PIPE;
+  return S < (2ull << 30) ? SWAP_MECH_SM : SWAP_MECH_CE_PIPE;
 }
 uint32_t mech(const swap_ctx* c) { return c->cur_mech; }
 int kind_of(swap_ctx* c) {

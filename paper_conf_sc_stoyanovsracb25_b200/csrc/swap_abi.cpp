@@ -163,7 +163,7 @@ swap_status swap_checkpoint(swap_ctx_t* c, swap_stream_t stream) {
   }
   DeviceGuard g(c->cfg.device);
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-  c->cur_mech = resolve_mech(c, 0, s == nullptr);
+  c->cur_mech = resolve_mech(c, 0);
   CUDA_TRY(c, cudaEventRecord(c->ev[0], s));
   bool hash_zero = false;
   swap_status st = apply_mask(c, s, &hash_zero);  // a new chunk mask: sets rebuilt, stale image bytes zeroed
@@ -218,7 +218,7 @@ swap_status swap_restore(swap_ctx_t* c, swap_stream_t stream) {
   if (st != SWAP_OK) return st;
   DeviceGuard g(c->cfg.device);
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-  c->cur_mech = resolve_mech(c, 1, s == nullptr);
+  c->cur_mech = resolve_mech(c, 1);
   DescSet& S = c->s_move;
   swk::Params p = base_params(c, S);
   CUDA_TRY(c, cudaMemsetAsync(&c->d_status->n_bad, 0, 8, s));
@@ -336,7 +336,7 @@ swap_status swap_set_mechanism(swap_ctx_t* c, uint32_t mechanism) {
 swap_status swap_get_mechanism(const swap_ctx_t* c, uint32_t* effective) {
   if (!c || !effective) return SWAP_EINVAL;
   if (c->st == St::CREATED) return SWAP_ESTATE;
-  *effective = resolve_mech(c, 1, false);
+  *effective = resolve_mech(c, 1);
   return SWAP_OK;
 }
 
