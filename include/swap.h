@@ -60,7 +60,7 @@ typedef int32_t swap_status;
 /* Data mover for checkpoint/restore (the image bytes are identical for all of them): */
 #define SWAP_MECH_AUTO 0u        /* default, resolved per call from the measured crossover: restore
                                     SM < 2 GiB, else CE_PIPE; checkpoint SM < 1 GiB, else CE_PIPE; XXH64 with
-                                    chunks > 4 MiB: restore CE_BATCH from 2 GiB (SM below), checkpoint SM */
+                                    chunks > 4 MiB: restore CE_BATCH from 2 GiB (SM below) */
 #define SWAP_MECH_SM 1u          /* one SM kernel: 16-B vector loads/stores to mapped pinned host memory with the
                                     chunk checksum fused from the same registers (one pass, bytes checked in flight) */
 #define SWAP_MECH_CE_REGION 2u   /* copy engine: cudaMemcpyAsync per region + separate HBM hash pass */

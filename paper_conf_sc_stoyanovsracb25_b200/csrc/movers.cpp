@@ -49,13 +49,15 @@ int grid_of(swap_ctx* c) { return c->cfg.grid_ctas ? (int)c->cfg.grid_ctas : 2 *
 //   checkpoint: < 1 GiB SM;  else CE_PIPE
 // XXH64 is not combinable: with chunks > 4 MiB a pipeline group holds too few chunks for the side-stream
 // hash to keep up with the link (config B, 16 MiB: CE_PIPE swap-in 15 GB/s), so restores from 2 GiB take
-// the coalesced CE_BATCH copies plus one hash pass and checkpoints the fused SM pass (51.6 vs 49.7). Up to
-// 4 MiB the rule is the CRC one (config B, 2 / 4 MiB: CE_PIPE 54.6 / 54.2 vs SM 50.8 / 50.6).
+// the coalesced CE_BATCH copies plus one hash pass (50.2 vs SM 48.7). Checkpoints follow the CRC rule: the
+// one whole-image hash pass overlaps every D2H copy (config B, 16 MiB: CE_PIPE 57.2 vs SM 51.5 GB/s,
+// `profiles/r01_bench_B_xxh64_16MiB_v2.json`). Up to 4 MiB the restore rule is the CRC one too (config B,
+// 2 / 4 MiB: CE_PIPE 54.6 / 54.2 vs SM 50.8 / 50.6).
 uint32_t resolve_mech(const swap_ctx* c, int dir) {
   if (c->cfg.mechanism != SWAP_MECH_AUTO) return c->cfg.mechanism;
   const uint64_t S = c->plan.payload_bytes;
-  if (c->plan.kind == SWAP_CHECKSUM_XXH64 && c->plan.C > (4ull << 20))
-    return (dir == 1 && S >= (2ull << 30)) ? SWAP_MECH_CE_BATCH : SWAP_MECH_SM;
+  if (dir == 1 && c->plan.kind == SWAP_CHECKSUM_XXH64 && c->plan.C > (4ull << 20))
+    return S >= (2ull << 30) ? SWAP_MECH_CE_BATCH : SWAP_MECH_SM;
   if (dir == 0) return S < (1ull << 30) ? SWAP_MECH_SM : SWAP_MECH_CE_PIPE;
   return S < (2ull << 30) ? SWAP_MECH_SM : SWAP_MECH_CE_PIPE;
 }
