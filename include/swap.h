@@ -194,6 +194,9 @@ SWAP_API swap_status swap_set_chunk_mask(swap_ctx_t* ctx, uint32_t region_index,
 SWAP_API swap_status swap_set_mechanism(swap_ctx_t* ctx, uint32_t mechanism);
 /* The mechanism the next restore will use (SWAP_MECH_AUTO resolved; REGISTERED+). */
 SWAP_API swap_status swap_get_mechanism(const swap_ctx_t* ctx, uint32_t* effective);
+/* The mechanism the next call of one direction will use: direction 0 = checkpoint, 1 = restore
+ * (AUTO resolves per direction, so the two can differ; REGISTERED+; EINVAL for another direction). */
+SWAP_API swap_status swap_get_mechanism_dir(const swap_ctx_t* ctx, int direction, uint32_t* effective);
 
 /* Borrowed views, valid until swap_destroy. The manifest is final only after swap_sync.
  * The image is writable: a caller may load a stored image into it and call swap_import. */

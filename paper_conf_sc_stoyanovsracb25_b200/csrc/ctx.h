@@ -95,6 +95,7 @@ struct swap_ctx {
     int dev = -1;
     cudaStream_t s = nullptr;
     uint8_t* staging = nullptr;
+    uint64_t staging_bytes = 0;  // the largest restore group's image range when the helpers were set
     cudaEvent_t ev = nullptr, done = nullptr;
   };
   std::vector<Helper> helpers;

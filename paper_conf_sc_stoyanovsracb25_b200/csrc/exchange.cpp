@@ -215,7 +215,8 @@ swap_status swap_set_helpers(swap_ctx_t* c, const int* devices, int n) {
     CUDA_TRY(c, cudaStreamCreateWithFlags(&h.s, cudaStreamNonBlocking));
     CUDA_TRY(c, cudaEventCreateWithFlags(&h.ev, cudaEventDisableTiming));
     CUDA_TRY(c, cudaEventCreateWithFlags(&h.done, cudaEventDisableTiming));
-    CUDA_TRY(c, cudaMalloc(&h.staging, std::max<uint64_t>(stage, 16)));
+    h.staging_bytes = std::max<uint64_t>(stage, 16);
+    CUDA_TRY(c, cudaMalloc(&h.staging, h.staging_bytes));
     c->helpers.push_back(h);
   }
   CUDA_TRY(c, cudaSetDevice(c->cfg.device));

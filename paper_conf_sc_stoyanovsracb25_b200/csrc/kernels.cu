@@ -178,6 +178,33 @@ __device__ __forceinline__ uint32_t crc_piece(uint32_t T, const int4& v, const u
 __device__ __forceinline__ uint64_t rotl64(uint64_t x, int r) { return (x << r) | (x >> (64 - r)); }
 __device__ __forceinline__ uint64_t xround(uint64_t acc, uint64_t in) { return rotl64(acc + in * P2, 31) * P1; }
 __device__ __forceinline__ uint64_t xmerge(uint64_t h, uint64_t v) { return (h ^ xround(0, v)) * P1 + P4; }
+
+// XXH64 accumulator chains in "t-form". The spec's round is v <- rotl(v + w*P2, 31) * P1; written
+// directly, ptxas puts the w*P2 multiply and a 64-bit add on the dependent chain (~11 serial SASS ops,
+// ~53 cycles per round measured in the quad kernel: ncu "wait" stalls). Carrying t = v_prev + w*P2
+// instead, one stripe is t <- rotl(t, 31) * P1 + w*P2: the rotate (two SHF.W) feeds one IMAD.WIDE.U32
+// whose 64-bit addend is w*P2 (computed off the chain) with the cross terms folded into the high word
+// -- four dependent ops per round. t0 = rotr(v0 * P1^-1, 31) (P1 is odd, so invertible mod 2^64) makes
+// every stripe, the first included, the same step, and v = rotl(t, 31) * P1 at the end (= v0 when the
+// chunk has no whole stripe). Bit-exact by construction; the finish uses v as the spec states.
+constexpr uint64_t inv64(uint64_t a) {  // a^-1 mod 2^64 for odd a (Newton: 3 -> 6 -> ... -> 96 bits)
+  uint64_t x = a;
+  for (int i = 0; i < 6; ++i) x *= 2 - a * x;
+  return x;
+}
+constexpr uint64_t rotr64c(uint64_t x, int r) { return (x >> r) | (x << (64 - r)); }
+constexpr uint64_t xt_of(uint64_t v) { return rotr64c(v * inv64(P1), 31); }
+constexpr uint64_t XT0 = xt_of(P1 + P2), XT1 = xt_of(P2), XT2 = xt_of(0), XT3 = xt_of(0ull - P1);
+static_assert(inv64(P1) * P1 == 1, "P1 inverse");
+__device__ __forceinline__ uint64_t xt_init(int j) { return j == 0 ? XT0 : j == 1 ? XT1 : j == 2 ? XT2 : XT3; }
+__device__ __forceinline__ uint64_t xt_step(uint64_t t, uint64_t w) {
+  const uint64_t x = w * P2;
+  const uint32_t tl = (uint32_t)t, th = (uint32_t)(t >> 32);
+  const uint32_t rl = __funnelshift_l(th, tl, 31), rh = __funnelshift_l(tl, th, 31);  // rotl(t, 31)
+  const uint32_t ch = rh * (uint32_t)P1 + (uint32_t)(x >> 32) + rl * (uint32_t)(P1 >> 32);
+  return (uint64_t)rl * (uint32_t)P1 + (((uint64_t)ch << 32) | (uint32_t)x);
+}
+__device__ __forceinline__ uint64_t xt_final(uint64_t t) { return rotl64(t, 31) * P1; }
 __device__ __forceinline__ uint64_t ld_u64_smem(const uint8_t* p) {  // 8-aligned not guaranteed
   uint64_t v = 0;
 #pragma unroll
@@ -835,15 +862,16 @@ __device__ __forceinline__ uint64_t w64(const uint32_t (&w)[8], int i) {
   return (uint64_t)w[2 * i] | ((uint64_t)w[2 * i + 1] << 32);
 }
 
+template <bool TF>
 __device__ __forceinline__ void xxh_stripe(uint64_t (&v)[4], const uint32_t (&w)[8]) {
 #pragma unroll
-  for (int i = 0; i < 4; ++i) v[i] = xround(v[i], w64(w, i));
+  for (int i = 0; i < 4; ++i) v[i] = TF ? xt_step(v[i], w64(w, i)) : xround(v[i], w64(w, i));
 }
 
 // Stripes [0, end) of one chunk into the four accumulators. A U-deep software pipeline (each 256-bit
 // load consumed U stripes after issue) keeps U stripes per lane in flight; without it ptxas sinks each
 // load next to its use.
-template <bool AL32, int U>
+template <bool AL32, int U, bool TF>
 __device__ __forceinline__ void xxh_stripes(const uint8_t* src, uint64_t end, uint64_t (&v)[4]) {
   const uint64_t n = end / 32;
   uint64_t t = 0;
@@ -855,18 +883,18 @@ __device__ __forceinline__ void xxh_stripes(const uint8_t* src, uint64_t end, ui
       const uint8_t* q = src + (t + U) * 32;
 #pragma unroll
       for (int u = 0; u < U; ++u) {
-        xxh_stripe(v, buf[u]);
+        xxh_stripe<TF>(v, buf[u]);
         ld32na<AL32>(q + u * 32, buf[u]);
       }
     }
 #pragma unroll
-    for (int u = 0; u < U; ++u) xxh_stripe(v, buf[u]);
+    for (int u = 0; u < U; ++u) xxh_stripe<TF>(v, buf[u]);
     t += U;
   }
   for (; t < n; ++t) {
     uint32_t w[8];
     ld32na<AL32>(src + t * 32, w);
-    xxh_stripe(v, w);
+    xxh_stripe<TF>(v, w);
   }
 }
 
@@ -912,12 +940,20 @@ __device__ __forceinline__ void xxh_finish(const Params& p, const SegDesc& d, co
 }
 
 // One whole chunk (descriptor d) by one lane.
-template <int MODE, int U>
+template <int MODE, int U, bool TF = true>
 __device__ __forceinline__ void xxh_chunk(const Params& p, const SegDesc& d) {
   const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
   uint64_t v[4] = {P1 + P2, P2, 0, 0ull - P1};
+  if (TF) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) v[i] = xt_init(i);
+  }
   const uint64_t stripes_end = (uint64_t)d.bytes / 32 * 32;
-  if ((d.dev & 31) == 0) xxh_stripes<true, U>(src, stripes_end, v); else xxh_stripes<false, U>(src, stripes_end, v);
+  if ((d.dev & 31) == 0) xxh_stripes<true, U, TF>(src, stripes_end, v); else xxh_stripes<false, U, TF>(src, stripes_end, v);
+  if (TF) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) v[i] = xt_final(v[i]);
+  }
   xxh_finish<MODE>(p, d, v);
 }
 
@@ -967,14 +1003,14 @@ __global__ void __launch_bounds__(MAXT) xxh_lane_kernel(const Params p) {
 // behind it). The static launches hand every lane its chunks up front, and under load some SMs are
 // served more slowly than others: ncu on config B showed SMs idle for 8 % (4 deep) / 26 % (8 deep) of
 // the kernel waiting for the slowest one. Here fast lanes simply hash more chunks.
-template <int MODE, int U, int MAXT>
+template <int MODE, int U, int MAXT, bool TF = true>
 __global__ void __launch_bounds__(MAXT) xxh_dyn_kernel(const Params p) {
   const uint32_t lanes = gridDim.x * blockDim.x;
   uint32_t idx = blockIdx.x * blockDim.x + threadIdx.x;
   while (idx < p.n_desc) {
     const SegDesc d = p.desc[idx];
     const uint32_t next = lanes + atomicAdd(p.ticket, 1u);
-    xxh_chunk<MODE, U>(p, d);
+    xxh_chunk<MODE, U, TF>(p, d);
     idx = next;
   }
 }
@@ -1081,6 +1117,123 @@ __global__ void __launch_bounds__(W * 32) xxh_coop_kernel(const Params p) {
   }
 }
 
+// Quad-per-chunk XXH64 for few, large chunks (C >= 2 MiB). A chunk's rate is bounded by its four
+// accumulator chains (v_j <- rotl(v_j + w*P2, 31)*P1, one round per 32-B stripe), so every chunk of the
+// image must be hashed at once and each must have enough bytes in flight to cover memory latency:
+//  * a warp owns 8 chunks, lane quad q <-> chunk q, lane j of the quad <-> accumulator v_(j+1): all 32
+//    lanes run rounds (the ring kernel used lanes 0..3 of a warp per chunk);
+//  * each chunk streams through its own S-stage ring of STG-byte stages in shared memory with TMA bulk
+//    copies (cp.async.bulk + one mbarrier per warp stage carrying the 8 chunks' bytes), (S-1) x STG
+//    bytes in flight per chunk without occupying registers;
+//  * ring q starts 32 x q bytes past a multiple of 128, so the warp's 8-B reads of one stripe (8 quads x
+//    32 B) hit every bank exactly twice (two wavefronts, the minimum for 256 B);
+//  * work: batches of 8 consecutive chunks; a warp's first batch is interleaved over CTAs (batch
+//    warp * grid + cta) so a short image spreads over all SMs, later batches come from the ticket.
+// The merge, the < 32-B tail (read from HBM) and the avalanche run on the quad's lane 0 (xxh_finish).
+template <int W, int S, int STG>
+struct XQ {
+  static constexpr uint32_t RING = S * STG + 32;                    // one chunk's ring + bank skew
+  static constexpr uint32_t WARP_BYTES = 8 * RING;
+  static constexpr size_t SMEM = (size_t)W * WARP_BYTES + (size_t)W * S * 8 + 128;
+};
+template <int MODE, int W, int S, int STG, bool TF>
+__global__ void __launch_bounds__(W * 32) xxh_quad_kernel(const Params p) {
+  using G = XQ<W, S, STG>;
+  extern __shared__ __align__(128) uint8_t smem[];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, q = lane >> 2, j = lane & 3;
+  uint8_t* wbase = smem + (size_t)warp * G::WARP_BYTES;
+  uint8_t* ring = wbase + q * G::RING;  // this quad's chunk ring (128-B aligned + 32 q)
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + (size_t)W * G::WARP_BYTES) + warp * S;
+  if (lane == 0) {
+    for (int s = 0; s < S; ++s) mbar_init(bars + s, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncwarp();
+  const uint32_t n_batches = (p.n_desc + 7) / 8;
+  const uint32_t warps = gridDim.x * W;
+  uint32_t batch = warp * gridDim.x + blockIdx.x;
+  uint32_t seq = 0;  // stages issued by this warp so far: buffer seq % S, parity (seq / S) & 1
+  while (batch < n_batches) {
+    uint32_t next = 0;
+    if (lane == 0) next = warps + atomicAdd(p.ticket, 1u);
+    next = __shfl_sync(0xffffffffu, next, 0);
+    const uint32_t idx = batch * 8 + q;
+    const bool mine = idx < p.n_desc;
+    SegDesc d{};
+    if (mine) d = p.desc[idx];
+    const uint64_t len = mine ? d.bytes : 0, len16 = len & ~15ull;
+    const uint32_t nst = (uint32_t)((len16 + STG - 1) / STG);
+    uint32_t nst_max = nst;
+#pragma unroll
+    for (int o = 16; o >= 4; o >>= 1) nst_max = max(nst_max, __shfl_xor_sync(0xffffffffu, nst_max, o));
+    // stage k of all 8 chunks: lane 0 arms the barrier with their byte total, quad leaders copy
+    auto issue = [&](uint32_t k) {
+      const uint32_t b = (seq + k) % S;
+      const uint64_t o = (uint64_t)k * STG;
+      const uint32_t sz = o < len16 ? (uint32_t)(len16 - o < STG ? len16 - o : STG) : 0u;
+      uint32_t tot = j == 0 ? sz : 0u;
+#pragma unroll
+      for (int x = 16; x > 0; x >>= 1) tot += __shfl_xor_sync(0xffffffffu, tot, x);
+      if (lane == 0) {
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        mbar_expect_tx(bars + b, tot);
+      }
+      __syncwarp();
+      if (j == 0 && sz) bulk_g2s(ring + (size_t)b * STG, reinterpret_cast<const uint8_t*>(d.dev) + o, sz, bars + b);
+    };
+    for (uint32_t k = 0; k < nst_max && k < (uint32_t)S; ++k) issue(k);
+    uint64_t v = TF ? xt_init(j) : j == 0 ? P1 + P2 : j == 1 ? P2 : j == 2 ? 0ull : 0ull - P1;
+    const uint64_t stripes = len / 32;
+    for (uint32_t k = 0; k < nst_max; ++k) {
+      const uint32_t b = (seq + k) % S;
+      mbar_wait(bars + b, ((seq + k) / S) & 1u);
+      const uint64_t s0 = (uint64_t)k * (STG / 32);
+      if (s0 < stripes) {
+        const uint8_t* qb = ring + (size_t)b * STG + 8 * j;
+        const uint32_t ns = (uint32_t)(stripes - s0 < (uint64_t)(STG / 32) ? stripes - s0 : (uint64_t)(STG / 32));
+        if (ns == STG / 32) {
+#pragma unroll 16
+          for (uint32_t s = 0; s < (uint32_t)(STG / 32); ++s) v = TF ? xt_step(v, lds_u64(qb + 32 * s)) : xround(v, lds_u64(qb + 32 * s));
+        } else {
+          for (uint32_t s = 0; s < ns; ++s) v = TF ? xt_step(v, lds_u64(qb + 32 * s)) : xround(v, lds_u64(qb + 32 * s));
+        }
+      }
+      __syncwarp();  // every lane is done with buffer b before it is refilled
+      if (k + S < nst_max) issue(k + S);
+    }
+    if (TF) v = xt_final(v);
+    uint64_t vv[4];
+#pragma unroll
+    for (int x = 0; x < 4; ++x) vv[x] = __shfl_sync(0xffffffffu, v, (lane & ~3) + x);
+    if (mine && j == 0) xxh_finish<MODE>(p, d, vv);
+    seq += nst_max;
+    batch = next;
+    __syncwarp();
+  }
+}
+
+template <int MODE, int W, int S, int STG, bool TF = true>
+static cudaError_t launch_xxh_quad(const Params& p, int sm_count, cudaStream_t s) {
+  using G = XQ<W, S, STG>;
+  if (!p.ticket) return cudaErrorInvalidValue;
+  static unsigned long long attr_set = 0;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (!((attr_set >> (dev & 63)) & 1ull)) {
+    e = cudaFuncSetAttribute(xxh_quad_kernel<MODE, W, S, STG, TF>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)G::SMEM);
+    if (e != cudaSuccess) return e;
+    attr_set |= 1ull << (dev & 63);
+  }
+  const uint32_t n_batches = (p.n_desc + 7) / 8;
+  // one CTA per SM while every warp slot has a batch; fewer CTAs only for tiny images
+  const int grid = (int)std::max<uint32_t>(1, std::min<uint32_t>((uint32_t)sm_count, n_batches));
+  e = cudaMemsetAsync(p.ticket, 0, sizeof(unsigned int), s);
+  if (e != cudaSuccess) return e;
+  xxh_quad_kernel<MODE, W, S, STG, TF><<<grid, W * 32, G::SMEM, s>>>(p);
+  return cudaGetLastError();
+}
+
 template <int MODE, int U>
 static cudaError_t launch_xxh_lane(const Params& p, int sm_count, cudaStream_t s) {
   const uint32_t blocks = (p.n_desc + XK_THREADS - 1) / XK_THREADS;
@@ -1119,7 +1272,7 @@ static cudaError_t launch_xxh_lane_bal(const Params& p, int sm_count, cudaStream
 
 // Dynamic lane launch: one CTA of T lanes per SM (SWAP_XXH_DYN_T overrides T, for measurements), the
 // ticket zeroed on the launching stream first.
-template <int MODE, int U>
+template <int MODE, int U, bool TF = true>
 static cudaError_t launch_xxh_dyn(const Params& p, int sm_count, cudaStream_t s) {
   constexpr int MAXT = U >= 8 ? 640 : 1024;
   if (!p.ticket) return launch_xxh_lane_bal<MODE, U>(p, sm_count, s);
@@ -1130,7 +1283,7 @@ static cudaError_t launch_xxh_dyn(const Params& p, int sm_count, cudaStream_t s)
   const int grid = (int)std::min<uint32_t>((uint32_t)sm_count, (p.n_desc + T - 1) / T);
   cudaError_t e = cudaMemsetAsync(p.ticket, 0, sizeof(unsigned int), s);
   if (e != cudaSuccess) return e;
-  xxh_dyn_kernel<MODE, U, MAXT><<<grid, T, 0, s>>>(p);
+  xxh_dyn_kernel<MODE, U, MAXT, TF><<<grid, T, 0, s>>>(p);
   return cudaGetLastError();
 }
 
@@ -1184,8 +1337,9 @@ static cudaError_t launch_t(const Params& p, int grid, cudaStream_t s) {
 static int xxh_variant() {
   const char* e = getenv("SWAP_XXH_KERNEL");
   if (!e) return 0;
-  const char* names[] = {"lane8", "bal", "bal8", "dyn", "coop", "coop16", "coop8", "ring"};
-  for (int i = 0; i < 8; ++i)
+  const char* names[] = {"lane8", "bal", "bal8", "dyn", "coop", "coop16", "coop8", "ring", "quad", "quad1k", "quad4k",
+                         "quad_x", "dyn_x"};
+  for (int i = 0; i < 13; ++i)
     if (!strcmp(e, names[i])) return i + 1;
   return 0;
 }
@@ -1193,7 +1347,7 @@ static int xxh_variant() {
 cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_t s) {
   if (p.n_desc == 0) return cudaSuccess;
   const bool st = mode == HASH_STORE;
-  switch (xxh_variant()) {  // forced: lane8 | bal | bal8 | dyn | coop | coop16 | coop8 | ring
+  switch (xxh_variant()) {  // forced: lane8 | bal | bal8 | dyn | coop | coop16 | coop8 | ring | quad | quad1k | quad4k
     case 1: return st ? launch_xxh_lane<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8>(p, sm_count, s);
     case 2: return st ? launch_xxh_lane_bal<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 4>(p, sm_count, s);
     case 3: return st ? launch_xxh_lane_bal<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8>(p, sm_count, s);
@@ -1202,6 +1356,12 @@ cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_
     case 6: return st ? launch_xxh_coop<HASH_STORE, 6, 2, 16>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 16>(p, sm_count, s);
     case 7: return st ? launch_xxh_coop<HASH_STORE, 6, 2, 8>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 8>(p, sm_count, s);
     case 8: return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
+    case 9: return st ? launch_xxh_quad<HASH_STORE, 4, 3, 2048>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 4, 3, 2048>(p, sm_count, s);
+    case 10: return st ? launch_xxh_quad<HASH_STORE, 6, 4, 1024>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 6, 4, 1024>(p, sm_count, s);
+    case 11: return st ? launch_xxh_quad<HASH_STORE, 2, 3, 4096>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 2, 3, 4096>(p, sm_count, s);
+    // the spec-form round (xround) instead of the t-form, for A/B measurements
+    case 12: return st ? launch_xxh_quad<HASH_STORE, 4, 3, 2048, false>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 4, 3, 2048, false>(p, sm_count, s);
+    case 13: return st ? launch_xxh_dyn<HASH_STORE, 4, false>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 4, false>(p, sm_count, s);
     default: break;
   }
   // Measured on config B and an 8-GiB cut of it (profiles/r01_xxh_variants.md): up to

@@ -189,6 +189,10 @@ swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, c
       auto& h = c->helpers[k - 1];
       uint8_t* lo = G.spans.front().host;
       uint8_t* hi = G.spans.back().host + G.spans.back().bytes;
+      if ((uint64_t)(hi - lo) > h.staging_bytes) {  // groups rebuilt without re-sizing the helpers
+        c->err = "restore group larger than the helper staging buffer (call swap_set_helpers again)";
+        return SWAP_EINTERNAL;
+      }
       CUDA_TRY(c, cudaSetDevice(h.dev));
       CUDA_TRY(c, cudaMemcpyAsync(h.staging, lo, (size_t)(hi - lo), cudaMemcpyHostToDevice, h.s));
       for (const Span& sp : G.spans)

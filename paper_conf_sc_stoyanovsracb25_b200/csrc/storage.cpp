@@ -18,6 +18,7 @@
 #include <vector>
 
 #include "../../include/swap.h"
+#include "ctx.h"
 
 namespace {
 
@@ -88,6 +89,17 @@ swap_status swap_save(const swap_ctx_t* ctx, const char* path) {
 
 swap_status swap_load(swap_ctx_t* ctx, const char* path) {
   if (!ctx || !path) return SWAP_EINVAL;
+  // the image is overwritten below: refuse before touching it while a checkpoint may still be writing
+  // it, and let any restore still reading it finish first
+  if (ctx->st == swc::St::CREATED || ctx->st == swc::St::CKPT_PENDING) {
+    ctx->err = ctx->st == swc::St::CREATED ? "swap_load before swap_register_regions" : "previous checkpoint not synced";
+    return SWAP_ESTATE;
+  }
+  {
+    swc::DeviceGuard g(ctx->cfg.device);
+    const cudaError_t e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) return swc::cuda_fail(ctx, e, "swap_load sync");
+  }
   void* img = nullptr;
   size_t n = 0;
   swap_status st = swap_get_image(ctx, &img, &n);

@@ -340,6 +340,13 @@ swap_status swap_get_mechanism(const swap_ctx_t* c, uint32_t* effective) {
   return SWAP_OK;
 }
 
+swap_status swap_get_mechanism_dir(const swap_ctx_t* c, int direction, uint32_t* effective) {
+  if (!c || !effective || (direction != 0 && direction != 1)) return SWAP_EINVAL;
+  if (c->st == St::CREATED) return SWAP_ESTATE;
+  *effective = resolve_mech(c, direction);
+  return SWAP_OK;
+}
+
 swap_status swap_get_manifest(const swap_ctx_t* c, const void** bytes, size_t* n) {
   if (!c || !bytes || !n) return SWAP_EINVAL;
   if (!c->image) return SWAP_ESTATE;
@@ -380,6 +387,11 @@ swap_status swap_import(swap_ctx_t* c) {
     if ((st = build_sets(c)) != SWAP_OK) return st;
     c->next_keep = pending;
     c->mask_dirty = true;
+    if (!c->helpers.empty()) {  // the restore groups changed: re-size the helpers' staging
+      std::vector<int> devs;
+      for (auto& h : c->helpers) devs.push_back(h.dev);
+      return swap_set_helpers(c, devs.data(), (int)devs.size());
+    }
   }
   return SWAP_OK;
 }

@@ -30,7 +30,7 @@ U64_MAX = (1 << 64) - 1
 
 EXPORTS = [
     "swap_config_default", "swap_create", "swap_register_regions", "swap_checkpoint", "swap_sync",
-    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_set_region_policy", "swap_set_chunk_mask", "swap_get_manifest", "swap_get_image",
+    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_get_mechanism_dir", "swap_set_region_policy", "swap_set_chunk_mask", "swap_get_manifest", "swap_get_image",
     "swap_get_summary", "swap_import", "swap_save", "swap_load", "swap_set_global", "swap_merge_global", "swap_plan_layout", "swap_plan_manifest", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
     "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
@@ -105,6 +105,7 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_verify": (st, [vp, vp, ctypes.c_int, P(swap_verify_result_t)]),
         "swap_set_mechanism": (st, [vp, u32]),
         "swap_get_mechanism": (st, [vp, P(u32)]),
+        "swap_get_mechanism_dir": (st, [vp, ctypes.c_int, P(u32)]),
         "swap_set_region_policy": (st, [vp, u32, u32]),
         "swap_set_chunk_mask": (st, [vp, u32, vp, ctypes.c_uint64]),
         "swap_get_manifest": (st, [vp, P(vp), P(sz)]),
@@ -364,10 +365,12 @@ class Swapper:
         k = np.ascontiguousarray(np.asarray(keep, dtype=np.uint8))
         self._check(load().swap_set_chunk_mask(self._ctx, region_index, k.ctypes.data, k.size))
 
-    def mechanism(self) -> str:
-        """Name of the mover the next call uses (AUTO resolved)."""
+    def mechanism(self, direction: str = "restore") -> str:
+        """Name of the mover the next call of `direction` ("restore" or "checkpoint") uses, AUTO
+        resolved per direction (swap_get_mechanism_dir)."""
         m = ctypes.c_uint32()
-        self._check(load().swap_get_mechanism(self._ctx, ctypes.byref(m)))
+        d = {"checkpoint": 0, "restore": 1}[direction]
+        self._check(load().swap_get_mechanism_dir(self._ctx, d, ctypes.byref(m)))
         return {v: k for k, v in MECHANISMS.items()}[m.value]
 
     def save(self, path: str):

@@ -131,6 +131,15 @@ def test_layout_brute_force(orc, C, A):
             assert man["size"] == image.size - moff
             assert (man["C"], man["A"], man["n"], man["m"], man["payload"]) == (C, A, n, len(want_chunks), payload)
             assert [r[4] for r in man["regs"]] == want_offs
+            # header constants and the region records' remaining fields, from the naive chunk list:
+            # first_i = how many chunks the regions before i produced, n_i = how many region i produced
+            assert (man["magic"], man["ver"], man["kind"], man["rank"], man["world"]) == (b"SWAPMAN1", 1, kind, 0, 1)
+            firsts = [sum(1 for c in want_chunks if c[0] < i) for i in range(n)]
+            counts = [sum(1 for c in want_chunks if c[0] == i) for i in range(n)]
+            assert [r[:4] for r in man["regs"]] == [(rid, k, a, s) for (rid, a, s, k) in regs]
+            assert [r[5] for r in man["regs"]] == firsts
+            assert [r[6] for r in man["regs"]] == counts
+            assert all(c[1] == 0 for c in man["chunks"])  # chunk-record pad
             assert [list(c[:1]) + list(c[2:4]) for c in man["chunks"]] == want_chunks
             for (ri, _, lo, ln, c) in man["chunks"]:
                 piece = contents[ri][lo:lo + ln]
@@ -210,10 +219,17 @@ def test_roundtrip_config_a(orc, seed, C, kind):
     man = image[moff:]
     assert orc.manifest_ok(man)
     h = parse_manifest(man.tobytes())
+    assert (h["magic"], h["ver"], h["kind"], h["C"], h["A"], h["n"]) == (b"SWAPMAN1", 1, kind, C, 4096, len(regs))
+    first = 0
     for (rid, addr, nb, k), rr in zip(regs, h["regs"]):
         assert rr[:4] == (rid, k, addr, nb)
+        n_i = len(range(0, nb, C))  # chunk starts 0, C, 2C, ... below nb
+        assert (rr[5], rr[6]) == (first, n_i)
+        assert [c[0] for c in h["chunks"][first:first + n_i]] == [regs.index((rid, addr, nb, k))] * n_i
+        first += n_i
         o = rr[4]
         assert np.array_equal(image[o:o + nb], arena[addr - base:addr - base + nb])
+    assert first == h["m"]
     # poison every region, restore, compare all bytes (guards included)
     for (_, addr, nb, _) in regs:
         arena[addr - base:addr - base + nb] = W.POISON_BYTE
