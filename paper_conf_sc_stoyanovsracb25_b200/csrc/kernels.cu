@@ -1130,26 +1130,31 @@ __global__ void __launch_bounds__(W * 32) xxh_coop_kernel(const Params p) {
 //  * work: batches of 8 consecutive chunks; a warp's first batch is interleaved over CTAs (batch
 //    warp * grid + cta) so a short image spreads over all SMs, later batches come from the ticket.
 // The merge, the < 32-B tail (read from HBM) and the avalanche run on the quad's lane 0 (xxh_finish).
-template <int W, int S, int STG>
+template <int W, int S, int STG, int LPC>
 struct XQ {
+  static constexpr int CPW = 32 / LPC;                              // chunks per warp
+  static constexpr int NC = 4 / LPC;                                // accumulator chains per lane
   static constexpr uint32_t RING = S * STG + 32;                    // one chunk's ring + bank skew
-  static constexpr uint32_t WARP_BYTES = 8 * RING;
+  static constexpr uint32_t WARP_BYTES = CPW * RING;                // CPW % 4 == 0: 128-B aligned
   static constexpr size_t SMEM = (size_t)W * WARP_BYTES + (size_t)W * S * 8 + 128;
 };
-template <int MODE, int W, int S, int STG, bool TF>
+// LPC = lanes per chunk: 4 (quad, one accumulator per lane) or 2 (pair: lane j of the pair holds
+// v_(j+1) and v_(j+3), two independent chains interleaved in one instruction stream).
+template <int MODE, int W, int S, int STG, bool TF, int LPC>
 __global__ void __launch_bounds__(W * 32) xxh_quad_kernel(const Params p) {
-  using G = XQ<W, S, STG>;
+  using G = XQ<W, S, STG, LPC>;
+  constexpr int CPW = G::CPW, NC = G::NC;
   extern __shared__ __align__(128) uint8_t smem[];
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, q = lane >> 2, j = lane & 3;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, q = lane / LPC, j = lane % LPC;
   uint8_t* wbase = smem + (size_t)warp * G::WARP_BYTES;
-  uint8_t* ring = wbase + q * G::RING;  // this quad's chunk ring (128-B aligned + 32 q)
+  uint8_t* ring = wbase + q * G::RING;  // this group's chunk ring (128-B aligned + 32 q)
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + (size_t)W * G::WARP_BYTES) + warp * S;
   if (lane == 0) {
     for (int s = 0; s < S; ++s) mbar_init(bars + s, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncwarp();
-  const uint32_t n_batches = (p.n_desc + 7) / 8;
+  const uint32_t n_batches = (p.n_desc + CPW - 1) / CPW;
   const uint32_t warps = gridDim.x * W;
   uint32_t batch = warp * gridDim.x + blockIdx.x;
   uint32_t seq = 0;  // stages issued by this warp so far: buffer seq % S, parity (seq / S) & 1
@@ -1157,23 +1162,18 @@ __global__ void __launch_bounds__(W * 32) xxh_quad_kernel(const Params p) {
     uint32_t next = 0;
     if (lane == 0) next = warps + atomicAdd(p.ticket, 1u);
     next = __shfl_sync(0xffffffffu, next, 0);
-    const uint32_t idx = batch * 8 + q;
+    const uint32_t idx = batch * CPW + q;
     const bool mine = idx < p.n_desc;
     SegDesc d{};
     if (mine) d = p.desc[idx];
     const uint64_t len = mine ? d.bytes : 0, len16 = len & ~15ull;
-    const uint32_t nst = (uint32_t)((len16 + STG - 1) / STG);
-    uint32_t nst_max = nst;
-#pragma unroll
-    for (int o = 16; o >= 4; o >>= 1) nst_max = max(nst_max, __shfl_xor_sync(0xffffffffu, nst_max, o));
-    // stage k of all 8 chunks: lane 0 arms the barrier with their byte total, quad leaders copy
+    const uint32_t nst_max = __reduce_max_sync(0xffffffffu, (uint32_t)((len16 + STG - 1) / STG));
+    // stage k of all the warp's chunks: lane 0 arms the barrier with their byte total, group leaders copy
     auto issue = [&](uint32_t k) {
       const uint32_t b = (seq + k) % S;
       const uint64_t o = (uint64_t)k * STG;
       const uint32_t sz = o < len16 ? (uint32_t)(len16 - o < STG ? len16 - o : STG) : 0u;
-      uint32_t tot = j == 0 ? sz : 0u;
-#pragma unroll
-      for (int x = 16; x > 0; x >>= 1) tot += __shfl_xor_sync(0xffffffffu, tot, x);
+      const uint32_t tot = __reduce_add_sync(0xffffffffu, j == 0 ? sz : 0u);
       if (lane == 0) {
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         mbar_expect_tx(bars + b, tot);
@@ -1182,7 +1182,12 @@ __global__ void __launch_bounds__(W * 32) xxh_quad_kernel(const Params p) {
       if (j == 0 && sz) bulk_g2s(ring + (size_t)b * STG, reinterpret_cast<const uint8_t*>(d.dev) + o, sz, bars + b);
     };
     for (uint32_t k = 0; k < nst_max && k < (uint32_t)S; ++k) issue(k);
-    uint64_t v = TF ? xt_init(j) : j == 0 ? P1 + P2 : j == 1 ? P2 : j == 2 ? 0ull : 0ull - P1;
+    uint64_t v[NC];
+#pragma unroll
+    for (int c = 0; c < NC; ++c) {
+      const int a = j + c * LPC;  // accumulator index 0..3
+      v[c] = TF ? xt_init(a) : a == 0 ? P1 + P2 : a == 1 ? P2 : a == 2 ? 0ull : 0ull - P1;
+    }
     const uint64_t stripes = len / 32;
     for (uint32_t k = 0; k < nst_max; ++k) {
       const uint32_t b = (seq + k) % S;
@@ -1191,20 +1196,30 @@ __global__ void __launch_bounds__(W * 32) xxh_quad_kernel(const Params p) {
       if (s0 < stripes) {
         const uint8_t* qb = ring + (size_t)b * STG + 8 * j;
         const uint32_t ns = (uint32_t)(stripes - s0 < (uint64_t)(STG / 32) ? stripes - s0 : (uint64_t)(STG / 32));
+        auto stripe = [&](uint32_t s) {
+#pragma unroll
+          for (int c = 0; c < NC; ++c) {
+            const uint64_t w = lds_u64(qb + 32 * s + 8 * LPC * c);
+            v[c] = TF ? xt_step(v[c], w) : xround(v[c], w);
+          }
+        };
         if (ns == STG / 32) {
 #pragma unroll 16
-          for (uint32_t s = 0; s < (uint32_t)(STG / 32); ++s) v = TF ? xt_step(v, lds_u64(qb + 32 * s)) : xround(v, lds_u64(qb + 32 * s));
+          for (uint32_t s = 0; s < (uint32_t)(STG / 32); ++s) stripe(s);
         } else {
-          for (uint32_t s = 0; s < ns; ++s) v = TF ? xt_step(v, lds_u64(qb + 32 * s)) : xround(v, lds_u64(qb + 32 * s));
+          for (uint32_t s = 0; s < ns; ++s) stripe(s);
         }
       }
       __syncwarp();  // every lane is done with buffer b before it is refilled
       if (k + S < nst_max) issue(k + S);
     }
-    if (TF) v = xt_final(v);
     uint64_t vv[4];
 #pragma unroll
-    for (int x = 0; x < 4; ++x) vv[x] = __shfl_sync(0xffffffffu, v, (lane & ~3) + x);
+    for (int c = 0; c < NC; ++c) {
+      if (TF) v[c] = xt_final(v[c]);
+#pragma unroll
+      for (int x = 0; x < LPC; ++x) vv[x + c * LPC] = __shfl_sync(0xffffffffu, v[c], (lane & ~(LPC - 1)) + x);
+    }
     if (mine && j == 0) xxh_finish<MODE>(p, d, vv);
     seq += nst_max;
     batch = next;
@@ -1212,25 +1227,25 @@ __global__ void __launch_bounds__(W * 32) xxh_quad_kernel(const Params p) {
   }
 }
 
-template <int MODE, int W, int S, int STG, bool TF = true>
+template <int MODE, int W, int S, int STG, bool TF = true, int LPC = 4>
 static cudaError_t launch_xxh_quad(const Params& p, int sm_count, cudaStream_t s) {
-  using G = XQ<W, S, STG>;
+  using G = XQ<W, S, STG, LPC>;
   if (!p.ticket) return cudaErrorInvalidValue;
   static unsigned long long attr_set = 0;
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
   if (!((attr_set >> (dev & 63)) & 1ull)) {
-    e = cudaFuncSetAttribute(xxh_quad_kernel<MODE, W, S, STG, TF>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)G::SMEM);
+    e = cudaFuncSetAttribute(xxh_quad_kernel<MODE, W, S, STG, TF, LPC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)G::SMEM);
     if (e != cudaSuccess) return e;
     attr_set |= 1ull << (dev & 63);
   }
-  const uint32_t n_batches = (p.n_desc + 7) / 8;
+  const uint32_t n_batches = (p.n_desc + G::CPW - 1) / G::CPW;
   // one CTA per SM while every warp slot has a batch; fewer CTAs only for tiny images
   const int grid = (int)std::max<uint32_t>(1, std::min<uint32_t>((uint32_t)sm_count, n_batches));
   e = cudaMemsetAsync(p.ticket, 0, sizeof(unsigned int), s);
   if (e != cudaSuccess) return e;
-  xxh_quad_kernel<MODE, W, S, STG, TF><<<grid, W * 32, G::SMEM, s>>>(p);
+  xxh_quad_kernel<MODE, W, S, STG, TF, LPC><<<grid, W * 32, G::SMEM, s>>>(p);
   return cudaGetLastError();
 }
 
@@ -1338,8 +1353,8 @@ static int xxh_variant() {
   const char* e = getenv("SWAP_XXH_KERNEL");
   if (!e) return 0;
   const char* names[] = {"lane8", "bal", "bal8", "dyn", "coop", "coop16", "coop8", "ring", "quad", "quad1k", "quad4k",
-                         "quad_x", "dyn_x"};
-  for (int i = 0; i < 13; ++i)
+                         "quad_x", "dyn_x", "quad2", "pair", "pair2", "quad3k"};
+  for (int i = 0; i < 17; ++i)
     if (!strcmp(e, names[i])) return i + 1;
   return 0;
 }
@@ -1362,37 +1377,27 @@ cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_
     // the spec-form round (xround) instead of the t-form, for A/B measurements
     case 12: return st ? launch_xxh_quad<HASH_STORE, 4, 3, 2048, false>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 4, 3, 2048, false>(p, sm_count, s);
     case 13: return st ? launch_xxh_dyn<HASH_STORE, 4, false>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 4, false>(p, sm_count, s);
+    case 14: return st ? launch_xxh_quad<HASH_STORE, 3, 2, 4096>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 3, 2, 4096>(p, sm_count, s);
+    case 15: return st ? launch_xxh_quad<HASH_STORE, 2, 3, 2048, true, 2>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 2, 3, 2048, true, 2>(p, sm_count, s);
+    case 16: return st ? launch_xxh_quad<HASH_STORE, 2, 2, 3072, true, 2>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 2, 2, 3072, true, 2>(p, sm_count, s);
+    case 17: return st ? launch_xxh_quad<HASH_STORE, 4, 2, 3072>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 4, 2, 3072>(p, sm_count, s);
     default: break;
   }
-  // Measured on config B and an 8-GiB cut of it (profiles/r01_xxh_variants.md): up to
-  // 256 KiB chunks the 8-deep lane kernel wins (5.6-6.0 TB/s); from 1 MiB with many chunks the
-  // dynamic 4-deep launch (5.2 TB/s, 2 % above the balanced one; 8 deep falls to 2.7-2.9 TB/s at 1 MiB
-  // once more than ~7 MB are in flight), with fewer chunks the
-  // balanced 8-deep launch (per-lane rate = bytes in flight / latency), and with only a few thousand
-  // chunks the warp-per-chunk TMA ring. From 2 MiB chunks the warp-cooperative kernel while there are
-  // enough batches for its warps (2 MiB: 4.3 vs 2.0 TB/s; 4 MiB: 3.1 vs 1.5; 8 MiB: 1.7 vs 1.0), else
-  // the ring.
+  // Measured on config B (52.57 GB, profiles/r02_xxh_quad.md), TB/s: the quad-per-chunk
+  // TMA-ring kernel with 4 warps x 2 stages of 3 KiB per chunk from 256 KiB to 4 MiB chunks (256 KiB 6.35
+  // vs the lane kernel 6.19; 512 KiB 6.26; 2 MiB 6.32); with 8 MiB and more (fewer than ~7 K chunks) 3
+  // warps x 2 stages of 4 KiB -- half the per-stage overhead per byte -- (16 MiB 5.06 vs 4.76; the r01
+  // kernels reached 1.16). Below 256 KiB and without a ticket counter, the lane kernels.
   const uint32_t n = p.n_desc, many = (uint32_t)sm_count * 192u;
-  if (p.chunk_bytes <= (256u << 10)) {
+  if (p.chunk_bytes < (256u << 10) || !p.ticket) {
     if (n >= many) return st ? launch_xxh_lane<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane<HASH_CHECK, 8>(p, sm_count, s);
-    return st ? launch_xxh_lane_bal<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8>(p, sm_count, s);
-  }
-  if (p.chunk_bytes >= (2u << 20) && p.ticket) {
-    // big chunks: the warp-cooperative kernel with as many chunks per warp (32 / 16 / 8: 4.9 / 3.6 /
-    // 2.4 GB/s per warp) as still keeps ~all 6 x SMs warps busy, else the ring
-    const uint32_t need = (uint32_t)sm_count * 6 * 85 / 100;
-    if (n / 32 >= need)
-      return st ? launch_xxh_coop<HASH_STORE, 6, 2, 32>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 32>(p, sm_count, s);
-    if (n / 16 >= need)
-      return st ? launch_xxh_coop<HASH_STORE, 6, 2, 16>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 16>(p, sm_count, s);
-    if (n / 8 >= need)
-      return st ? launch_xxh_coop<HASH_STORE, 6, 2, 8>(p, sm_count, s) : launch_xxh_coop<HASH_CHECK, 6, 2, 8>(p, sm_count, s);
+    if (hash_xxh_lane_ok(sm_count, n) || !p.ticket)
+      return st ? launch_xxh_lane_bal<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8>(p, sm_count, s);
     return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
   }
-  if (n >= many) return st ? launch_xxh_dyn<HASH_STORE, 4>(p, sm_count, s) : launch_xxh_dyn<HASH_CHECK, 4>(p, sm_count, s);
-  if (hash_xxh_lane_ok(sm_count, n))
-    return st ? launch_xxh_lane_bal<HASH_STORE, 8>(p, sm_count, s) : launch_xxh_lane_bal<HASH_CHECK, 8>(p, sm_count, s);
-  return st ? launch_xxh_ring<HASH_STORE>(p, sm_count, s) : launch_xxh_ring<HASH_CHECK>(p, sm_count, s);
+  if (p.chunk_bytes >= (8u << 20))
+    return st ? launch_xxh_quad<HASH_STORE, 3, 2, 4096>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 3, 2, 4096>(p, sm_count, s);
+  return st ? launch_xxh_quad<HASH_STORE, 4, 2, 3072>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 4, 2, 3072>(p, sm_count, s);
 }
 
 cudaError_t launch_mover(int mode, int kind, const Params& p, int grid, cudaStream_t s) {

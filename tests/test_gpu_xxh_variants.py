@@ -36,7 +36,7 @@ print("variant ok")
 '''
 
 
-@pytest.mark.parametrize("variant", ["lane8", "bal", "bal8", "dyn", "coop", "coop16", "coop8", "ring", "quad", "quad1k", "quad4k", "quad_x", "dyn_x"])
+@pytest.mark.parametrize("variant", ["lane8", "bal", "bal8", "dyn", "coop", "coop16", "coop8", "ring", "quad", "quad1k", "quad4k", "quad_x", "dyn_x", "quad2", "pair", "pair2"])
 def test_xxh64_kernel_variant(variant):
     env = dict(os.environ, SWAP_XXH_KERNEL=variant)
     out = subprocess.run([sys.executable, "-c", SCRIPT, ROOT], capture_output=True, text=True, env=env, timeout=600)

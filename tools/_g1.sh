@@ -1,5 +1,5 @@
 cd "${GRAFT_REPO_ROOT:-.}"; mkdir -p gpurun_out
-timeout 900 python -m pytest tests/test_gpu_xxh_variants.py -q -x --timeout 600 2>&1 | tail -3
-for C in 16777216 4194304 1048576 262144; do
-  timeout 600 python tools/hash_bench.py --checksum xxh64 --chunk $C --reps 8 --variants dyn,dyn_x,quad,quad_x,quad1k,lane8 2>&1 | grep -v Warn
+for C in 262144 524288 2097152 8388608 16777216; do
+  timeout 600 python tools/hash_bench.py --checksum xxh64 --chunk $C --reps 8 --variants quad,quad2,quad3k,quad1k,lane8,dyn 2>&1 | grep -v Warn
 done
+timeout 600 python tools/hash_bench.py --checksum crc32c --chunk 1048576 --reps 8 2>&1 | grep -v Warn
