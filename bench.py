@@ -5,9 +5,10 @@
 One step = one pass of the whole hot path over the engine image:
   a3 checkpoint (gather + fused chunk checksums)  -> a4 manifest seal (swap_sync)
   -> a5 summary all-gather (N>1)  -> a6 poison the regions (harness; outside the swap-in clock)
-  -> a7 restore (scatter + fused compare) -> a8 HBM verify pass -> a9 mismatch all-reduce (N>1).
-value = whole-job swap-in throughput: sum over ranks of image payload bytes / max over ranks of
-the mean device time of (restore + verify), CUDA events on the launching stream.
+  -> barrier -> a7 restore (scatter + fused compare) -> a8 HBM verify pass -> a9 mismatch all-reduce (K6).
+Swap-in latency of a step = max over ranks of (a7 + a8 + a9) measured on the device with CUDA events on
+the ctx's stream, every rank released by the same barrier. value = whole-job swap-in
+throughput = sum over ranks of image payload bytes / mean over the timed steps of that per-step max.
 
     python bench.py [--gpus N --steps K --warmup W] [--impl reference]
     torchrun --nproc-per-node N bench.py --gpus N ...   (one rank per GPU, NCCL)
@@ -15,16 +16,18 @@ the mean device time of (restore + verify), CUDA events on the launching stream.
 Workload (config.workload): N=1 -> BASELINE.json configs[1] (Llama-3.1-8B bf16 engine, 291
 regions, 52.57 GB); N>1 -> each rank its shard of configs[3] (Llama-3.1-70B TP=8, 627 regions,
 30.53 GB/rank; weak scaling). Inputs are far larger than the 126 MB L2, so no flush is needed.
+Each rank's pinned image lives on its GPU's NUMA node and the rank runs on that node's CPUs.
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import platform
 import statistics
 import subprocess
 import sys
-import tempfile
+import threading
 import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
@@ -43,8 +46,8 @@ RESTORE_KERNEL = {
     "ce_batch": "restore phase: coalesced cudaMemcpyAsync runs + HBM hash pass",
 }
 VERIFY_KERNEL = {"crc32c": "hash_kernel<HASH_CHECK> (CRC-32C: quad-line 256-bit loads, per-lane replicated slice-by-4 + Z^96 tables)",
-                 "xxh64": "xxh_dyn_kernel<HASH_CHECK> (XXH64, one lane per chunk, chunks claimed from a ticket; "
-                           "lane / TMA-ring kernels for other chunk sizes and counts)"}
+                 "xxh64": "xxh_quad_kernel<HASH_CHECK> (XXH64: a lane quad per chunk, per-chunk TMA rings in shared memory; "
+                          "lane kernels below 256 KiB chunks)"}
 PCIE_GEN5_X16_GBPS = 63.015  # 64 GB/s x 128/130 (nominal, per direction)
 MEASURED_PEAKS = os.path.join(ROOT, "MEASURED_PEAKS.json")
 NCU_TRAFFIC = os.path.join(ROOT, "profiles", "ncu_traffic.json")  # dram bytes per verify launch (ncu --set full)
@@ -77,35 +80,144 @@ def parse():
     ap.add_argument("--grid", type=int, default=0)
     ap.add_argument("--no-compare", action="store_true", help="skip the other-mechanism comparison")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--sample-bytes", type=int, default=1 << 30, help="oracle sample size per step")
+    ap.add_argument("--no-assisted", action="store_true", help="skip the N>1 NVLink-assisted restore leg")
+    ap.add_argument("--sample-bytes", type=int, default=8 << 30, help="oracle sample size per step")
+    ap.add_argument("--allow-kv-shrink", action="store_true",
+                    help="if host RAM cannot hold every rank's image, shrink the KV pool (the line then names a "
+                         "different workload) instead of refusing to run")
     ap.add_argument("--out", default=None, help="also append the JSON line to this file")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo: test mode, several ranks may share one GPU (collectives on CPU)")
     return ap.parse_args()
 
 
-def host_mem_available() -> int:
+# ---------------------------------------------------------------------------- host topology
+def _read(path: str) -> str:
     try:
-        with open("/proc/meminfo") as f:
-            for line in f:
-                if line.startswith("MemAvailable:"):
-                    return int(line.split()[1]) * 1024
+        with open(path) as f:
+            return f.read().strip()
     except OSError:
-        pass
+        return ""
+
+
+def parse_cpulist(s: str) -> list[int]:
+    out = []
+    for part in s.split(","):
+        part = part.strip()
+        if not part:
+            continue
+        if "-" in part:
+            a, b = part.split("-")
+            out.extend(range(int(a), int(b) + 1))
+        else:
+            out.append(int(part))
+    return out
+
+
+def numa_nodes() -> list[int]:
+    return parse_cpulist(_read("/sys/devices/system/node/online")) or [0]
+
+
+def pci_bus(device: int) -> str:
+    """The device's PCI function as sysfs names it ("0000:1b:00.0"), "" if unknown."""
+    try:
+        import torch
+
+        p = torch.cuda.get_device_properties(device)
+        return f"{p.pci_domain_id:04x}:{p.pci_bus_id:02x}:{p.pci_device_id:02x}.0"
+    except Exception:  # noqa: BLE001
+        return ""
+
+
+def gpu_numa_node(device: int) -> int:
+    """NUMA node of the GPU's PCI function (sysfs), -1 if unknown."""
+    v = _read(f"/sys/bus/pci/devices/{pci_bus(device)}/numa_node")
+    return int(v) if v.lstrip("-").isdigit() else -1
+
+
+def node_cpus(node: int) -> list[int]:
+    return parse_cpulist(_read(f"/sys/devices/system/node/node{node}/cpulist")) if node >= 0 else []
+
+
+def physical_cores(cpus: list[int]) -> int:
+    """Distinct (package, core) pairs among `cpus` (hyperthreads counted once)."""
+    seen = set()
+    for c in cpus:
+        pkg = _read(f"/sys/devices/system/cpu/cpu{c}/topology/physical_package_id")
+        core = _read(f"/sys/devices/system/cpu/cpu{c}/topology/core_id")
+        seen.add((pkg, core) if core else (None, c))
+    return len(seen)
+
+
+def cpu_model() -> str:
+    for line in _read("/proc/cpuinfo").splitlines():
+        if line.startswith("model name"):
+            return line.split(":", 1)[1].strip()
+    return platform.processor() or "unknown"
+
+
+def run_cmd(cmd: list[str], timeout: float = 20) -> str:
+    try:
+        return subprocess.run(cmd, capture_output=True, text=True, timeout=timeout).stdout.strip()
+    except (OSError, subprocess.SubprocessError):
+        return ""
+
+
+def topology() -> dict:
+    """Host link / NUMA record for the line (topo -m, PCIe gen/width, numactl -H)."""
+    q = run_cmd(["nvidia-smi", "--query-gpu=index,pci.bus_id,pcie.link.gen.current,pcie.link.gen.max,"
+                 "pcie.link.width.current,pcie.link.width.max", "--format=csv,noheader"])
+    links = []
+    for line in q.splitlines():
+        f = [x.strip() for x in line.split(",")]
+        if len(f) == 6:
+            links.append({"gpu": int(f[0]), "bus": f[1], "gen": f[2], "gen_max": f[3], "width": f[4], "width_max": f[5]})
+    numactl = run_cmd(["numactl", "-H"])
+    nodes = {}
+    for n in numa_nodes():
+        cpus = node_cpus(n)
+        mem = _read(f"/sys/devices/system/node/node{n}/meminfo")
+        total_kb = next((int(l.split()[-2]) for l in mem.splitlines() if "MemTotal" in l), 0)
+        nodes[str(n)] = {"cpus": len(cpus), "physical_cores": physical_cores(cpus), "mem_gb": round(total_kb / 1e6, 1)}
+    return {"pcie": links, "topo_m": run_cmd(["nvidia-smi", "topo", "-m"]).splitlines(),
+            "numactl_H": numactl.splitlines()[:12] if numactl else "numactl not installed (sysfs below)",
+            "numa_nodes": nodes, "cpu_model": cpu_model(), "host_cpus": os.cpu_count()}
+
+
+def bind_to_node(node: int) -> list[int]:
+    """Runs this rank on its GPU's NUMA node (no-op on one-node hosts); returns the CPUs used."""
+    cpus = node_cpus(node) if node >= 0 and len(numa_nodes()) > 1 else []
+    if cpus:
+        try:
+            os.sched_setaffinity(0, cpus)
+        except OSError:
+            cpus = []
+    return cpus
+
+
+def host_mem_available() -> int:
+    for line in _read("/proc/meminfo").splitlines():
+        if line.startswith("MemAvailable:"):
+            return int(line.split()[1]) * 1024
     return 0
 
 
-def fit_host(specs, local_ranks: int):
+def check_host(specs, local_ranks: int, allow_shrink: bool):
     """Every rank pins an image as large as its payload. If the node's free RAM cannot hold all local
-    ranks' images (with 20 % headroom), shrink the KV-pool regions uniformly and say so; weights and
-    workspace keep their shapes. Returns (specs, kv_scale)."""
+    ranks' images (with 15 % headroom), refuse to run (a smaller workload is not the named config);
+    with --allow-kv-shrink, shrink the KV-pool regions uniformly and say so in the workload name.
+    Returns (specs, kv_scale)."""
     avail = host_mem_available()
     need = sum(r.nbytes for r in specs) * local_ranks
-    if not avail or need <= 0.8 * avail:
+    if not avail or need <= 0.85 * avail:
         return specs, 1.0
+    if not allow_shrink:
+        raise SystemExit(f"bench.py: {local_ranks} ranks x {need / local_ranks / GB:.1f} GB of pinned image exceed "
+                         f"85% of MemAvailable ({avail / GB:.1f} GB); refusing to measure a smaller workload "
+                         f"(pass --allow-kv-shrink to shrink the KV pool under a different workload name)")
     kv = sum(r.nbytes for r in specs if r.kind == W.KIND_KV)
     other = sum(r.nbytes for r in specs) - kv
-    budget = 0.8 * avail / local_ranks - other
+    budget = 0.85 * avail / local_ranks - other
     scale = max(0.05, budget / kv) if kv else 1.0
     out = [W.RegionSpec(r.name, r.kind, int(r.nbytes * scale) // 4096 * 4096, r.dtype) if r.kind == W.KIND_KV else r
            for r in specs]
@@ -124,48 +236,89 @@ def workload(cfg: str, rank: int, world: int):
     return "D", W.config_d(rank), "Llama-3.1-70B bf16 TP=8 engine shard per rank (BASELINE configs[3])"
 
 
+# ---------------------------------------------------------------------------- clocks
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    """SM clock, power and throttle reasons sampled every 5 ms during the timed region (NVML in a
+    thread; nvidia-smi -lms 20 when NVML is unavailable), so even a 64 MiB image gets samples."""
 
-    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
-         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap")
+    HW_SLOWDOWN, SW_THERMAL, HW_THERMAL, SW_POWER = 0x8, 0x20, 0x40, 0x4
+    PERIOD = 0.005
 
     def __init__(self, device: int):
         self.device = device
-        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
-        self.p = None
+        self.bus = pci_bus(device)  # NVML / nvidia-smi index by PCI bus id (CUDA_VISIBLE_DEVICES-proof)
+        self.rows: list[tuple[float, float, float, int]] = []
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._t = None
+        self._nvml = None
 
     def start(self):
         try:
-            self.p = subprocess.Popen(["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.Q}",
-                                       "--format=csv,noheader,nounits", "-lms", "200"], stdout=self.f,
-                                      stderr=subprocess.DEVNULL)
+            import pynvml
+
+            pynvml.nvmlInit()
+            h = pynvml.nvmlDeviceGetHandleByPciBusId(self.bus.encode()) if self.bus else \
+                pynvml.nvmlDeviceGetHandleByIndex(self.device)
+            self.max_mhz = float(pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM))
+            self._nvml = (pynvml, h)
+        except Exception:  # noqa: BLE001 - no NVML: fall back to nvidia-smi
+            self._nvml = None
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+
+    def _sample_nvml(self):
+        pynvml, h = self._nvml
+        sm = float(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM))
+        pw = pynvml.nvmlDeviceGetPowerUsage(h) / 1000.0
+        rs = int(pynvml.nvmlDeviceGetCurrentClocksThrottleReasons(h))
+        return sm, pw, rs
+
+    def _run(self):
+        if self._nvml is not None:
+            while not self._stop.is_set():
+                try:
+                    sm, pw, rs = self._sample_nvml()
+                    self.rows.append((time.perf_counter(), sm, pw, rs))
+                except Exception:  # noqa: BLE001
+                    pass
+                self._stop.wait(self.PERIOD)
+            return
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        try:
+            p = subprocess.Popen(["nvidia-smi", "-i", self.bus or str(self.device), f"--query-gpu={q}", "--format=csv,noheader,nounits",
+                                  "-lms", "20"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
         except OSError:
-            self.p = None
+            return
+        bits = [self.HW_SLOWDOWN, self.HW_THERMAL, self.SW_THERMAL, self.SW_POWER]
+        for line in p.stdout:
+            if self._stop.is_set():
+                break
+            f = [x.strip() for x in line.split(",")]
+            if len(f) == 7 and f[0].replace(".", "").isdigit():
+                self.max_mhz = float(f[1])
+                rs = sum(b for b, v in zip(bits, f[3:]) if v.lower().startswith("active"))
+                self.rows.append((time.perf_counter(), float(f[0]), float(f[2]) if f[2].replace(".", "").isdigit() else 0.0, rs))
+        p.terminate()
 
     def stop(self) -> dict:
-        if self.p is None:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        self.p.terminate()
-        self.p.wait(5)
-        self.f.flush()
-        rows = []
-        with open(self.f.name) as fh:
-            for line in fh:
-                parts = [x.strip() for x in line.split(",")]
-                if len(parts) == 8 and parts[1].replace(".", "").isdigit():
-                    rows.append(parts)
-        os.unlink(self.f.name)
-        if not rows:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in rows for i in range(4) if r[4 + i].lower().startswith("active")})
-        return {"sm_mhz": statistics.median(float(r[1]) for r in rows), "sm_max_mhz": float(rows[0][2]),
-                "power_w_max": max(float(r[3]) for r in rows if r[3].replace(".", "").isdigit()) if rows else None,
-                "samples": len(rows), "reasons": reasons}
+        self._stop.set()
+        if self._t:
+            self._t.join(5)
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["no samples"], "samples": 0}
+        names = {self.HW_SLOWDOWN: "hw_slowdown", self.HW_THERMAL: "hw_thermal_slowdown",
+                 self.SW_THERMAL: "sw_thermal_slowdown", self.SW_POWER: "sw_power_cap"}
+        reasons = sorted({n for b, n in names.items() for r in self.rows if r[3] & b})
+        return {"sm_mhz": statistics.median(r[1] for r in self.rows), "sm_max_mhz": self.max_mhz,
+                "power_w_max": round(max(r[2] for r in self.rows), 1), "samples": len(self.rows),
+                "period_ms": int(self.PERIOD * 1000), "source": "nvml" if self._nvml else "nvidia-smi",
+                "reasons": reasons}
 
 
+# ---------------------------------------------------------------------------- CPU oracle timing
 def oracle_sample_specs(specs, limit: int):
     """A prefix of the workload's regions, at most `limit` bytes (bounded CPU sample)."""
     out, tot = [], 0
@@ -177,7 +330,7 @@ def oracle_sample_specs(specs, limit: int):
     return out, tot
 
 
-def time_oracle_restore(orc, specs, host, offs, threads: int, reps: int):
+def time_oracle_restore(orc, specs, host, offs, threads: int, reps: int, fast: bool = False):
     """Oracle restore (memcpy + chunk checksum compare) of the sample; returns (GB/s list, bytes)."""
     base = 1 << 40
     regs = [(i, base + o, r.nbytes, r.kind) for i, (r, o) in enumerate(zip(specs, offs))]
@@ -187,11 +340,24 @@ def time_oracle_restore(orc, specs, host, offs, threads: int, reps: int):
     rates = []
     for _ in range(reps):
         t0 = time.perf_counter()
-        rc, nbad, _ = orc.restore(image, moff, host, base, threads=threads)
+        rc, nbad, _ = orc.restore(image, moff, host, base, threads=threads, fast=fast)
         dt = time.perf_counter() - t0
         assert rc == 0 and nbad == 0
         rates.append(payload / dt / GB)
     return rates, payload
+
+
+def cpu_threads() -> int:
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+def cpu_context(cpus: list[int]) -> dict:
+    mine = cpus or sorted(os.sched_getaffinity(0))
+    return {"cpu_model": cpu_model(), "threads_used": len(mine), "physical_cores_used": physical_cores(mine),
+            "host_logical_cpus": os.cpu_count(), "numa_nodes": len(numa_nodes())}
 
 
 def overhead(compare: dict, restore_gbps: float, ce: dict) -> dict | None:
@@ -205,13 +371,6 @@ def overhead(compare: dict, restore_gbps: float, ce: dict) -> dict | None:
     if ce.get("h2d"):
         out["default_restore_vs_bare_ce_h2d"] = round(ce["h2d"] / restore_gbps - 1, 4)
     return out or None
-
-
-def cpu_threads() -> int:
-    try:
-        return len(os.sched_getaffinity(0))
-    except AttributeError:
-        return os.cpu_count() or 1
 
 
 # ---------------------------------------------------------------------------- reference arm
@@ -229,18 +388,22 @@ def run_reference(args):
     rates, payload = time_oracle_restore(oracle, sample, host, offs, th, args.warmup + args.steps)
     timed = rates[args.warmup:]
     v = statistics.mean(timed)
+    total = sum(r.nbytes for r in specs)
     line = {
         "impl": "reference", "metric": METRIC, "value": round(v, 3),
         "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(payload / (v * GB) * 1e3, 3), "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": {"workload": f"{name}: {desc}", "regions_per_rank": len(specs),
-                   "payload_bytes_per_rank": sum(r.nbytes for r in specs), "chunk_bytes": 1 << 20,
+                   "payload_bytes_per_rank": total, "chunk_bytes": 1 << 20,
                    "checksum": "crc32c", "mechanism": "cpu oracle",
-                   "sample": f"each step restores the first {len(sample)} regions ({payload} B) on the host"},
+                   "sample": f"each step restores the first {len(sample)} regions ({payload} B = "
+                             f"{payload / total:.1%} of the per-rank image) on the host"},
         "cpu_baseline": {"value": round(v, 3), "unit": "GB/s", "cores": th, "kind": "oracle",
                          "sample": f"oracle_restore (memcpy + Sarwate CRC-32C per 1 MiB chunk) over the first "
-                                   f"{len(sample)} regions of workload {name} ({payload} B), {th} OpenMP threads"},
+                                   f"{len(sample)} regions of workload {name} ({payload} B = {payload / total:.1%} "
+                                   f"of the image), {th} OpenMP threads",
+                         **cpu_context([])},
         "e2e": {"value": round(v, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -257,12 +420,15 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", "1"))
     if world != args.gpus:
         print(f"warning: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
     ndev = torch.cuda.device_count()
     local_dev = local % ndev if args.dist_backend == "gloo" else local
     torch.cuda.set_device(local_dev)
     dev = torch.device("cuda", local_dev)
+    node = gpu_numa_node(local_dev)
+    my_cpus = bind_to_node(node)  # before any large host allocation or thread
     if world > 1:
         if args.dist_backend == "nccl":
             tdist.init_process_group("nccl", device_id=dev)
@@ -271,26 +437,32 @@ def run_ours(args):
     cdev = dev if args.dist_backend == "nccl" else torch.device("cpu")  # where collective tensors live
 
     def barrier():
+        torch.cuda.synchronize()
         if world > 1:
             tdist.barrier()
-        torch.cuda.synchronize()
+
+    def allreduce(vals: list[float], op) -> list[float]:
+        if world == 1:
+            return list(vals)
+        t = torch.tensor(vals, dtype=torch.float64, device=cdev)
+        tdist.all_reduce(t, op=op)
+        return t.cpu().tolist()
 
     def allmax(x: float) -> float:
-        if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device=cdev)
-        tdist.all_reduce(t, op=tdist.ReduceOp.MAX)
-        return float(t.item())
+        return allreduce([x], tdist.ReduceOp.MAX if world > 1 else None)[0]
 
     def allsum(x: float) -> float:
+        return allreduce([x], tdist.ReduceOp.SUM if world > 1 else None)[0]
+
+    def gather_obj(x):
         if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device=cdev)
-        tdist.all_reduce(t, op=tdist.ReduceOp.SUM)
-        return float(t.item())
+            return [x]
+        out = [None] * world
+        tdist.all_gather_object(out, x)
+        return out
 
     name, specs, desc = workload(args.config, rank, world)
-    specs, kv_scale = fit_host(specs, int(os.environ.get("LOCAL_WORLD_SIZE", "1")))
+    specs, kv_scale = check_host(specs, local_world, args.allow_kv_shrink)
     offs, arena_bytes = W.place(specs)
     payload = sum(r.nbytes for r in specs)
     t0 = time.perf_counter()
@@ -305,7 +477,8 @@ def run_ours(args):
     sw = swap.Swapper(regions, chunk_bytes=args.chunk, checksum=kind, mechanism=args.mechanism, device=local_dev,
                       rank=rank, world=world, grid_ctas=args.grid)
     t_register = time.perf_counter() - t0
-    eff_mech = sw.mechanism()
+    eff_mech = sw.mechanism("restore")
+    eff_mech_ckpt = sw.mechanism("checkpoint")
     stream = torch.cuda.Stream(device=dev)
 
     def poison():
@@ -314,23 +487,30 @@ def run_ours(args):
                 if r.nbytes:
                     arena[o:o + r.nbytes].fill_(W.POISON_BYTE)
 
+    def agree(res) -> int:  # a9 (K6), ordered after the verify on the ctx's stream
+        if world == 1:
+            return res["n_bad"] + res["hbm_n_bad"] + (0 if res["manifest_ok"] else 1)
+        with torch.cuda.stream(stream):
+            return sdist.agree_restore(res, None)
+
     def step(record: dict | None):
         """One pass of the hot path; returns per-phase device/host times."""
         sw.checkpoint(stream, sync=True)  # a3 + a4
         if world > 1:
             sdist.gather_manifest(sw, None)  # a5
-        poison()  # a6 (harness, untimed): finish it before the host clock starts, or e2e would count
-        stream.synchronize()  # ~10 ms of HBM fills that precede the restore on the stream
+        poison()  # a6 (harness, untimed): finished before the clock starts
+        stream.synchronize()
+        barrier()  # every rank starts its swap-in together (SURVEY.md §8(d))
         ev0 = torch.cuda.Event(enable_timing=True)
         ev1 = torch.cuda.Event(enable_timing=True)
         ev0.record(stream)
         h0 = time.perf_counter()
         sw.restore(stream)  # a7
         res = sw.verify(stream, hbm_pass=True)  # a8 (synchronises the stream)
-        h1 = time.perf_counter()
+        bad = agree(res)  # a9 (K6): inside both clocks
         ev1.record(stream)
-        bad = sdist.agree_restore(res, None) if world > 1 else res["n_bad"] + res["hbm_n_bad"]  # a9
         ev1.synchronize()
+        h1 = time.perf_counter()
         assert bad == 0 and res["status"] == 0, res
         if record is not None:
             t = sw.timings()
@@ -358,9 +538,14 @@ def run_ours(args):
     launches = sw.launch_count() - launches0
     step_ms = allmax(e_start.elapsed_time(e_end) / args.steps)
 
-    swapin_ms = allmax(statistics.mean(rec["swapin_ms"]))
-    host_ms = allmax(statistics.mean(rec["host_ms"]))
-    restore_ms = statistics.mean(rec["restore_ms"])
+    # per-step max over ranks, then the mean over steps (latency = max over ranks)
+    op_max = tdist.ReduceOp.MAX if world > 1 else None
+    swapin_steps = allreduce(rec["swapin_ms"], op_max)
+    host_steps = allreduce(rec["host_ms"], op_max)
+    restore_steps = allreduce(rec["restore_ms"], op_max)
+    swapin_ms = statistics.mean(swapin_steps)
+    host_ms = statistics.mean(host_steps)
+    restore_ms = statistics.mean(rec["restore_ms"])  # this rank's (the roofline is per GPU)
     verify_ms = statistics.mean(rec["verify_ms"])
     ckpt_ms = allmax(statistics.mean(rec["ckpt_ms"]))
     total_payload = allsum(payload)
@@ -407,22 +592,55 @@ def run_ours(args):
             lazy.append(h1 - h0)
         sw.bind_arena(None)
 
-    # copy-engine link peaks measured here (torch pinned copies, 2 GiB)
+    # copy-engine link peaks at the same concurrency: every rank copies 2 GiB each way at once
+    n = min(2 << 30, arena_bytes)
+    h = torch.empty(n, dtype=torch.uint8, pin_memory=True)
     ce = {}
-    if rank == 0:
-        n = min(2 << 30, arena_bytes)
-        h = torch.empty(n, dtype=torch.uint8, pin_memory=True)
-        for nm, (dst, src) in {"h2d": (arena[:n], h), "d2h": (h, arena[:n])}.items():
-            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            with torch.cuda.stream(stream):
+    for nm, (dst, src) in {"h2d": (arena[:n], h), "d2h": (h, arena[:n])}.items():
+        barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        with torch.cuda.stream(stream):
+            dst.copy_(src, non_blocking=True)
+            a.record(stream)
+            for _ in range(3):
                 dst.copy_(src, non_blocking=True)
-                a.record(stream)
+            b.record(stream)
+        b.synchronize()
+        ce[nm] = 3 * n / (a.elapsed_time(b) * 1e-3) / GB
+    del h
+    ce_all = gather_obj({k: round(v, 2) for k, v in ce.items()})
+
+    # NEXT-2: rank 0's swap-in assisted by k idle peers (their PCIe links into HBM staging, then NVLink),
+    # the other ranks idle in a barrier (outside the timed region)
+    assisted = None
+    if world > 1 and args.dist_backend == "nccl" and ndev > 1 and not args.no_assisted:
+        assisted = {}
+        for k in (1, 3, 7):
+            if k > ndev - 1:
+                break
+            barrier()
+            if rank == 0:
+                helpers = [(local_dev + i) % ndev for i in range(1, k + 1)]
+                sw.set_mechanism("ce_pipe")
+                sw.set_helpers(helpers)
+                ts = []
                 for _ in range(3):
-                    dst.copy_(src, non_blocking=True)
-                b.record(stream)
-            b.synchronize()
-            ce[nm] = 3 * n / (a.elapsed_time(b) * 1e-3) / GB
-        del h
+                    poison()
+                    stream.synchronize()
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record(stream)
+                    sw.restore(stream)
+                    res = sw.verify(stream, hbm_pass=True)
+                    e1.record(stream)
+                    e1.synchronize()
+                    assert res["status"] == 0 and res["n_bad"] == 0 and res["hbm_n_bad"] == 0, res
+                    ts.append(e0.elapsed_time(e1) * 1e-3)
+                sw.set_helpers([])
+                sw.set_mechanism(args.mechanism)
+                t = statistics.median(ts[1:])
+                assisted[str(k)] = {"helpers": helpers, "swap_in_s": round(t, 4), "GBps": round(payload / t / GB, 2),
+                                    "frac_of_k_plus_1_links": round(payload / t / GB / ((k + 1) * ce["h2d"]), 3)}
+            barrier()
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:  # the oracle beside N=1 only
@@ -432,38 +650,50 @@ def run_ours(args):
         s_offs, s_total = W.place(sample)
         s_host = arena[:s_total].cpu().numpy()  # same placement recipe: the arena prefix holds the sample
         th = cpu_threads()
-        rates, sbytes = time_oracle_restore(oracle, sample, s_host, s_offs, th, 3)
-        cpu = {"value": round(statistics.mean(rates), 3), "unit": "GB/s", "cores": th, "kind": "oracle",
+        ref_rates, sbytes = time_oracle_restore(oracle, sample, s_host, s_offs, th, 3)
+        fast_rates, _ = time_oracle_restore(oracle, sample, s_host, s_offs, th, 3, fast=True)
+        del s_host
+        cpu = {"value": round(statistics.mean(ref_rates), 3), "unit": "GB/s", "cores": th, "kind": "oracle",
                "sample": f"oracle_restore (memcpy + Sarwate CRC-32C per 1 MiB chunk) over the first {len(sample)} "
-                         f"regions of workload {name} ({sbytes} B, contents copied from the GPU arena), "
-                         f"{th} OpenMP threads, mean of 3"}
+                         f"regions of workload {name} ({sbytes} B = {sbytes / payload:.1%} of the image, contents "
+                         f"copied from the GPU arena), {th} OpenMP threads, mean of 3",
+               "fast": {"value": round(statistics.mean(fast_rates), 3), "unit": "GB/s",
+                        "how": "same sample and threads, CRC-32C by the SSE4.2 crc32 instruction"},
+               **cpu_context(my_cpus)}
 
+    numa = sw.numa()
+    placement = gather_obj({"rank": rank, "gpu": local_dev, "gpu_numa_node": node, "cpus": len(my_cpus),
+                            "image_numa_node": numa["node"], "image_local_fraction": numa["local_fraction"]})
     if rank == 0:
         value = total_payload / (swapin_ms * 1e-3) / GB
         achieved = payload / (restore_ms * 1e-3) / GB
         peaks = json.load(open(MEASURED_PEAKS)) if os.path.exists(MEASURED_PEAKS) else {}
         hbm_peak = peaks.get("hbm_gbs", 6650.0)
+        workload_name = f"{name}: {desc}" + ("" if kv_scale == 1.0 else f" -- KV pool SHRUNK x{kv_scale} to fit host RAM (not the named config)")
         line = {
-            "metric": METRIC, "value": round(value, 3),
+            "metric": METRIC if kv_scale == 1.0 else METRIC + " (KV pool shrunk)", "value": round(value, 3),
             "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
             "ms_per_step": round(step_ms, 3), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "u8", "data": "synthetic",
-            "config": {"workload": f"{name}: {desc}" + ("" if kv_scale == 1.0 else f" (KV pool scaled x{kv_scale} to fit host RAM)"),
+            "config": {"workload": workload_name,
                        "regions_per_rank": len(specs),
                        "payload_bytes_per_rank": payload, "chunk_bytes": args.chunk, "checksum": args.checksum,
-                       "mechanism": f"{args.mechanism} -> {eff_mech}",
+                       "mechanism": f"{args.mechanism} -> restore {eff_mech}, checkpoint {eff_mech_ckpt}",
                        "l2": "no flush: every step moves the whole image (>> 126 MB L2)",
-                       "parallelism": "single GPU" if world == 1 else f"tp{world} shard per rank (no data collective)"},
+                       "parallelism": "single GPU" if world == 1 else f"tp{world} shard per rank (no data collective)",
+                       "timing": "per step: barrier, then restore + HBM verify + K6 all-reduce on the ctx stream (CUDA "
+                                 "events); value uses the mean over steps of the per-step max over ranks"},
             "swap_in_latency_s": round(swapin_ms * 1e-3, 5),
-            "swap_in_latency_s_range": [round(min(rec["swapin_ms"]) * 1e-3, 5), round(max(rec["swapin_ms"]) * 1e-3, 5)],
+            "swap_in_latency_s_range": [round(min(swapin_steps) * 1e-3, 5), round(max(swapin_steps) * 1e-3, 5)],
             "restore_GBps_per_gpu": round(achieved, 3),
+            "restore_GBps_per_gpu_slowest": round(payload / (max(restore_steps) * 1e-3) / GB, 3),
             "checkpoint_GBps_per_gpu": round(payload / (ckpt_ms * 1e-3) / GB, 3),
             "roofline": {"bound": "host_link", "kernel": RESTORE_KERNEL[eff_mech],
                          "achieved": round(achieved, 3), "peak": PCIE_GEN5_X16_GBPS, "unit": "GB/s",
                          "frac": round(achieved / PCIE_GEN5_X16_GBPS, 4), "traffic": None,
                          "traffic_note": "copy-engine / link transfer: no kernel DRAM counters (see roofline_verify.traffic)",
                          "peak_source": "PCIe Gen5 x16 nominal per direction after 128b/130b (MEASURED_PEAKS.json has no host-link figure)",
-                         "frac_of_measured_ce_h2d": round(achieved / ce["h2d"], 4) if ce else None},
+                         "frac_of_measured_ce_h2d": round(achieved / ce["h2d"], 4)},
             "roofline_verify": {"bound": "hbm", "kernel": VERIFY_KERNEL[args.checksum],
                                 "achieved": round(payload / (verify_ms * 1e-3) / GB, 1), "peak": hbm_peak,
                                 "unit": "GB/s", "frac": round(payload / (verify_ms * 1e-3) / GB / hbm_peak, 4),
@@ -471,21 +701,25 @@ def run_ours(args):
                                 "traffic_detail": ncu_traffic(name, args.checksum, payload),
                                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)"},
             "measured_ce_GBps": {k: round(v, 2) for k, v in ce.items()},
+            "measured_ce_GBps_all_ranks": ce_all,
             "mechanisms": compare,
             "fused_checksum_overhead": overhead(compare, achieved, ce),
+            "assisted_swap_in": assisted,
             "setup_s": {"fill": round(t_fill, 2), "register_pin": round(t_register, 2)},
             "swap_in_with_hbm_reacquire_s": round(statistics.mean(x[1] for x in reacq), 4),
             "hbm_reacquire_s": round(statistics.mean(x[0] for x in reacq), 4),
             "swap_in_with_overlapped_reacquire_s": round(statistics.mean(lazy), 4),
             "e2e": {"value": round(total_payload / (host_ms * 1e-3) / GB, 3), "unit": "GB/s",
                     "h2d_bytes_per_step": payload, "d2h_bytes_per_step": 32,
-                    "how": "host wall clock (perf_counter) around swap_restore + swap_verify called through the C ABI "
-                           "(ctypes), image in pinned host DRAM: the H2D copy of every payload byte and the D2H read "
-                           "of the 32-B verify status are inside; the harness poison is finished before the clock "
-                           "starts. It lands within ~0.1 % of the device-timed value because the device-timed "
-                           "metric is itself the host-to-device transfer"},
+                    "how": "host wall clock (perf_counter) around swap_restore + swap_verify (+ the K6 all-reduce) "
+                           "called through the C ABI (ctypes), image in pinned host DRAM: the H2D copy of every payload "
+                           "byte and the D2H read of the 32-B verify status are inside; per-step max over ranks. The "
+                           "harness poison is finished before the clock starts. It lands near the device-timed value "
+                           "because the device-timed metric is itself the host-to-device transfer"},
             "gpu_launches": int(launches),
             "clocks": clk,
+            "placement": placement,
+            "topology": topology(),
             "cpu_baseline": cpu,
         }
         s = json.dumps(line)

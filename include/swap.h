@@ -104,6 +104,13 @@ typedef struct {
                            one segment per warp slot of the GPU, 4 KiB .. 256 KiB) */
   uint32_t pipe_mib;    /* SWAP_MECH_CE_PIPE group size in MiB (rounded up to whole chunks); 0 -> auto: payload/32
                            clamped to [16, 256] MiB */
+  int32_t host_numa;    /* host NUMA placement of the image (per-GPU topology fixed at init):
+                           0 -> auto: the node sysfs reports for the device's PCI function
+                           (/sys/bus/pci/devices/<bus id>/numa_node), preferred policy (mbind
+                           MPOL_PREFERRED) and zero-filling threads pinned to that node's CPUs;
+                           n >= 1 -> node n-1; -1 -> no placement (first touch by unbound threads).
+                           A single-node host or an unknown node means no placement. */
+  uint32_t reserved0;   /* 0 */
 } swap_config_t;
 
 typedef struct {
@@ -248,6 +255,11 @@ typedef struct {
   float reserved;
 } swap_timings_t;
 SWAP_API swap_status swap_get_timings(const swap_ctx_t* ctx, swap_timings_t* out);
+
+/* Where the pinned image lives (REGISTERED+): *node = the NUMA node placement targeted (-1 none),
+ * *local_fraction = share of the image's pages found on that node (256 pages sampled with
+ * get_mempolicy(MPOL_F_NODE | MPOL_F_ADDR); 1.0 when no placement was targeted). */
+SWAP_API swap_status swap_get_numa(const swap_ctx_t* ctx, int32_t* node, double* local_fraction);
 
 /* Number of libswap kernels this ctx has launched in total (for the bench's gpu_launches). */
 SWAP_API swap_status swap_get_launch_count(const swap_ctx_t* ctx, uint64_t* launches);

@@ -85,8 +85,9 @@ def lib():
         L.oracle_summary.restype = ctypes.c_int
         L.oracle_global_digest.argtypes = [u8p, u64]
         L.oracle_global_digest.restype = u32
-        L.oracle_restore.argtypes = [u8p, u64, u8p, u64, u64, u64p, u64p, ctypes.c_int]
-        L.oracle_restore.restype = ctypes.c_int
+        for name in ("oracle_restore", "oracle_restore_fast"):
+            getattr(L, name).argtypes = [u8p, u64, u8p, u64, u64, u64p, u64p, ctypes.c_int]
+            getattr(L, name).restype = ctypes.c_int
         L.oracle_verify.argtypes = [u8p, u8p, u64, u64, u64p, u64p, ctypes.c_int]
         L.oracle_verify.restype = ctypes.c_int
         L.oracle_manifest_ok.argtypes = [u8p]
@@ -230,11 +231,13 @@ def global_digest(summaries: bytes) -> int:
     return lib().oracle_global_digest(_ptr(b), b.size // 64)
 
 
-def restore(image: np.ndarray, manifest_off: int, mem: np.ndarray, mem_base: int, threads: int = 1):
-    """Returns (rc, n_bad, first_bad); writes mem in place."""
+def restore(image: np.ndarray, manifest_off: int, mem: np.ndarray, mem_base: int, threads: int = 1,
+            fast: bool = False):
+    """Returns (rc, n_bad, first_bad); writes mem in place. fast: CRC-32C by the SSE4.2 instruction
+    instead of the Sarwate table (same results; the bench's "fast" CPU timing)."""
     nb, fb = ctypes.c_uint64(), ctypes.c_uint64()
-    rc = lib().oracle_restore(_ptr(image), manifest_off, _ptr(mem), mem_base, mem.size,
-                              ctypes.byref(nb), ctypes.byref(fb), threads)
+    fn = lib().oracle_restore_fast if fast else lib().oracle_restore
+    rc = fn(_ptr(image), manifest_off, _ptr(mem), mem_base, mem.size, ctypes.byref(nb), ctypes.byref(fb), threads)
     return rc, nb.value, fb.value
 
 

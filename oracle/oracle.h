@@ -81,6 +81,9 @@ uint32_t oracle_global_digest(const uint8_t* summaries, uint64_t world);
  * region byte and counts chunks whose hash over the moved bytes != recorded. */
 int oracle_restore(const uint8_t* image, uint64_t manifest_off, uint8_t* mem, uint64_t mem_base,
                    uint64_t mem_len, uint64_t* n_bad, uint64_t* first_bad, int threads);
+/* Same as oracle_restore with CRC-32C from the SSE4.2 instruction: the "fast" CPU timing of the bench. */
+int oracle_restore_fast(const uint8_t* image, uint64_t manifest_off, uint8_t* mem, uint64_t mem_base,
+                        uint64_t mem_len, uint64_t* n_bad, uint64_t* first_bad, int threads);
 int oracle_verify(const uint8_t* manifest, uint8_t* mem, uint64_t mem_base, uint64_t mem_len,
                   uint64_t* n_bad, uint64_t* first_bad, int threads);
 /* Manifest CRC check alone: 1 = intact. */

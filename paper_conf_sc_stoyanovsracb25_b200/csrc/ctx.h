@@ -99,6 +99,8 @@ struct swap_ctx {
     cudaEvent_t ev = nullptr, done = nullptr;
   };
   std::vector<Helper> helpers;
+  int numa_node = -1;         // NUMA node the image placement targeted (-1: none)
+  double numa_local = 1.0;    // sampled share of image pages on numa_node
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };
 

@@ -134,6 +134,8 @@ uint32_t crc32c_host(const void* data, size_t n, uint32_t crc) {
   return ~c;
 }
 
+static_assert(sizeof(swap_config_t) == 56, "swap_config_t layout (include/swap.h)");
+
 swap_status normalize_config(swap_config_t* c, std::string* err) {
   if (c->chunk_bytes == 0) c->chunk_bytes = 1ull << 20;
   if (c->align == 0) c->align = 4096;
@@ -156,6 +158,10 @@ swap_status normalize_config(swap_config_t* c, std::string* err) {
   }
   if (c->seg_bytes != 0 && !pow2_ge(c->seg_bytes, 4096)) {
     *err = "seg_bytes must be 0 (auto) or a power of 2 >= 4096";
+    return SWAP_EINVAL;
+  }
+  if (c->host_numa < -1) {
+    *err = "host_numa must be 0 (auto), -1 (none) or node + 1";
     return SWAP_EINVAL;
   }
   if (c->chunk_bytes > (1ull << 31)) {

@@ -4,12 +4,15 @@
 // P:L115):
 //   CREATED --register--> REGISTERED --checkpoint--> CKPT_PENDING --sync--> CHECKPOINTED
 //   CHECKPOINTED|RESTORED --restore--> RESTORED;   REGISTERED|CHECKPOINTED|RESTORED --checkpoint--> CKPT_PENDING
+#include <sched.h>
 #include <sys/mman.h>
+#include <sys/syscall.h>
 #include <unistd.h>
 
 #include <algorithm>
 #include <cstdio>
 #include <cstring>
+#include <fstream>
 #include <string>
 #include <thread>
 #include <vector>
@@ -77,18 +80,85 @@ swap_status swap_create(const swap_config_t* cfg_in, swap_ctx_t** out) {
   return SWAP_OK;
 }
 
+// ---- host NUMA placement of the image (swap_config_t.host_numa; P:L230 per-GPU topology at init)
+static std::string read_line(const std::string& path) {
+  std::ifstream f(path);
+  std::string s;
+  std::getline(f, s);
+  return s;
+}
+// "0-7,16-23" -> {0..7, 16..23}
+static std::vector<int> parse_list(const std::string& s) {
+  std::vector<int> out;
+  size_t i = 0;
+  while (i < s.size()) {
+    size_t j = s.find(',', i);
+    if (j == std::string::npos) j = s.size();
+    const std::string t = s.substr(i, j - i);
+    int a = -1, b = -1;
+    if (sscanf(t.c_str(), "%d-%d", &a, &b) == 2) {
+      for (int x = a; x <= b; ++x) out.push_back(x);
+    } else if (sscanf(t.c_str(), "%d", &a) == 1) {
+      out.push_back(a);
+    }
+    i = j + 1;
+  }
+  return out;
+}
+static int numa_nodes_online() { return (int)parse_list(read_line("/sys/devices/system/node/online")).size(); }
+// The NUMA node sysfs reports for the device's PCI function, or -1.
+static int device_numa_node(int dev) {
+  char bus[64] = {0};
+  if (cudaDeviceGetPCIBusId(bus, sizeof bus, dev) != cudaSuccess) return -1;
+  unsigned dom = 0, b = 0, d = 0, fn = 0;
+  if (sscanf(bus, "%x:%x:%x.%x", &dom, &b, &d, &fn) != 4) return -1;
+  char path[128];
+  snprintf(path, sizeof path, "/sys/bus/pci/devices/%04x:%02x:%02x.%x/numa_node", dom, b, d, fn);
+  const std::string v = read_line(path);
+  return v.empty() ? -1 : atoi(v.c_str());
+}
+constexpr int kMpolPreferred = 1, kMpolFNode = 1, kMpolFAddr = 2;
+static bool mbind_preferred(void* p, size_t n, int node) {
+  if (node < 0 || node >= 1024) return false;
+  unsigned long mask[16] = {0};
+  mask[node / 64] = 1ul << (node % 64);
+  return syscall(SYS_mbind, p, n, kMpolPreferred, mask, 1025ul, 0u) == 0;
+}
+// Share of `samples` evenly spaced pages of [p, p+n) that reside on `node`.
+static double local_share(const uint8_t* p, size_t n, int node, int samples = 256) {
+  int hit = 0, seen = 0;
+  for (int i = 0; i < samples; ++i) {
+    const uint8_t* a = p + (n / samples) * (size_t)i;
+    int where = -1;
+    if (syscall(SYS_get_mempolicy, &where, nullptr, 0ul, a, (unsigned long)(kMpolFNode | kMpolFAddr)) != 0) continue;
+    ++seen;
+    hit += where == node;
+  }
+  return seen ? (double)hit / seen : 0.0;
+}
+
 // Faults the image's pages in (the kernel zero-fills them) from several threads before pinning:
-// cudaHostRegister would otherwise fault and zero every page from the calling thread alone.
-static void prefault(uint8_t* p, size_t n) {
+// cudaHostRegister would otherwise fault and zero every page from the calling thread alone. With a
+// NUMA node, the threads run on that node's CPUs (first touch + the preferred policy keep the pages there).
+static void prefault(uint8_t* p, size_t n, int node) {
   const size_t page = 2u << 20;
-  const unsigned hw = std::thread::hardware_concurrency();
+  std::vector<int> cpus;
+  if (node >= 0) cpus = parse_list(read_line("/sys/devices/system/node/node" + std::to_string(node) + "/cpulist"));
+  const unsigned hw = cpus.empty() ? std::thread::hardware_concurrency() : (unsigned)cpus.size();
   const size_t k = std::max<size_t>(1, std::min<size_t>({hw ? hw : 1u, 32u, n / page}));
   const size_t per = (n / k + page - 1) / page * page;
   std::vector<std::thread> th;
   for (size_t t = 0; t < k; ++t) {
     const size_t lo = t * per, hi = std::min(n, lo + per);
     if (lo >= hi) break;
-    th.emplace_back([p, lo, hi] {
+    th.emplace_back([p, lo, hi, &cpus] {
+      if (!cpus.empty()) {
+        cpu_set_t set;
+        CPU_ZERO(&set);
+        for (int c : cpus)
+          if (c >= 0 && c < CPU_SETSIZE) CPU_SET(c, &set);
+        sched_setaffinity(0, sizeof set, &set);  // this thread only
+      }
       volatile uint8_t* q = p;
       for (size_t o = lo; o < hi; o += 4096) q[o] = 0;  // a write: a read would map the shared zero page
     });
@@ -121,7 +191,14 @@ swap_status swap_register_regions(swap_ctx_t* c, const swap_region_t* regions, s
   }
   c->image = static_cast<uint8_t*>(m);
   madvise(m, c->map_bytes, MADV_HUGEPAGE);
-  prefault(c->image, c->map_bytes);
+  int node = -1;
+  if (c->cfg.host_numa != -1 && numa_nodes_online() > 1) {
+    node = c->cfg.host_numa > 0 ? c->cfg.host_numa - 1 : device_numa_node(c->cfg.device);
+    if (node >= 0 && !mbind_preferred(m, c->map_bytes, node)) node = -1;
+  }
+  prefault(c->image, c->map_bytes, node);
+  c->numa_node = node;
+  c->numa_local = node >= 0 ? local_share(c->image, c->map_bytes, node) : 1.0;
   cudaError_t e = cudaHostRegister(m, c->map_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
   if (e != cudaSuccess) {
     cudaGetLastError();
@@ -337,6 +414,14 @@ swap_status swap_get_mechanism(const swap_ctx_t* c, uint32_t* effective) {
   if (!c || !effective) return SWAP_EINVAL;
   if (c->st == St::CREATED) return SWAP_ESTATE;
   *effective = resolve_mech(c, 1);
+  return SWAP_OK;
+}
+
+swap_status swap_get_numa(const swap_ctx_t* c, int32_t* node, double* local_fraction) {
+  if (!c || !node || !local_fraction) return SWAP_EINVAL;
+  if (!c->image) return SWAP_ESTATE;
+  *node = c->numa_node;
+  *local_fraction = c->numa_local;
   return SWAP_OK;
 }
 

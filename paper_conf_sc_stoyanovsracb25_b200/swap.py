@@ -30,7 +30,7 @@ U64_MAX = (1 << 64) - 1
 
 EXPORTS = [
     "swap_config_default", "swap_create", "swap_register_regions", "swap_checkpoint", "swap_sync",
-    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_get_mechanism_dir", "swap_set_region_policy", "swap_set_chunk_mask", "swap_get_manifest", "swap_get_image",
+    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_get_mechanism_dir", "swap_get_numa", "swap_set_region_policy", "swap_set_chunk_mask", "swap_get_manifest", "swap_get_image",
     "swap_get_summary", "swap_import", "swap_save", "swap_load", "swap_set_global", "swap_merge_global", "swap_plan_layout", "swap_plan_manifest", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
     "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
@@ -50,7 +50,7 @@ class swap_config_t(ctypes.Structure):
     _fields_ = [("chunk_bytes", ctypes.c_uint64), ("align", ctypes.c_uint64), ("checksum", ctypes.c_uint32),
                 ("mechanism", ctypes.c_uint32), ("device", ctypes.c_int32), ("rank", ctypes.c_int32),
                 ("world", ctypes.c_int32), ("grid_ctas", ctypes.c_uint32), ("seg_bytes", ctypes.c_uint32),
-                ("pipe_mib", ctypes.c_uint32)]
+                ("pipe_mib", ctypes.c_uint32), ("host_numa", ctypes.c_int32), ("reserved0", ctypes.c_uint32)]
 
 
 class swap_verify_result_t(ctypes.Structure):
@@ -74,7 +74,7 @@ class swap_timings_t(ctypes.Structure):
                 ("reserved", ctypes.c_float)]
 
 
-assert ctypes.sizeof(swap_shard_summary_t) == 64 and ctypes.sizeof(swap_config_t) == 48
+assert ctypes.sizeof(swap_shard_summary_t) == 64 and ctypes.sizeof(swap_config_t) == 56
 
 _lib = None
 
@@ -106,6 +106,7 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_set_mechanism": (st, [vp, u32]),
         "swap_get_mechanism": (st, [vp, P(u32)]),
         "swap_get_mechanism_dir": (st, [vp, ctypes.c_int, P(u32)]),
+        "swap_get_numa": (st, [vp, P(ctypes.c_int32), P(ctypes.c_double)]),
         "swap_set_region_policy": (st, [vp, u32, u32]),
         "swap_set_chunk_mask": (st, [vp, u32, vp, ctypes.c_uint64]),
         "swap_get_manifest": (st, [vp, P(vp), P(sz)]),
@@ -253,7 +254,10 @@ class Swapper:
 
     def __init__(self, regions, chunk_bytes: int = 1 << 20, checksum: int = SWAP_CHECKSUM_CRC32C,
                  mechanism: int | str = SWAP_MECH_AUTO, device: int | None = None, rank: int = 0, world: int = 1,
-                 align: int = 4096, grid_ctas: int = 0, seg_bytes: int = 0, pipe_mib: int = 0):
+                 align: int = 4096, grid_ctas: int = 0, seg_bytes: int = 0, pipe_mib: int = 0,
+                 host_numa: int = 0):
+        """host_numa: 0 = place the pinned image on the device's NUMA node (auto), -1 = no placement,
+        n >= 1 = NUMA node n-1 (swap_config_t.host_numa)."""
         L = load()
         table = []
         for i, r in enumerate(regions):
@@ -277,6 +281,7 @@ class Swapper:
         cfg.chunk_bytes, cfg.checksum, cfg.mechanism, cfg.align = chunk_bytes, checksum, mechanism, align
         cfg.device, cfg.rank, cfg.world = device, rank, world
         cfg.grid_ctas, cfg.seg_bytes, cfg.pipe_mib = grid_ctas, seg_bytes, pipe_mib
+        cfg.host_numa = host_numa
         st, h = swap_create(cfg)
         if st:
             raise SwapError(st, "swap_create failed (no sm_100 GPU / bad config)")
@@ -394,6 +399,13 @@ class Swapper:
         p, n = ctypes.c_void_p(), ctypes.c_size_t()
         self._check(load().swap_get_manifest(self._ctx, ctypes.byref(p), ctypes.byref(n)))
         return np.ctypeslib.as_array(ctypes.cast(p, ctypes.POINTER(ctypes.c_uint8)), shape=(n.value,))
+
+    def numa(self) -> dict:
+        """Host NUMA placement of the image (swap_get_numa): the node targeted (-1 none) and the
+        sampled share of its pages on that node."""
+        node, frac = ctypes.c_int32(), ctypes.c_double()
+        self._check(load().swap_get_numa(self._ctx, ctypes.byref(node), ctypes.byref(frac)))
+        return {"node": node.value, "local_fraction": round(frac.value, 4)}
 
     def summary(self) -> bytes:
         s = swap_shard_summary_t()

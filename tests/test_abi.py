@@ -49,11 +49,13 @@ def test_struct_sizes_match_header(swp):
     assert ctypes.sizeof(swp.swap_shard_summary_t) == 64
     assert ctypes.sizeof(swp.swap_region_t) == 24
     assert ctypes.sizeof(swp.swap_verify_result_t) == 40
+    assert ctypes.sizeof(swp.swap_config_t) == 56
 
 
 def test_config_default(swp):
     c = swp.swap_config_default()
     assert (c.chunk_bytes, c.align, c.checksum, c.mechanism, c.world, c.seg_bytes) == (1 << 20, 4096, 1, 0, 1, 0)
+    assert (c.host_numa, c.reserved0) == (0, 0)  # auto NUMA placement
 
 
 def test_status_strings(swp):

@@ -37,3 +37,22 @@ def test_reference_arm_two_ranks():
     assert len(lines) == 1
     rec = json.loads(lines[0])
     assert rec["impl"] == "reference" and rec["cpu_baseline"]["kind"] == "oracle"
+
+
+def test_host_helpers():
+    sys.path.insert(0, ROOT)
+    import bench
+    import workloads as W
+
+    assert bench.parse_cpulist("0-3,8,10-11") == [0, 1, 2, 3, 8, 10, 11]
+    assert bench.parse_cpulist("") == []
+    assert bench.numa_nodes()  # at least node 0
+    topo = bench.topology()
+    assert topo["numa_nodes"] and topo["cpu_model"]
+    specs = W.config_d(0)
+    # an image set that cannot fit is refused unless the shrink is asked for (and then it is named)
+    with pytest.raises(SystemExit):
+        bench.check_host(specs, 10 ** 4, allow_shrink=False)
+    shrunk, scale = bench.check_host(specs, 10 ** 4, allow_shrink=True)
+    assert scale < 1.0 and sum(r.nbytes for r in shrunk) < sum(r.nbytes for r in specs)
+    assert bench.check_host(W.config_a(0), 1, allow_shrink=False) == (W.config_a(0), 1.0)

@@ -27,3 +27,26 @@ def test_bench_two_ranks_gloo():
     assert rec["n_gpus"] == 2 and rec["scaling"] == "weak" and rec["value"] > 0
     assert rec["config"]["payload_bytes_per_rank"] == 1 << 26
     assert rec["gpu_launches"] > 0
+
+
+@pytest.mark.timeout(900)
+def test_bench_two_ranks_gloo_config_d():
+    """The N>1 code path at full per-rank size: two config-D shards (Llama-3.1-70B TP=8, 30.5 GB each) share
+    cuda:0; the line carries per-rank placement, the copy-engine peak measured on all ranks at once, the
+    topology record and clock samples; per-step max over ranks drives the value."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr=127.0.0.1", "--master-port=29535", os.path.join(ROOT, "bench.py"), "--gpus", "2",
+           "--config", "D", "--steps", "2", "--warmup", "1", "--no-compare", "--no-cpu-baseline",
+           "--dist-backend", "gloo"]
+    out = subprocess.run(cmd, capture_output=True, text=True, timeout=840, cwd=ROOT)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, out.stdout
+    rec = json.loads(lines[0])
+    assert rec["n_gpus"] == 2 and rec["value"] > 0 and "shrunk" not in rec["metric"]
+    assert rec["config"]["payload_bytes_per_rank"] > 30e9
+    assert [p["rank"] for p in rec["placement"]] == [0, 1]
+    assert len(rec["measured_ce_GBps_all_ranks"]) == 2
+    assert rec["topology"]["numa_nodes"] and rec["clocks"]["samples"] > 0
+    lo, hi = rec["swap_in_latency_s_range"]
+    assert lo <= rec["swap_in_latency_s"] <= hi
