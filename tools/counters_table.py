@@ -3,6 +3,7 @@
 counters per payload byte (PCIe read/write, DRAM read/write) and the range's rates.
 
     python tools/counters_table.py gpurun_out/counters.csv gpurun_out/counter_cases.json > profiles/rNN_counters_crossover.md
+    python tools/counters_table.py gpurun_out/counters_tma.csv probe_tma     # tools/probe_tma ranges (1 GiB each)
 """
 import csv
 import json
@@ -30,7 +31,12 @@ def load(csv_path, cases_path):
         elif unit == "Gbyte":
             v *= 1e9
         by.setdefault(int(d["ID"]), {})[d["Metric Name"]] = v
-    cases = json.load(open(cases_path))
+    if cases_path == "probe_tma":
+        names = ["ce_h2d", "ce_d2h", "ldg_h2d", "stg_d2h", "tma_h2d", "tma_d2h"]
+        cases = [{"mechanism": nm, "chunk": 0, "phase": "h2d" if "h2d" in nm else "d2h", "payload": 1 << 30}
+                 for nm in names]
+    else:
+        cases = json.load(open(cases_path))
     assert len(cases) == len(by), (len(cases), len(by))
     return [dict(c, **by[i]) for i, c in enumerate(cases)]
 

@@ -4,6 +4,8 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstdint>
+#include <cstring>
+#include <cuda_profiler_api.h>
 #include <cuda_runtime.h>
 
 #define CK(x) do { cudaError_t e = (x); if (e != cudaSuccess) { \
@@ -98,7 +100,40 @@ template <int ST> void L_tma(const char* s, char* d, size_t n, cudaStream_t st) 
   tma_copy<ST><<<g_grid, 32, sm, st>>>(s, d, n, g_tile);
 }
 
-int main() {
+// `probe_tma ranges`: one CE / LDG / TMA transfer of 1 GiB per direction, each in its own
+// cudaProfilerStart/Stop range, for ncu --replay-mode app-range PCIe counters (profiles/r02_counters_crossover.md).
+static int ranges_main() {
+  const size_t n = 1ull << 30;
+  cudaDeviceProp p; CK(cudaGetDeviceProperties(&p, 0));
+  char *h, *d;
+  CK(cudaHostAlloc((void**)&h, n, cudaHostAllocMapped));
+  CK(cudaMalloc(&d, n));
+  CK(cudaMemset(d, 3, n)); memset(h, 5, n);
+  cudaStream_t s; CK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  g_grid = p.multiProcessorCount; g_tile = 16384;
+  const char* names[6] = {"ce_h2d", "ce_d2h", "ldg_h2d", "stg_d2h", "tma_h2d", "tma_d2h"};
+  for (int c = 0; c < 6; ++c) {
+    for (int rep = 0; rep < 2; ++rep) {  // rep 0 warms up (attributes, first launch), rep 1 is profiled
+      CK(cudaStreamSynchronize(s));
+      if (rep) CK(cudaProfilerStart());
+      switch (c) {
+        case 0: CK(cudaMemcpyAsync(d, h, n, cudaMemcpyHostToDevice, s)); break;
+        case 1: CK(cudaMemcpyAsync(h, d, n, cudaMemcpyDeviceToHost, s)); break;
+        case 2: L_ldg<8, 0>(h, d, n, s); break;
+        case 3: L_ldg<8, 0>(d, h, n, s); break;
+        case 4: L_tma<4>(h, d, n, s); break;
+        case 5: L_tma<4>(d, h, n, s); break;
+      }
+      CK(cudaStreamSynchronize(s));
+      if (rep) CK(cudaProfilerStop());
+    }
+    printf("range %d %s %zu\n", c, names[c], n);
+  }
+  return 0;
+}
+
+int main(int argc, char** argv) {
+  if (argc > 1 && !strcmp(argv[1], "ranges")) return ranges_main();
   size_t n = 4ull << 30;
   cudaDeviceProp p; CK(cudaGetDeviceProperties(&p, 0));
   g_sms = p.multiProcessorCount;
