@@ -81,6 +81,7 @@ def parse():
     ap.add_argument("--no-compare", action="store_true", help="skip the other-mechanism comparison")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-assisted", action="store_true", help="skip the N>1 NVLink-assisted restore leg")
+    ap.add_argument("--no-dp", action="store_true", help="skip the N>1 data-parallel replica leg")
     ap.add_argument("--sample-bytes", type=int, default=8 << 30, help="oracle sample size per step")
     ap.add_argument("--allow-kv-shrink", action="store_true",
                     help="if host RAM cannot hold every rank's image, shrink the KV pool (the line then names a "
@@ -664,6 +665,59 @@ def run_ours(args):
     numa = sw.numa()
     placement = gather_obj({"rank": rank, "gpu": local_dev, "gpu_numa_node": node, "cpus": len(my_cpus),
                             "image_numa_node": numa["node"], "image_local_fraction": numa["local_fraction"]})
+    sw.close()
+    vmm.close()
+    del arena
+
+    # NEXT-2, data-parallel replicas (outside the timed region): every rank holds a replica of rank 0's
+    # engine image; striped swap-in (each replica pulls 1/N over its own link, stripes broadcast over
+    # NVLink, HBM verify of everything) vs every replica pulling the whole image over its own link
+    dp = None
+    if world > 1 and args.dist_backend == "nccl" and ndev > 1 and not args.no_dp:
+        _, specs0, _ = workload(args.config, 0, world)
+        offs0, bytes0 = W.place(specs0)
+        arena0 = torch.empty(bytes0, dtype=torch.uint8, device=dev)
+        W.fill_device_arena(arena0, specs0, offs0, seed=0)  # identical bytes on every replica
+        regions0 = [(arena0.data_ptr() + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs0, offs0))]
+        payload0 = sum(r.nbytes for r in specs0)
+        with swap.Swapper(regions0, chunk_bytes=args.chunk, checksum=kind, mechanism="ce_pipe",
+                          device=local_dev) as swd, torch.cuda.stream(stream):
+            swd.checkpoint(stream, sync=True)
+
+            def poison0():
+                for r, o in zip(specs0, offs0):
+                    if r.nbytes:
+                        arena0[o:o + r.nbytes].fill_(W.POISON_BYTE)
+                stream.synchronize()
+
+            def timed(fn):
+                ts = []
+                for _ in range(3):
+                    poison0()
+                    barrier()
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record(stream)
+                    res = fn()
+                    e1.record(stream)
+                    e1.synchronize()
+                    assert res["status"] == 0 and res["n_bad"] == 0 and res["hbm_n_bad"] == 0, res
+                    ts.append(e0.elapsed_time(e1) * 1e-3)
+                return statistics.median(allreduce(ts, tdist.ReduceOp.MAX)[1:])
+
+            t_striped = timed(lambda: sdist.restore_replicas(swd, None, stream))
+
+            def independent():
+                swd.restore(stream)
+                return swd.verify(stream, hbm_pass=True)
+
+            t_indep = timed(independent)
+        del arena0
+        dp = {"replicas": world, "image_bytes": payload0, "striped_swap_in_s": round(t_striped, 4),
+              "independent_swap_in_s": round(t_indep, 4), "speedup": round(t_indep / t_striped, 3),
+              "striped_GBps_per_replica": round(payload0 / t_striped / GB, 2),
+              "host_link_bytes_per_replica": payload0 // world,
+              "how": "swap_restore_stripe (1/N of the CE_PIPE groups per replica over its own PCIe link) + in-place "
+                     "NCCL broadcasts of every stripe span from its owner + HBM verify of all chunks, max over ranks"}
     if rank == 0:
         value = total_payload / (swapin_ms * 1e-3) / GB
         achieved = payload / (restore_ms * 1e-3) / GB
@@ -705,6 +759,7 @@ def run_ours(args):
             "mechanisms": compare,
             "fused_checksum_overhead": overhead(compare, achieved, ce),
             "assisted_swap_in": assisted,
+            "dp_replicas": dp,
             "setup_s": {"fill": round(t_fill, 2), "register_pin": round(t_register, 2)},
             "swap_in_with_hbm_reacquire_s": round(statistics.mean(x[1] for x in reacq), 4),
             "hbm_reacquire_s": round(statistics.mean(x[0] for x in reacq), 4),
@@ -727,8 +782,6 @@ def run_ours(args):
         if args.out:
             with open(args.out, "a") as f:
                 f.write(s + "\n")
-    sw.close()
-    vmm.close()
     if world > 1:
         tdist.barrier()
         tdist.destroy_process_group()

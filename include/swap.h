@@ -205,6 +205,30 @@ SWAP_API swap_status swap_get_mechanism(const swap_ctx_t* ctx, uint32_t* effecti
  * (AUTO resolves per direction, so the two can differ; REGISTERED+; EINVAL for another direction). */
 SWAP_API swap_status swap_get_mechanism_dir(const swap_ctx_t* ctx, int direction, uint32_t* effective);
 
+/* Data-parallel replicas (NEXT-2, "swap-in time depends on the GPU memory utilized", P:L230 one
+ * backend per GPU set): k replicas hold the same engine image, each in its own ctx/process. Instead of
+ * every replica pulling the whole image over its own PCIe link, replica r restores only the copy-engine
+ * restore groups g with g % n_stripes == stripe (copy engine H2D + the fused per-group hash check, as
+ * SWAP_MECH_CE_PIPE does), and the replicas then exchange their stripes over NVLink (the caller's
+ * collective: dist.restore_replicas broadcasts each span from its owner with NCCL). Until that exchange
+ * the other stripes' bytes on this device are stale; swap_verify(hbm_pass = 1) afterwards checks every
+ * chunk against this ctx's manifest. Zero chunks (DISCARD, masks) are zero-filled in full on every replica.
+ * n_stripes == 1 is swap_restore with CE_PIPE. EINVAL: stripe >= n_stripes, or helper devices are set.
+ * State as swap_restore (-> RESTORED). */
+SWAP_API swap_status swap_restore_stripe(swap_ctx_t* ctx, uint32_t stripe, uint32_t n_stripes, swap_stream_t stream);
+
+/* One coalesced copy of a restore group: `bytes` at device address dev_addr <- image[image_offset ..). */
+typedef struct {
+  uint32_t group;        /* restore group index (the striping unit of swap_restore_stripe) */
+  uint32_t reserved;     /* 0 */
+  uint64_t dev_addr;
+  uint64_t image_offset;
+  uint64_t bytes;
+} swap_span_t;
+/* The restore spans in group order (REGISTERED+). Writes min(cap, total) spans to out (out may be NULL
+ * when cap == 0) and the total count to *n. Replicas with the same region layout get the same list. */
+SWAP_API swap_status swap_get_restore_spans(const swap_ctx_t* ctx, swap_span_t* out, size_t cap, size_t* n);
+
 /* Borrowed views, valid until swap_destroy. The manifest is final only after swap_sync.
  * The image is writable: a caller may load a stored image into it and call swap_import. */
 SWAP_API swap_status swap_get_manifest(const swap_ctx_t* ctx, const void** bytes, size_t* n);

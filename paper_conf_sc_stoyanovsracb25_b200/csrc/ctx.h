@@ -99,6 +99,7 @@ struct swap_ctx {
     cudaEvent_t ev = nullptr, done = nullptr;
   };
   std::vector<Helper> helpers;
+  uint32_t stripe = 0, n_stripes = 1;  // CE_PIPE restore groups this restore moves (swap_restore_stripe)
   int numa_node = -1;         // NUMA node the image placement targeted (-1: none)
   double numa_local = 1.0;    // sampled share of image pages on numa_node
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
@@ -124,6 +125,7 @@ swap_status launch(swap_ctx* c, int mode, int kind, const swk::Params& p, cudaSt
 swap_status memcpy_dir(swap_ctx* c, const Span& sp, int dir, cudaStream_t s);
 swap_status ce_copy(swap_ctx* c, DescSet& S, int dir, cudaStream_t s);
 swap_status copy_spans(swap_ctx* c, const std::vector<Span>& spans, int dir, cudaStream_t s);
+std::vector<Span> coalesce(const std::vector<Span>& spans);
 swap_status map_spans(swap_ctx* c, const std::vector<Span>& spans);
 swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, cudaStream_t s);
 swap_status collect_timing(swap_ctx* c, int p);

@@ -182,6 +182,7 @@ swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, c
   for (size_t g = 0; g < S.groups.size(); ++g) {
     const Group& G = S.groups[g];
     if (dir == 1 && (st = map_spans(c, G.spans)) != SWAP_OK) return st;  // lazy HBM re-acquire
+    if (dir == 1 && c->n_stripes > 1 && g % c->n_stripes != c->stripe) continue;  // another replica's stripe
     const size_t k = H ? g % (H + 1) : 0;
     if (k > 0) {
       // helper k-1: H2D of the group's image range into its staging over its own PCIe link, then

@@ -285,8 +285,9 @@ swap_status swap_sync(swap_ctx_t* c, swap_stream_t stream) {
   return SWAP_OK;
 }
 
-swap_status swap_restore(swap_ctx_t* c, swap_stream_t stream) {
-  if (!c) return SWAP_EINVAL;
+// The restore (swap_restore), or with n_stripes > 1 only the CE_PIPE groups g with g % n_stripes == stripe
+// (swap_restore_stripe: DP replicas each pull one stripe over their own link, NEXT-2).
+static swap_status restore_impl(swap_ctx* c, swap_stream_t stream, uint32_t stripe, uint32_t n_stripes) {
   if (c->st != St::CHECKPOINTED && c->st != St::RESTORED) {
     c->err = "restore needs a completed checkpoint (swap_sync) or an imported image";
     return SWAP_ESTATE;
@@ -295,7 +296,9 @@ swap_status swap_restore(swap_ctx_t* c, swap_stream_t stream) {
   if (st != SWAP_OK) return st;
   DeviceGuard g(c->cfg.device);
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
-  c->cur_mech = resolve_mech(c, 1);
+  c->cur_mech = n_stripes > 1 ? (uint32_t)SWAP_MECH_CE_PIPE : resolve_mech(c, 1);
+  c->stripe = stripe;
+  c->n_stripes = n_stripes;
   DescSet& S = c->s_move;
   swk::Params p = base_params(c, S);
   CUDA_TRY(c, cudaMemsetAsync(&c->d_status->n_bad, 0, 8, s));
@@ -319,7 +322,10 @@ swap_status swap_restore(swap_ctx_t* c, swap_stream_t stream) {
   }
   if ((st = zero_fill_device(c, zs)) != SWAP_OK) return st;
   if (mech(c) == SWAP_MECH_CE_PIPE) {
-    if ((st = ce_pipe(c, S, 1, p, s)) != SWAP_OK) return st;
+    st = ce_pipe(c, S, 1, p, s);
+    c->stripe = 0;
+    c->n_stripes = 1;
+    if (st != SWAP_OK) return st;
   } else if (is_ce(mech(c))) {
     if ((st = ce_copy(c, S, 1, s)) != SWAP_OK) return st;
     if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, s)) != SWAP_OK) return st;
@@ -329,6 +335,34 @@ swap_status swap_restore(swap_ctx_t* c, swap_stream_t stream) {
   CUDA_TRY(c, cudaEventRecord(c->ev[3], s));
   c->pending[1] = true;
   c->st = St::RESTORED;
+  return SWAP_OK;
+}
+
+swap_status swap_restore(swap_ctx_t* c, swap_stream_t stream) {
+  if (!c) return SWAP_EINVAL;
+  return restore_impl(c, stream, 0, 1);
+}
+
+swap_status swap_restore_stripe(swap_ctx_t* c, uint32_t stripe, uint32_t n_stripes, swap_stream_t stream) {
+  if (!c || n_stripes == 0 || stripe >= n_stripes) return SWAP_EINVAL;
+  if (n_stripes > 1 && !c->helpers.empty()) {
+    c->err = "stripe restores and helper devices do not combine";
+    return SWAP_EINVAL;
+  }
+  return restore_impl(c, stream, stripe, n_stripes);
+}
+
+swap_status swap_get_restore_spans(const swap_ctx_t* c, swap_span_t* out, size_t cap, size_t* n) {
+  if (!c || !n || (cap && !out)) return SWAP_EINVAL;
+  if (c->st == St::CREATED) return SWAP_ESTATE;
+  size_t k = 0;
+  const DescSet& S = c->s_move;
+  for (size_t g = 0; g < S.groups.size(); ++g)
+    for (const Span& sp : coalesce(S.groups[g].spans)) {
+      if (k < cap) out[k] = swap_span_t{(uint32_t)g, 0u, sp.dev, (uint64_t)(sp.host - c->image), sp.bytes};
+      ++k;
+    }
+  *n = k;
   return SWAP_OK;
 }
 

@@ -9,6 +9,10 @@ only exchanges are
       engine API is active").
 Both go through torch.distributed (NCCL over NVLink on the GPU box; gloo in CPU tests).
 Validation and the digest run in libswap (swap_set_global / swap_merge_global).
+
+Data-parallel replicas (NEXT-2) are the one place payload crosses NVLink: restore_replicas pulls
+1/k of the image per replica over its own PCIe link (swap_restore_stripe) and broadcasts each
+replica's stripe to the others in place, then every replica runs the HBM verify pass.
 """
 from __future__ import annotations
 
@@ -48,6 +52,39 @@ def gather_manifest(sw: Swapper, group=None) -> tuple[bytes, int]:
     """After a checkpoint on every rank: all-gather summaries, install them in the ctx."""
     allb = all_gather_summaries(sw.summary(), group)
     return allb, sw.set_global(allb)
+
+
+class _DeviceBytes:
+    """A raw device range as a uint8 tensor (zero-copy, __cuda_array_interface__)."""
+
+    def __init__(self, ptr: int, nbytes: int):
+        self.__cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (ptr, False),
+                                         "version": 3, "strides": None}
+
+
+def device_view(ptr: int, nbytes: int, device: int) -> torch.Tensor:
+    return torch.as_tensor(_DeviceBytes(ptr, nbytes), device=torch.device("cuda", device))
+
+
+def restore_replicas(sw: Swapper, group=None, stream=None) -> dict:
+    """Swap-in of k data-parallel replicas of one engine image (NEXT-2; PAPER.md L203 latency grows with
+    the bytes moved, L230 one backend per GPU set). Replica r = rank r of `group`: swap_restore_stripe
+    moves groups g = r (mod k) from its pinned image over its own PCIe link (with the fused per-group
+    check); then, in group order, the owner of every restore span broadcasts it in place to the other
+    replicas (NCCL over NVLink on the GPU box); finally every replica verifies all chunks from HBM.
+    Returns the verify result (swap_verify with the HBM pass) of this replica."""
+    k, r = dist.get_world_size(group), dist.get_rank(group)
+    s = stream if stream is not None else torch.cuda.current_stream(sw.device)
+    with torch.cuda.stream(s):
+        sw.restore_stripe(r, k, s)
+        spans = sw.restore_spans()
+        # collectives are issued on `s`, after the stripe's copies; each span comes from its owner
+        works = [dist.broadcast(device_view(dev, nb, sw.device), src=dist.get_global_rank(group, g % k) if group else g % k,
+                                group=group, async_op=True)
+                 for (g, dev, _, nb) in spans]
+        for w in works:
+            w.wait()
+        return sw.verify(s, hbm_pass=True, raise_on_corrupt=False)
 
 
 def agree_restore(verify_result: dict, group=None) -> int:

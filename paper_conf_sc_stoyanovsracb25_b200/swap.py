@@ -30,7 +30,7 @@ U64_MAX = (1 << 64) - 1
 
 EXPORTS = [
     "swap_config_default", "swap_create", "swap_register_regions", "swap_checkpoint", "swap_sync",
-    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_get_mechanism_dir", "swap_get_numa", "swap_set_region_policy", "swap_set_chunk_mask", "swap_get_manifest", "swap_get_image",
+    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_get_mechanism_dir", "swap_get_numa", "swap_restore_stripe", "swap_get_restore_spans", "swap_set_region_policy", "swap_set_chunk_mask", "swap_get_manifest", "swap_get_image",
     "swap_get_summary", "swap_import", "swap_save", "swap_load", "swap_set_global", "swap_merge_global", "swap_plan_layout", "swap_plan_manifest", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
     "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
@@ -60,6 +60,11 @@ class swap_verify_result_t(ctypes.Structure):
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class swap_span_t(ctypes.Structure):
+    _fields_ = [("group", ctypes.c_uint32), ("reserved", ctypes.c_uint32), ("dev_addr", ctypes.c_uint64),
+                ("image_offset", ctypes.c_uint64), ("bytes", ctypes.c_uint64)]
 
 
 class swap_shard_summary_t(ctypes.Structure):
@@ -107,6 +112,8 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_get_mechanism": (st, [vp, P(u32)]),
         "swap_get_mechanism_dir": (st, [vp, ctypes.c_int, P(u32)]),
         "swap_get_numa": (st, [vp, P(ctypes.c_int32), P(ctypes.c_double)]),
+        "swap_restore_stripe": (st, [vp, u32, u32, vp]),
+        "swap_get_restore_spans": (st, [vp, vp, ctypes.c_size_t, P(ctypes.c_size_t)]),
         "swap_set_region_policy": (st, [vp, u32, u32]),
         "swap_set_chunk_mask": (st, [vp, u32, vp, ctypes.c_uint64]),
         "swap_get_manifest": (st, [vp, P(vp), P(sz)]),
@@ -399,6 +406,18 @@ class Swapper:
         p, n = ctypes.c_void_p(), ctypes.c_size_t()
         self._check(load().swap_get_manifest(self._ctx, ctypes.byref(p), ctypes.byref(n)))
         return np.ctypeslib.as_array(ctypes.cast(p, ctypes.POINTER(ctypes.c_uint8)), shape=(n.value,))
+
+    def restore_stripe(self, stripe: int, n_stripes: int, stream=None):
+        """Restore only CE_PIPE groups g with g % n_stripes == stripe (swap_restore_stripe; DP replicas)."""
+        self._check(load().swap_restore_stripe(self._ctx, stripe, n_stripes, _torch_stream(stream)))
+
+    def restore_spans(self) -> list[tuple[int, int, int, int]]:
+        """(group, dev_addr, image_offset, bytes) of every coalesced restore copy (swap_get_restore_spans)."""
+        n = ctypes.c_size_t()
+        self._check(load().swap_get_restore_spans(self._ctx, None, 0, ctypes.byref(n)))
+        arr = (swap_span_t * max(1, n.value))()
+        self._check(load().swap_get_restore_spans(self._ctx, arr, n.value, ctypes.byref(n)))
+        return [(x.group, x.dev_addr, x.image_offset, x.bytes) for x in arr[:n.value]]
 
     def numa(self) -> dict:
         """Host NUMA placement of the image (swap_get_numa): the node targeted (-1 none) and the

@@ -1,6 +1,5 @@
 cd "${GRAFT_REPO_ROOT:-.}"; mkdir -p gpurun_out
-timeout 600 ncu --replay-mode app-range --metrics pcie__read_bytes.sum,pcie__write_bytes.sum,dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum \
-  --csv --log-file gpurun_out/counters_tma.csv tools/probe_tma ranges > gpurun_out/counters_tma.log 2>&1; echo "tma rc=$?"; cat gpurun_out/counters_tma.log | tail -8
-timeout 1200 ncu --replay-mode app-range --metrics pcie__read_bytes.sum,pcie__write_bytes.sum,dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum \
-  --csv --log-file gpurun_out/counters8.csv python tools/counters.py --gib 8 --chunks 1048576,16777216 --cases-out gpurun_out/counter_cases8.json > gpurun_out/counters8.log 2>&1
-echo "counters8 rc=$?"
+timeout 600 python -m pytest tests/test_gpu_dp_replicas.py -q -x --timeout 300 2>&1 | tail -15
+timeout 2400 python -m pytest tests -m gpu -q --timeout 900 > gpurun_out/pytest_gpu_r02.log 2>&1; echo "tests rc=$?"; tail -5 gpurun_out/pytest_gpu_r02.log
+timeout 300 python __graft_entry__.py smoke 2>&1 | tail -2
+timeout 900 python bench.py --checksum xxh64 --no-compare > gpurun_out/bench_B_xxh64_r02.log 2>&1; echo "bench rc=$?"; tail -1 gpurun_out/bench_B_xxh64_r02.log | cut -c1-300
