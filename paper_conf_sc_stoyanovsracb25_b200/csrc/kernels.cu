@@ -94,6 +94,12 @@ void build_tables(uint32_t* tab, uint64_t L1, uint64_t seg) {
       for (int z = 0; z < 96; ++z) r = t[r & 0xFFu] ^ (r >> 8);
       tab[TAB_Z96N + kk * 16 + v] = r;
     }
+  for (int kk = 0; kk < 4; ++kk)  // Z^96 of byte e at byte position kk
+    for (uint32_t e = 0; e < 256; ++e) {
+      uint32_t r = e << (8 * kk);
+      for (int z = 0; z < 96; ++z) r = t[r & 0xFFu] ^ (r >> 8);
+      tab[TAB_Z96B + kk * 256 + e] = r;
+    }
 }
 
 // ------------------------------------------------------------------ device helpers
@@ -501,16 +507,25 @@ __global__ void __launch_bounds__(THREADS, 2) mover_kernel(const Params p) {
 // wavefronts (the r1 contiguous-run layout needed 32 + 32).
 constexpr int HT_THREADS = 1024;
 constexpr int HT_WARPS = HT_THREADS / 32;
-constexpr int HT_U = 4;  // lines in flight per lane
-// Shared layout (offsets from a 32-KiB-aligned base B inside the dynamic allocation): slicing table k at
-// B + k*32 KiB, entry e of lane l at + e*128 + l*4; Z^96 nibble table k at B + 128 KiB + k*2 KiB. With
-// B 32-KiB aligned, a lookup address is (index << 7) | (B + 4*lane) plus an immediate table offset: one
-// shift + one LOP3 per lookup.
+// Shared layout, in absolute shared-window addresses. Dynamic shared memory starts at 0x400 on sm_100 (the
+// first KiB of the CTA window is reserved; tools/probe_smem_base.cu measures it) and the kernel traps if it
+// does not, so the tables' alignment costs no padding: descriptors + mbarriers at 0x400, the Z^96 nibble
+// tables at 0x1000 (8 x 16 entries x 32 lanes, 16 KiB, 2-KiB aligned), the four slicing tables at 0x8000
+// (table k at 0x8000 + k*32 KiB, entry e of lane l at + e*128 + l*4: 32-KiB aligned, so a lookup address
+// is (index << 7) | (0x8000 + 4*lane) plus an immediate table offset: one shift + one LOP3). Variant ZB
+// adds Z^96 *byte* tables at 0x28000 (4 x 256 entries x 16 copies, lanes l and l+16 share copy l&15:
+// entry e of copy c at word e*16 + c, 16-KiB aligned) and drops the nibble tables.
+constexpr uint32_t HT_SMEM_BASE = 0x400;
+constexpr uint32_t HT_A_DESC = 0x400;
+constexpr uint32_t HT_A_BAR = HT_A_DESC + 2 * HT_WARPS * 32;  // 2 rounds x 32 descriptors x 32 B
+constexpr uint32_t HT_A_ZN = 0x1000;
+constexpr uint32_t HT_A_TAB = 0x8000;
 constexpr uint32_t HT_TAB_BYTES = 4 * 256 * 128;
-constexpr uint32_t HT_Z_BYTES = 8 * 16 * 128;
-constexpr uint32_t HT_OFF_DESC = HT_TAB_BYTES + HT_Z_BYTES;
-constexpr uint32_t HT_OFF_BAR = HT_OFF_DESC + 2 * HT_WARPS * sizeof(SegDesc);
-constexpr size_t HT_SMEM = 32768 + HT_OFF_BAR + 16;  // + worst-case alignment padding
+constexpr uint32_t HT_A_ZB = HT_A_TAB + HT_TAB_BYTES;          // 0x28000
+constexpr uint32_t HT_ZB_BYTES = 4 * 256 * 16 * 4;              // 64 KiB
+template <bool ZB>
+constexpr size_t ht_smem() { return (ZB ? HT_A_ZB + HT_ZB_BYTES : HT_A_TAB + HT_TAB_BYTES) - HT_SMEM_BASE; }
+static_assert(HT_A_BAR + 16 <= HT_A_ZN && HT_A_ZN + 8 * 16 * 128 <= HT_A_TAB, "hash kernel shared layout");
 
 __device__ __forceinline__ void ld32(const uint8_t* p, uint32_t (&w)[8]) {
   asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
@@ -560,32 +575,45 @@ __device__ __forceinline__ uint32_t lds_off(uint32_t addr) {
 // busy); moving one address per word to the FMA pipe measured +6 % (interleaved A/B on config B; the
 // other splits tried — bytes 1-3 or all four via IMAD/IMAD.HI, byte-permute addressing with 64-KiB
 // table pairs — were slower: IMAD.HI and PRMT cost two ALU-equivalent issue slots).
+template <bool B0F>
 __device__ __forceinline__ uint32_t crc_word4(uint32_t c, uint32_t w, uint32_t lb, uint32_t m128) {
   c ^= w;
-  return lds_off<3 * 32768>(((c << 7) & 0x7F80u) | lb) ^ lds_off<2 * 32768>(((c >> 1) & 0x7F80u) | lb) ^
+  // B0F: byte 0's shift by 7 as an IMAD by the opaque 128 (FMA pipe, idle in this kernel) instead of a SHF
+  const uint32_t s0 = B0F ? c * m128 : c << 7;
+  return lds_off<3 * 32768>((s0 & 0x7F80u) | lb) ^ lds_off<2 * 32768>(((c >> 1) & 0x7F80u) | lb) ^
          lds_off<1 * 32768>(((c >> 9) & 0x7F80u) | lb) ^ lds_off<0>((c >> 24) * m128 + lb);
 }
-// Z^96(T) from 8 nibble lookups; lz = B + 128K + 4*lane: nibble table k entry v at lz + k*2K + v*128
-__device__ __forceinline__ uint32_t z96(uint32_t T, uint32_t lz) {
-  return lds_off<0 * 2048>(((T << 7) & 0x780u) | lz) ^ lds_off<1 * 2048>(((T << 3) & 0x780u) | lz) ^
+// Z^96(T) from 8 nibble lookups; lz = 0x1000 + 4*lane: nibble table k entry v at lz + k*2K + v*128
+template <bool B0F>
+__device__ __forceinline__ uint32_t z96(uint32_t T, uint32_t lz, uint32_t m128) {
+  const uint32_t s0 = B0F ? T * m128 : T << 7;
+  const uint32_t a7 = B0F ? (T >> 28) * m128 + lz : ((T >> 21) & 0x780u) | lz;
+  return lds_off<0 * 2048>((s0 & 0x780u) | lz) ^ lds_off<1 * 2048>(((T << 3) & 0x780u) | lz) ^
          lds_off<2 * 2048>(((T >> 1) & 0x780u) | lz) ^ lds_off<3 * 2048>(((T >> 5) & 0x780u) | lz) ^
          lds_off<4 * 2048>(((T >> 9) & 0x780u) | lz) ^ lds_off<5 * 2048>(((T >> 13) & 0x780u) | lz) ^
-         lds_off<6 * 2048>(((T >> 17) & 0x780u) | lz) ^ lds_off<7 * 2048>(((T >> 21) & 0x780u) | lz);
+         lds_off<6 * 2048>(((T >> 17) & 0x780u) | lz) ^ lds_off<7 * 2048>(a7);
+}
+// Z^96(T) from 4 byte lookups; lzb = 0x28000 + 4*(lane & 15): byte table k entry e at lzb + k*16K + e*64
+// (lanes l and l+16 share a copy: they meet in a bank only when their entries have equal parity)
+__device__ __forceinline__ uint32_t z96b(uint32_t T, uint32_t lzb, uint32_t m64) {
+  return lds_off<0 * 16384>(((T << 6) & 0x3FC0u) | lzb) ^ lds_off<1 * 16384>(((T >> 2) & 0x3FC0u) | lzb) ^
+         lds_off<2 * 16384>(((T >> 10) & 0x3FC0u) | lzb) ^ lds_off<3 * 16384>((T >> 24) * m64 + lzb);
 }
 
 // One 32-B piece: advance the register across the 96-B gap, then through the piece's 8 words.
+template <bool ZB, bool B0F>
 __device__ __forceinline__ uint32_t crc_piece32(uint32_t c, const uint32_t (&w)[8], uint32_t lb, uint32_t lz,
                                                 uint32_t m128) {
-  c = z96(c, lz);
+  c = ZB ? z96b(c, lz, m128 >> 1) : z96<B0F>(c, lz, m128);
 #pragma unroll
-  for (int j = 0; j < 8; ++j) c = crc_word4(c, w[j], lb, m128);
+  for (int j = 0; j < 8; ++j) c = crc_word4<B0F>(c, w[j], lb, m128);
   return c;
 }
 
 // Register of one lane over its pieces s0, s0+128, ... < send (send = min(strand end, len)).
 // A 4-deep software pipeline: each 256-bit load is consumed one loop iteration after it is issued,
 // so ptxas cannot sink it next to its use and four loads per lane stay in flight.
-template <bool AL32>
+template <bool AL32, bool ZB, bool B0F>
 __device__ __forceinline__ uint32_t lane_pieces_crc(const uint8_t* src, uint64_t s0, uint64_t send, uint32_t lb,
                                                     uint32_t lz, uint32_t m128) {
   uint32_t c = 0;
@@ -599,51 +627,68 @@ __device__ __forceinline__ uint32_t lane_pieces_crc(const uint8_t* src, uint64_t
     ld32a<AL32>(src + s0 + 384, e);
     for (; t + 8 <= n; t += 4) {
       const uint8_t* q = src + s0 + (t + 4) * 128;
-      c = crc_piece32(c, a, lb, lz, m128);
+      c = crc_piece32<ZB, B0F>(c, a, lb, lz, m128);
       ld32a<AL32>(q, a);
-      c = crc_piece32(c, b, lb, lz, m128);
+      c = crc_piece32<ZB, B0F>(c, b, lb, lz, m128);
       ld32a<AL32>(q + 128, b);
-      c = crc_piece32(c, d, lb, lz, m128);
+      c = crc_piece32<ZB, B0F>(c, d, lb, lz, m128);
       ld32a<AL32>(q + 256, d);
-      c = crc_piece32(c, e, lb, lz, m128);
+      c = crc_piece32<ZB, B0F>(c, e, lb, lz, m128);
       ld32a<AL32>(q + 384, e);
     }
-    c = crc_piece32(c, a, lb, lz, m128);
-    c = crc_piece32(c, b, lb, lz, m128);
-    c = crc_piece32(c, d, lb, lz, m128);
-    c = crc_piece32(c, e, lb, lz, m128);
+    c = crc_piece32<ZB, B0F>(c, a, lb, lz, m128);
+    c = crc_piece32<ZB, B0F>(c, b, lb, lz, m128);
+    c = crc_piece32<ZB, B0F>(c, d, lb, lz, m128);
+    c = crc_piece32<ZB, B0F>(c, e, lb, lz, m128);
     t += 4;
   }
   for (; t < n; ++t) {
     uint32_t w[8];
     ld32a<AL32>(src + s0 + t * 128, w);
-    c = crc_piece32(c, w, lb, lz, m128);
+    c = crc_piece32<ZB, B0F>(c, w, lb, lz, m128);
   }
   uint64_t s = s0 + n * 128;
   if (s < send) {  // a partial last piece (only at the end of the segment)
-    c = z96(c, lz);
+    c = ZB ? z96b(c, lz, m128 >> 1) : z96<B0F>(c, lz, m128);
     for (; s < send; ++s) c = lds_at((((c ^ src[s]) & 0xFFu) << 7) | lb) ^ (c >> 8);  // table 0 = one byte
   }
   return c;
 }
 
-template <int MODE>
+template <int MODE, bool ZB, bool B0F>
 __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
-  const uint32_t B = (raw + 32767u) & ~32767u;  // 32-KiB aligned table base (shared address)
-  uint8_t* smem = smem_raw + (B - raw);
-  uint32_t* sT = reinterpret_cast<uint32_t*>(smem);
-  SegDesc* sDesc = reinterpret_cast<SegDesc*>(smem + HT_OFF_DESC);
-  uint64_t* sBar = reinterpret_cast<uint64_t*>(smem + HT_OFF_BAR);
+  if (raw != HT_SMEM_BASE) __trap();  // the layout below assumes dynamic shared memory at 0x400
+  uint8_t* smem = smem_raw - HT_SMEM_BASE;  // generic pointer of shared address 0
+  uint32_t* sT = reinterpret_cast<uint32_t*>(smem + HT_A_TAB);
+  SegDesc* sDesc = reinterpret_cast<SegDesc*>(smem + HT_A_DESC);
+  uint64_t* sBar = reinterpret_cast<uint64_t*>(smem + HT_A_BAR);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 
-  // replicate T0..T3 (the first four slicing tables) and the Z^96 nibble table once per lane
-  for (int i = tid; i < 4 * 256 + 8 * 16; i += HT_THREADS) {
-    const uint32_t v = i < 4 * 256 ? __ldg(p.tables + TAB_T16 + i) : __ldg(p.tables + TAB_Z96N + (i - 4 * 256));
-    uint4* dst = reinterpret_cast<uint4*>(sT + (size_t)i * 32);  // the Z table follows the slicing tables
+  // replicate T0..T3 (the first four slicing tables) once per lane, and the Z^96 tables
+  for (int i = tid; i < 4 * 256; i += HT_THREADS) {
+    const uint32_t v = __ldg(p.tables + TAB_T16 + i);
+    uint4* dst = reinterpret_cast<uint4*>(sT + (size_t)i * 32);
 #pragma unroll
     for (int r = 0; r < 8; ++r) dst[r] = make_uint4(v, v, v, v);
+  }
+  if (ZB) {
+    uint32_t* sZ = reinterpret_cast<uint32_t*>(smem + HT_A_ZB);
+    for (int i = tid; i < 4 * 256; i += HT_THREADS) {
+      const uint32_t v = __ldg(p.tables + TAB_Z96B + i);
+      uint4* dst = reinterpret_cast<uint4*>(sZ + (size_t)i * 16);
+#pragma unroll
+      for (int r = 0; r < 4; ++r) dst[r] = make_uint4(v, v, v, v);
+    }
+  } else {
+    uint32_t* sZ = reinterpret_cast<uint32_t*>(smem + HT_A_ZN);
+    for (int i = tid; i < 8 * 16; i += HT_THREADS) {
+      const uint32_t v = __ldg(p.tables + TAB_Z96N + i);
+      uint4* dst = reinterpret_cast<uint4*>(sZ + (size_t)i * 32);
+#pragma unroll
+      for (int r = 0; r < 8; ++r) dst[r] = make_uint4(v, v, v, v);
+    }
   }
   const uint32_t per_round = gridDim.x * HT_WARPS;
   const uint32_t first0 = blockIdx.x * HT_WARPS;
@@ -664,7 +709,8 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
     if (rounds > 1) issue(1);
   }
   __syncthreads();
-  const uint32_t lb = B + 4u * lane, lz = B + HT_TAB_BYTES + 4u * lane;
+  const uint32_t lb = HT_A_TAB + 4u * lane;
+  const uint32_t lz = ZB ? HT_A_ZB + 4u * (lane & 15) : HT_A_ZN + 4u * lane;
   const uint32_t m128 = blockDim.x >> 3;  // = 128 (HT_THREADS = 1024), opaque to ptxas
   const uint32_t* x2n = p.tables + TAB_X2N;
 
@@ -682,8 +728,8 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
       const bool al32 = ((d.dev & 31) == 0);
       uint32_t X = 0;
       if (s0 < send) {
-        const uint32_t c = al32 ? lane_pieces_crc<true>(src, s0, send, lb, lz, m128)
-                                : lane_pieces_crc<false>(src, s0, send, lb, lz, m128);
+        const uint32_t c = al32 ? lane_pieces_crc<true, ZB, B0F>(src, s0, send, lb, lz, m128)
+                                : lane_pieces_crc<false, ZB, B0F>(src, s0, send, lb, lz, m128);
         const uint32_t k = (len == p.hlane_len) ? __ldg(p.tables + TAB_HLANE + lane)
                                                 : x2nmodp(len - hash_lane_end(len, lane), 3, x2n);
         X = multmodp(k, c);
@@ -700,19 +746,35 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
   }
 }
 
-template <int MODE>
-static cudaError_t launch_hash(const Params& p, int grid, cudaStream_t s) {
+template <int MODE, bool ZB, bool B0F>
+static cudaError_t launch_hash_t(const Params& p, int grid, cudaStream_t s) {
   static unsigned long long attr_set = 0;
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
   if (!((attr_set >> (dev & 63)) & 1ull)) {
-    e = cudaFuncSetAttribute(hash_kernel<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)HT_SMEM);
+    e = cudaFuncSetAttribute(hash_kernel<MODE, ZB, B0F>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ht_smem<ZB>());
     if (e != cudaSuccess) return e;
     attr_set |= 1ull << (dev & 63);
   }
-  hash_kernel<MODE><<<grid, HT_THREADS, HT_SMEM, s>>>(p);
+  hash_kernel<MODE, ZB, B0F><<<grid, HT_THREADS, ht_smem<ZB>(), s>>>(p);
   return cudaGetLastError();
+}
+
+// CRC-32C hash-pass variant: b0f (default), or forced with SWAP_CRC_KERNEL (base | b0f | zb | zbb0f) for
+// A/B measurements (read at every launch). In-process on config B (profiles/r02_crc_variants.md): b0f
+// +0.9..1.7 % over base at 4 KiB / 1 MiB / 16 MiB chunks; the Z^96 byte tables (zb) -10 % -- their 2-way
+// conflicts cost more than the 4 lookups they save.
+template <int MODE>
+static cudaError_t launch_hash(const Params& p, int grid, cudaStream_t s) {
+  int v = 1;
+  if (const char* e = getenv("SWAP_CRC_KERNEL")) v = !strcmp(e, "base") ? 0 : !strcmp(e, "zb") ? 2 : !strcmp(e, "zbb0f") ? 3 : 1;
+  switch (v) {
+    case 0: return launch_hash_t<MODE, false, false>(p, grid, s);
+    case 2: return launch_hash_t<MODE, true, false>(p, grid, s);
+    case 3: return launch_hash_t<MODE, true, true>(p, grid, s);
+    default: return launch_hash_t<MODE, false, true>(p, grid, s);
+  }
 }
 
 int hash_grid(int sm_count, uint32_t n_desc) {

@@ -44,7 +44,8 @@ constexpr int TAB_HLANE = TAB_X2N + 32;       // [32] hash kernel: Z^(L1 - end_l
 constexpr int TAB_Z96N = TAB_HLANE + 32;       // [8][16] hash kernel: Z^96 of nibble v at position k
 constexpr int ZS_N = 1024;
 constexpr int TAB_ZS = TAB_Z96N + 128;         // [ZS_N] x^(8*m*seg) mod P: shift by m whole segments
-constexpr int TAB_WORDS = TAB_ZS + ZS_N;
+constexpr int TAB_Z96B = TAB_ZS + ZS_N;        // [4][256] hash kernel (ZB variant): Z^96 of byte e at position k
+constexpr int TAB_WORDS = TAB_Z96B + 4 * 256;
 constexpr int TAB_SMEM_WORDS = TAB_LANE + 32;  // the part staged in shared memory
 
 struct Params {
