@@ -82,6 +82,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-assisted", action="store_true", help="skip the N>1 NVLink-assisted restore leg")
     ap.add_argument("--no-dp", action="store_true", help="skip the N>1 data-parallel replica leg")
+    ap.add_argument("--force-legs", action="store_true",
+                    help="run the N>1 assisted and DP legs even over gloo / on one device (tests: degenerate helpers)")
     ap.add_argument("--sample-bytes", type=int, default=8 << 30, help="oracle sample size per step")
     ap.add_argument("--allow-kv-shrink", action="store_true",
                     help="if host RAM cannot hold every rank's image, shrink the KV pool (the line then names a "
@@ -614,33 +616,41 @@ def run_ours(args):
     # NEXT-2: rank 0's swap-in assisted by k idle peers (their PCIe links into HBM staging, then NVLink),
     # the other ranks idle in a barrier (outside the timed region)
     assisted = None
-    if world > 1 and args.dist_backend == "nccl" and ndev > 1 and not args.no_assisted:
+    multi = world > 1 and ((args.dist_backend == "nccl" and ndev > 1) or args.force_legs)
+    if multi and not args.no_assisted:
         assisted = {}
         for k in (1, 3, 7):
-            if k > ndev - 1:
+            if k > (world - 1 if args.force_legs else min(world, ndev) - 1):  # helpers: the job's own GPUs
                 break
             barrier()
             if rank == 0:
                 helpers = [(local_dev + i) % ndev for i in range(1, k + 1)]
-                sw.set_mechanism("ce_pipe")
-                sw.set_helpers(helpers)
-                ts = []
-                for _ in range(3):
-                    poison()
-                    stream.synchronize()
-                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                    e0.record(stream)
-                    sw.restore(stream)
-                    res = sw.verify(stream, hbm_pass=True)
-                    e1.record(stream)
-                    e1.synchronize()
-                    assert res["status"] == 0 and res["n_bad"] == 0 and res["hbm_n_bad"] == 0, res
-                    ts.append(e0.elapsed_time(e1) * 1e-3)
-                sw.set_helpers([])
-                sw.set_mechanism(args.mechanism)
-                t = statistics.median(ts[1:])
-                assisted[str(k)] = {"helpers": helpers, "swap_in_s": round(t, 4), "GBps": round(payload / t / GB, 2),
-                                    "frac_of_k_plus_1_links": round(payload / t / GB / ((k + 1) * ce["h2d"]), 3)}
+                try:
+                    sw.set_mechanism("ce_pipe")
+                    sw.set_helpers(helpers)
+                    ts = []
+                    for _ in range(3):
+                        poison()
+                        stream.synchronize()
+                        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                        e0.record(stream)
+                        sw.restore(stream)
+                        res = sw.verify(stream, hbm_pass=True)
+                        e1.record(stream)
+                        e1.synchronize()
+                        assert res["status"] == 0 and res["n_bad"] == 0 and res["hbm_n_bad"] == 0, res
+                        ts.append(e0.elapsed_time(e1) * 1e-3)
+                    t = statistics.median(ts[1:])
+                    assisted[str(k)] = {"helpers": helpers, "swap_in_s": round(t, 4), "GBps": round(payload / t / GB, 2),
+                                        "frac_of_k_plus_1_links": round(payload / t / GB / ((k + 1) * ce["h2d"]), 3)}
+                except Exception as ex:  # noqa: BLE001 - an informational leg must not sink the line
+                    assisted[str(k)] = {"helpers": helpers, "error": f"{type(ex).__name__}: {ex}"[:300]}
+                finally:
+                    try:
+                        sw.set_helpers([])
+                        sw.set_mechanism(args.mechanism)
+                    except Exception:  # noqa: BLE001
+                        pass
             barrier()
 
     cpu = None
@@ -673,21 +683,28 @@ def run_ours(args):
     # engine image; striped swap-in (each replica pulls 1/N over its own link, stripes broadcast over
     # NVLink, HBM verify of everything) vs every replica pulling the whole image over its own link
     dp = None
-    if world > 1 and args.dist_backend == "nccl" and ndev > 1 and not args.no_dp:
-        _, specs0, _ = workload(args.config, 0, world)
-        offs0, bytes0 = W.place(specs0)
-        arena0 = torch.empty(bytes0, dtype=torch.uint8, device=dev)
-        W.fill_device_arena(arena0, specs0, offs0, seed=0)  # identical bytes on every replica
-        regions0 = [(arena0.data_ptr() + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs0, offs0))]
-        payload0 = sum(r.nbytes for r in specs0)
-        with swap.Swapper(regions0, chunk_bytes=args.chunk, checksum=kind, mechanism="ce_pipe",
-                          device=local_dev) as swd, torch.cuda.stream(stream):
-            swd.checkpoint(stream, sync=True)
-
+    if multi and not args.no_dp:
+        dp_err, swd, arena0 = "", None, None
+        try:  # local setup first; collectives only if every rank got this far
+            _, specs0, _ = workload(args.config, 0, world)
+            offs0, bytes0 = W.place(specs0)
+            arena0 = torch.empty(bytes0, dtype=torch.uint8, device=dev)
+            W.fill_device_arena(arena0, specs0, offs0, seed=0)  # identical bytes on every replica
+            regions0 = [(arena0.data_ptr() + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs0, offs0))]
+            payload0 = sum(r.nbytes for r in specs0)
+            swd = swap.Swapper(regions0, chunk_bytes=args.chunk, checksum=kind, mechanism="ce_pipe", device=local_dev)
+            with torch.cuda.stream(stream):
+                swd.checkpoint(stream, sync=True)
+        except Exception as ex:  # noqa: BLE001
+            dp_err = f"rank {rank}: {type(ex).__name__}: {ex}"[:300]
+        if allreduce([1.0 if dp_err else 0.0], tdist.ReduceOp.MAX)[0] > 0:
+            dp = {"error": dp_err or "setup failed on another rank"}
+        else:
             def poison0():
-                for r, o in zip(specs0, offs0):
-                    if r.nbytes:
-                        arena0[o:o + r.nbytes].fill_(W.POISON_BYTE)
+                with torch.cuda.stream(stream):
+                    for r, o in zip(specs0, offs0):
+                        if r.nbytes:
+                            arena0[o:o + r.nbytes].fill_(W.POISON_BYTE)
                 stream.synchronize()
 
             def timed(fn):
@@ -704,20 +721,23 @@ def run_ours(args):
                     ts.append(e0.elapsed_time(e1) * 1e-3)
                 return statistics.median(allreduce(ts, tdist.ReduceOp.MAX)[1:])
 
-            t_striped = timed(lambda: sdist.restore_replicas(swd, None, stream))
-
             def independent():
                 swd.restore(stream)
                 return swd.verify(stream, hbm_pass=True)
 
-            t_indep = timed(independent)
+            with torch.cuda.stream(stream):
+                t_striped = timed(lambda: sdist.restore_replicas(swd, None, stream))
+                t_indep = timed(independent)
+            dp = {"replicas": world, "image_bytes": payload0, "striped_swap_in_s": round(t_striped, 4),
+                  "independent_swap_in_s": round(t_indep, 4), "speedup": round(t_indep / t_striped, 3),
+                  "striped_GBps_per_replica": round(payload0 / t_striped / GB, 2),
+                  "host_link_bytes_per_replica": payload0 // world,
+                  "how": "swap_restore_stripe (1/N of the CE_PIPE groups per replica over its own PCIe link) + in-place "
+                         "NCCL broadcasts of every stripe span from its owner + HBM verify of all chunks, max over ranks"}
+        if swd is not None:
+            swd.close()
         del arena0
-        dp = {"replicas": world, "image_bytes": payload0, "striped_swap_in_s": round(t_striped, 4),
-              "independent_swap_in_s": round(t_indep, 4), "speedup": round(t_indep / t_striped, 3),
-              "striped_GBps_per_replica": round(payload0 / t_striped / GB, 2),
-              "host_link_bytes_per_replica": payload0 // world,
-              "how": "swap_restore_stripe (1/N of the CE_PIPE groups per replica over its own PCIe link) + in-place "
-                     "NCCL broadcasts of every stripe span from its owner + HBM verify of all chunks, max over ranks"}
+
     if rank == 0:
         value = total_payload / (swapin_ms * 1e-3) / GB
         achieved = payload / (restore_ms * 1e-3) / GB

@@ -18,7 +18,7 @@ def test_bench_two_ranks_gloo():
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr=127.0.0.1", "--master-port=29533", os.path.join(ROOT, "bench.py"), "--gpus", "2",
            "--config", "A", "--steps", "2", "--warmup", "1", "--no-compare", "--no-cpu-baseline",
-           "--dist-backend", "gloo"]
+           "--dist-backend", "gloo", "--force-legs"]
     out = subprocess.run(cmd, capture_output=True, text=True, timeout=540, cwd=ROOT)
     assert out.returncode == 0, out.stderr[-3000:]
     lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
@@ -27,6 +27,11 @@ def test_bench_two_ranks_gloo():
     assert rec["n_gpus"] == 2 and rec["scaling"] == "weak" and rec["value"] > 0
     assert rec["config"]["payload_bytes_per_rank"] == 1 << 26
     assert rec["gpu_launches"] > 0
+    # the N>1 legs, forced on one device: helper = the target GPU (degenerate), two DP replicas over gloo
+    assert "error" not in rec["assisted_swap_in"]["1"], rec["assisted_swap_in"]
+    assert rec["assisted_swap_in"]["1"]["GBps"] > 0
+    dp = rec["dp_replicas"]
+    assert "error" not in dp and dp["replicas"] == 2 and dp["striped_swap_in_s"] > 0, dp
 
 
 @pytest.mark.timeout(900)
