@@ -728,12 +728,22 @@ def run_ours(args):
             with torch.cuda.stream(stream):
                 t_striped = timed(lambda: sdist.restore_replicas(swd, None, stream))
                 t_indep = timed(independent)
+                try:  # fused NVLink pull: CUDA IPC maps of the other replicas' arenas
+                    deltas, bases = sdist.map_replicas(arena0.data_ptr(), local_dev, None)
+                    t_pull = timed(lambda: sdist.pull_replicas(swd, deltas, None, stream))
+                    for b_ in bases:
+                        swap.ipc_close(local_dev, b_)
+                except Exception as ex:  # noqa: BLE001
+                    t_pull = f"{type(ex).__name__}: {ex}"[:200]
             dp = {"replicas": world, "image_bytes": payload0, "striped_swap_in_s": round(t_striped, 4),
                   "independent_swap_in_s": round(t_indep, 4), "speedup": round(t_indep / t_striped, 3),
                   "striped_GBps_per_replica": round(payload0 / t_striped / GB, 2),
+                  "striped_fused_pull_swap_in_s": round(t_pull, 4) if isinstance(t_pull, float) else t_pull,
                   "host_link_bytes_per_replica": payload0 // world,
                   "how": "swap_restore_stripe (1/N of the CE_PIPE groups per replica over its own PCIe link) + in-place "
-                         "NCCL broadcasts of every stripe span from its owner + HBM verify of all chunks, max over ranks"}
+                         "NCCL broadcasts of every stripe span from its owner + HBM verify of all chunks, max over ranks; "
+                         "fused pull: the other stripes read from the owners' HBM over NVLink by the SM mover with the "
+                         "chunk check from the same registers (swap_pull_stripes), then the HBM verify"}
         if swd is not None:
             swd.close()
         del arena0

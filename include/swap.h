@@ -217,6 +217,25 @@ SWAP_API swap_status swap_get_mechanism_dir(const swap_ctx_t* ctx, int direction
  * State as swap_restore (-> RESTORED). */
 SWAP_API swap_status swap_restore_stripe(swap_ctx_t* ctx, uint32_t stripe, uint32_t n_stripes, swap_stream_t stream);
 
+/* DP replicas, fused NVLink pull (NEXT-2): after swap_restore_stripe(ctx, stripe, n_stripes, ...), moves
+ * every chunk of the other stripes from the replica that restored it, reading that replica's HBM directly
+ * (over NVLink; the peer memory mapped into this process, e.g. by swap_ipc_import) with the SM mover kernel,
+ * which checks each chunk's checksum from the same registers: the all-gather and the chunk check are one
+ * kernel; mismatches add to the restore's n_bad / first_bad_chunk. peer_delta[o] for o != stripe =
+ * (this process's address of replica o's copy of a region byte) - (address of this ctx's copy): the
+ * replicas' regions must have one layout up to a constant shift per replica (e.g. one arena each, same
+ * offsets). The peers must have completed their stripe restores (caller's barrier). ESTATE unless
+ * RESTORED; EINVAL for n_stripes < 2, stripe >= n_stripes or no deltas. */
+SWAP_API swap_status swap_pull_stripes(swap_ctx_t* ctx, uint32_t stripe, uint32_t n_stripes, const int64_t* peer_delta,
+                                       swap_stream_t stream);
+/* CUDA IPC of a device range (for swap_pull_stripes across processes). export: 64-B handle of the
+ * cudaMalloc allocation holding dev_ptr and dev_ptr's offset in it (ECUDA for memory IPC cannot export,
+ * e.g. VMM arenas). import (in another process, device = the importer's): *base = the mapped allocation
+ * (pass to swap_ipc_close), *mapped = *base + offset. Opening a handle in its own process fails (ECUDA). */
+SWAP_API swap_status swap_ipc_export(int device, const void* dev_ptr, uint8_t* handle, uint64_t* offset);
+SWAP_API swap_status swap_ipc_import(int device, const uint8_t* handle, uint64_t offset, void** base, void** mapped);
+SWAP_API swap_status swap_ipc_close(int device, void* base);
+
 /* One coalesced copy of a restore group: `bytes` at device address dev_addr <- image[image_offset ..). */
 typedef struct {
   uint32_t group;        /* restore group index (the striping unit of swap_restore_stripe) */

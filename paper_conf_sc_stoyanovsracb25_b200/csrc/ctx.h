@@ -46,6 +46,7 @@ struct DescSet {
   std::vector<size_t> ce_bytes;
   std::vector<Group> groups;              // CE_PIPE
   std::vector<cudaEvent_t> group_ev;
+  std::vector<swk::SegDesc> h_desc;       // host copy of d_desc (the fused peer pull rewrites sources)
   bool owned = false;                     // false: an alias of another set
 };
 
@@ -100,6 +101,8 @@ struct swap_ctx {
   };
   std::vector<Helper> helpers;
   uint32_t stripe = 0, n_stripes = 1;  // CE_PIPE restore groups this restore moves (swap_restore_stripe)
+  swk::SegDesc* d_pull = nullptr;      // descriptors of the last swap_pull_stripes (sources in peer HBM)
+  size_t pull_cap = 0;
   int numa_node = -1;         // NUMA node the image placement targeted (-1: none)
   double numa_local = 1.0;    // sampled share of image pages on numa_node
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;

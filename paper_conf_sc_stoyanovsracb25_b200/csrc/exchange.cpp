@@ -3,6 +3,8 @@
 //                     HBM handed over slab by slab within the victims' memory + headroom (NEXT-1);
 //   swap_set_helpers  NVLink-assisted restore: peers pull restore groups over their own PCIe links into
 //                     HBM staging and copy them to the target over NVLink (NEXT-2).
+#include <cuda.h>
+
 #include <algorithm>
 #include <cstring>
 #include <string>
@@ -221,6 +223,102 @@ swap_status swap_set_helpers(swap_ctx_t* c, const int* devices, int n) {
   }
   CUDA_TRY(c, cudaSetDevice(c->cfg.device));
   return SWAP_OK;
+}
+
+// ---- DP replicas, fused NVLink pull (NEXT-2; include/swap.h). After swap_restore_stripe, every chunk of
+// the other replicas' stripes is moved by the SM mover kernel (SCATTER) from the replica that restored it:
+// the descriptors' source field points into that replica's HBM (mapped into this process by CUDA IPC, read
+// over NVLink), so the chunk checksum is computed from the same registers that carry the bytes -- the
+// all-gather and the check are one kernel.
+swap_status swap_pull_stripes(swap_ctx_t* c, uint32_t stripe, uint32_t n_stripes, const int64_t* peer_delta,
+                              swap_stream_t stream) {
+  if (!c || !peer_delta || n_stripes < 2 || stripe >= n_stripes) return SWAP_EINVAL;
+  if (c->st != St::RESTORED) {
+    c->err = "swap_pull_stripes needs this replica's stripe restored first (swap_restore_stripe)";
+    return SWAP_ESTATE;
+  }
+  DeviceGuard g(c->cfg.device);
+  cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  const DescSet& S = c->s_move;
+  std::vector<swk::SegDesc> d;
+  d.reserve(S.h_desc.size());
+  for (size_t gi = 0; gi < S.groups.size(); ++gi) {
+    const uint32_t o = (uint32_t)(gi % n_stripes);
+    if (o == stripe) continue;
+    for (uint32_t i = S.groups[gi].d0; i < S.groups[gi].d1; ++i) {
+      swk::SegDesc x = S.h_desc[i];
+      x.host = (uint64_t)((int64_t)x.dev + peer_delta[o]);
+      d.push_back(x);
+    }
+  }
+  if (d.empty()) return SWAP_OK;
+  if (d.size() > c->pull_cap) {
+    if (c->d_pull) cudaFree(c->d_pull);
+    c->d_pull = nullptr;
+    c->pull_cap = 0;
+    CUDA_TRY(c, cudaMalloc(&c->d_pull, d.size() * sizeof(swk::SegDesc)));
+    c->pull_cap = d.size();
+  }
+  // pageable source: the call returns once the bytes are staged, so `d` may go out of scope
+  CUDA_TRY(c, cudaMemcpyAsync(c->d_pull, d.data(), d.size() * sizeof(swk::SegDesc), cudaMemcpyHostToDevice, s));
+  swk::Params p = base_params(c, S);
+  p.desc = c->d_pull;
+  p.n_desc = (uint32_t)d.size();
+  return launch(c, swk::SCATTER, hash_kind(c), p, s);
+}
+
+namespace {
+using GetRange = CUresult (*)(CUdeviceptr*, size_t*, CUdeviceptr);
+GetRange get_range() {
+  static GetRange f = [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &p, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      return (GetRange) nullptr;
+    return reinterpret_cast<GetRange>(p);
+  }();
+  return f;
+}
+}  // namespace
+
+swap_status swap_ipc_export(int device, const void* dev_ptr, uint8_t* handle, uint64_t* offset) {
+  if (!dev_ptr || !handle || !offset) return SWAP_EINVAL;
+  DeviceGuard g(device);
+  GetRange f = get_range();
+  CUdeviceptr base = 0;
+  size_t size = 0;
+  if (!f || f(&base, &size, reinterpret_cast<CUdeviceptr>(dev_ptr)) != CUDA_SUCCESS) return SWAP_ECUDA;
+  cudaIpcMemHandle_t h;
+  if (cudaIpcGetMemHandle(&h, reinterpret_cast<void*>(base)) != cudaSuccess) {
+    cudaGetLastError();
+    return SWAP_ECUDA;  // not a cudaMalloc allocation (e.g. a VMM arena)
+  }
+  static_assert(sizeof(h) == 64, "cudaIpcMemHandle_t is 64 B");
+  memcpy(handle, &h, 64);
+  *offset = reinterpret_cast<uint64_t>(dev_ptr) - (uint64_t)base;
+  return SWAP_OK;
+}
+
+swap_status swap_ipc_import(int device, const uint8_t* handle, uint64_t offset, void** base, void** mapped) {
+  if (!handle || !base || !mapped) return SWAP_EINVAL;
+  DeviceGuard g(device);
+  cudaIpcMemHandle_t h;
+  memcpy(&h, handle, 64);
+  void* b = nullptr;
+  if (cudaIpcOpenMemHandle(&b, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+    cudaGetLastError();
+    return SWAP_ECUDA;
+  }
+  *base = b;
+  *mapped = static_cast<uint8_t*>(b) + offset;
+  return SWAP_OK;
+}
+
+swap_status swap_ipc_close(int device, void* base) {
+  if (!base) return SWAP_EINVAL;
+  DeviceGuard g(device);
+  return cudaIpcCloseMemHandle(base) == cudaSuccess ? SWAP_OK : SWAP_ECUDA;
 }
 
 }  // extern "C"

@@ -299,6 +299,9 @@ void release(swap_ctx* c) {
   if (c->d_zspans) cudaFree(c->d_zspans);
   c->d_zspans = nullptr;
   if (c->d_partial) cudaFree(c->d_partial);
+  if (c->d_pull) cudaFree(c->d_pull);
+  c->d_pull = nullptr;
+  c->pull_cap = 0;
   if (c->d_arrive) cudaFree(c->d_arrive);
   if (c->d_status) cudaFree(c->d_status);
   if (c->h_status) cudaFreeHost(c->h_status);
@@ -381,6 +384,7 @@ static swap_status build_set(swap_ctx* c, DescSet* S, Pick pick, bool zero_src) 
     CUDA_TRY(c, cudaMemcpy(S->d_desc, desc.data(), desc.size() * sizeof(swk::SegDesc), cudaMemcpyHostToDevice));
   S->group_ev.assign(S->groups.size(), nullptr);
   for (auto& e : S->group_ev) CUDA_TRY(c, cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  S->h_desc = std::move(desc);
   return SWAP_OK;
 }
 

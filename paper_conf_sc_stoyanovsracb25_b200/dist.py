@@ -19,7 +19,7 @@ from __future__ import annotations
 import torch
 import torch.distributed as dist
 
-from .swap import SWAP_OK, SwapError, Swapper, swap_merge_global
+from .swap import SWAP_OK, SwapError, Swapper, ipc_export, ipc_import, swap_merge_global
 
 
 def _comm_device(group=None) -> torch.device:
@@ -85,6 +85,42 @@ def restore_replicas(sw: Swapper, group=None, stream=None) -> dict:
         for w in works:
             w.wait()
         return sw.verify(s, hbm_pass=True, raise_on_corrupt=False)
+
+
+def map_replicas(local_ptr: int, device: int, group=None) -> tuple[list[int], list[int]]:
+    """CUDA IPC mapping of every other replica's arena into this process (for pull_replicas): all-gathers
+    each replica's (handle, offset, address) of its arena base; returns (peer_delta, bases to close) with
+    peer_delta[o] = mapped address of replica o's arena base - local_ptr (0 for this replica)."""
+    k, r = dist.get_world_size(group), dist.get_rank(group)
+    h, off = ipc_export(device, local_ptr)
+    allh = [None] * k
+    dist.all_gather_object(allh, (h, off), group=group)
+    deltas, bases = [], []
+    for o, (ho, offo) in enumerate(allh):
+        if o == r:
+            deltas.append(0)
+            continue
+        base, mapped = ipc_import(device, ho, offo)
+        bases.append(base)
+        deltas.append(mapped - local_ptr)
+    return deltas, bases
+
+
+def pull_replicas(sw: Swapper, peer_delta: list[int], group=None, stream=None) -> dict:
+    """Swap-in of k data-parallel replicas with the fused NVLink pull (NEXT-2): replica r restores its
+    stripe over its own PCIe link (swap_restore_stripe); once every stripe has landed (barrier), one SM
+    kernel per replica pulls the other stripes straight from the owners' HBM and checks every chunk from the
+    registers that carried it (swap_pull_stripes); then the HBM verify pass. A closing barrier keeps any
+    replica from overwriting its stripe while a peer may still be reading it. Returns the verify result."""
+    k, r = dist.get_world_size(group), dist.get_rank(group)
+    s = stream if stream is not None else torch.cuda.current_stream(sw.device)
+    sw.restore_stripe(r, k, s)
+    s.synchronize()
+    dist.barrier(group=group)
+    sw.pull_stripes(r, k, peer_delta, s)
+    res = sw.verify(s, hbm_pass=True, raise_on_corrupt=False)
+    dist.barrier(group=group)
+    return res
 
 
 def agree_restore(verify_result: dict, group=None) -> int:

@@ -30,7 +30,7 @@ U64_MAX = (1 << 64) - 1
 
 EXPORTS = [
     "swap_config_default", "swap_create", "swap_register_regions", "swap_checkpoint", "swap_sync",
-    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_get_mechanism_dir", "swap_get_numa", "swap_restore_stripe", "swap_get_restore_spans", "swap_set_region_policy", "swap_set_chunk_mask", "swap_get_manifest", "swap_get_image",
+    "swap_restore", "swap_verify", "swap_set_mechanism", "swap_get_mechanism", "swap_get_mechanism_dir", "swap_get_numa", "swap_restore_stripe", "swap_get_restore_spans", "swap_pull_stripes", "swap_ipc_export", "swap_ipc_import", "swap_ipc_close", "swap_set_region_policy", "swap_set_chunk_mask", "swap_get_manifest", "swap_get_image",
     "swap_get_summary", "swap_import", "swap_save", "swap_load", "swap_set_global", "swap_merge_global", "swap_plan_layout", "swap_plan_manifest", "swap_get_timings",
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
     "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
@@ -114,6 +114,10 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_get_numa": (st, [vp, P(ctypes.c_int32), P(ctypes.c_double)]),
         "swap_restore_stripe": (st, [vp, u32, u32, vp]),
         "swap_get_restore_spans": (st, [vp, vp, ctypes.c_size_t, P(ctypes.c_size_t)]),
+        "swap_pull_stripes": (st, [vp, u32, u32, P(ctypes.c_int64), vp]),
+        "swap_ipc_export": (st, [ctypes.c_int, vp, vp, P(ctypes.c_uint64)]),
+        "swap_ipc_import": (st, [ctypes.c_int, vp, ctypes.c_uint64, P(vp), P(vp)]),
+        "swap_ipc_close": (st, [ctypes.c_int, vp]),
         "swap_set_region_policy": (st, [vp, u32, u32]),
         "swap_set_chunk_mask": (st, [vp, u32, vp, ctypes.c_uint64]),
         "swap_get_manifest": (st, [vp, P(vp), P(sz)]),
@@ -205,6 +209,30 @@ def swap_verify(ctx, stream: int = 0, hbm_pass: bool = True):
     res = swap_verify_result_t()
     st = load().swap_verify(ctx, ctypes.c_void_p(stream), 1 if hbm_pass else 0, ctypes.byref(res))
     return st, res
+
+
+def ipc_export(device: int, ptr: int) -> tuple[bytes, int]:
+    """(64-B CUDA IPC handle of the allocation holding ptr, ptr's offset in it) -- swap_ipc_export."""
+    h = (ctypes.c_uint8 * 64)()
+    off = ctypes.c_uint64()
+    st = load().swap_ipc_export(device, ctypes.c_void_p(ptr), h, ctypes.byref(off))
+    if st:
+        raise SwapError(st, "swap_ipc_export failed (not a cudaMalloc allocation?)")
+    return bytes(h), off.value
+
+
+def ipc_import(device: int, handle: bytes, offset: int) -> tuple[int, int]:
+    """Maps another process's allocation: (base to close, mapped address of the exported pointer)."""
+    h = (ctypes.c_uint8 * 64).from_buffer_copy(handle)
+    base, mapped = ctypes.c_void_p(), ctypes.c_void_p()
+    st = load().swap_ipc_import(device, h, offset, ctypes.byref(base), ctypes.byref(mapped))
+    if st:
+        raise SwapError(st, "swap_ipc_import failed")
+    return base.value, mapped.value
+
+
+def ipc_close(device: int, base: int):
+    load().swap_ipc_close(device, ctypes.c_void_p(base))
 
 
 def swap_merge_global(summaries: bytes, world: int):
@@ -410,6 +438,12 @@ class Swapper:
     def restore_stripe(self, stripe: int, n_stripes: int, stream=None):
         """Restore only CE_PIPE groups g with g % n_stripes == stripe (swap_restore_stripe; DP replicas)."""
         self._check(load().swap_restore_stripe(self._ctx, stripe, n_stripes, _torch_stream(stream)))
+
+    def pull_stripes(self, stripe: int, n_stripes: int, peer_delta: list[int], stream=None):
+        """Fused NVLink pull of the other replicas' stripes with the chunk check (swap_pull_stripes);
+        peer_delta[o] = replica o's mapped address of a byte minus this replica's (ignored for o == stripe)."""
+        arr = (ctypes.c_int64 * n_stripes)(*peer_delta)
+        self._check(load().swap_pull_stripes(self._ctx, stripe, n_stripes, arr, _torch_stream(stream)))
 
     def restore_spans(self) -> list[tuple[int, int, int, int]]:
         """(group, dev_addr, image_offset, bytes) of every coalesced restore copy (swap_get_restore_spans)."""

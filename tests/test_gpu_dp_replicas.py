@@ -3,7 +3,9 @@ image share cuda:0 over gloo; each restores only its stripe of the restore group
 and the stripes are exchanged by in-place broadcasts (dist.restore_replicas), then every replica verifies
 all chunks from HBM. Checked against the oracle: the restored arenas equal the original bytes, a bit
 flipped in replica 1's image inside a group replica 1 owns is reported (same chunk) by both replicas' HBM
-passes and by replica 1's fused check, and a flip inside a group replica 0 owns is never read."""
+passes and by replica 1's fused check, and a flip inside a group replica 0 owns is never read. The fused
+NVLink pull variant (CUDA IPC mapping of the other replica's arena, swap_pull_stripes) restores the same
+bytes, and there replica 0's pull kernel itself reports the chunk it read corrupted from replica 1."""
 import os
 import tempfile
 
@@ -72,6 +74,22 @@ def _worker(rank, world, init_file, q):
             res = sdist.restore_replicas(sw, None, s)
             out["flip"] = (res["n_bad"], res["first_bad_chunk"], res["hbm_n_bad"], res["hbm_first_bad"])
             out["flip_chunk"] = chunk_of[p1]
+            # the same with the fused NVLink pull (CUDA IPC of the other replica's arena; same device here):
+            # replica 0's pull kernel reads replica 1's corrupted stripe and its fused check reports it
+            deltas, bases = sdist.map_replicas(base, 0, None)
+            poison(arena, specs, offs)
+            res = sdist.pull_replicas(sw, deltas, None, s)
+            out["pull_flip"] = (res["n_bad"], res["first_bad_chunk"], res["hbm_n_bad"], res["hbm_first_bad"])
+            if rank == 1:  # undo the flips: a clean pulled swap-in restores every byte
+                img[p1] ^= 0x01
+                img[p0] ^= 0x01
+            dist.barrier()
+            poison(arena, specs, offs)
+            res = sdist.pull_replicas(sw, deltas, None, s)
+            out["pull_clean"] = (res["n_bad"], res["hbm_n_bad"], res["manifest_ok"])
+            out["pull_mem_equal"] = bool(np.array_equal(arena.cpu().numpy(), host))
+            for b in bases:
+                swap.ipc_close(0, b)
         q.put((rank, out))
     except Exception:  # report instead of leaving the parent waiting on the queue
         import traceback
@@ -104,3 +122,8 @@ def test_two_replicas_striped_restore():
     # the flip in replica 0's stripe was never read
     assert res[1]["flip"] == (1, g, 1, g)
     assert res[0]["flip"] == (0, (1 << 64) - 1, 1, g)
+    # fused pull: replica 0's pull kernel checks the chunk it read from replica 1's HBM
+    assert res[1]["pull_flip"] == (1, g, 1, g)
+    assert res[0]["pull_flip"] == (1, g, 1, g)
+    for r in range(world):
+        assert res[r]["pull_clean"] == (0, 0, 1) and res[r]["pull_mem_equal"], r

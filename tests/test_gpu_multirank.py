@@ -32,6 +32,7 @@ def test_bench_two_ranks_gloo():
     assert rec["assisted_swap_in"]["1"]["GBps"] > 0
     dp = rec["dp_replicas"]
     assert "error" not in dp and dp["replicas"] == 2 and dp["striped_swap_in_s"] > 0, dp
+    assert isinstance(dp["striped_fused_pull_swap_in_s"], float), dp
 
 
 @pytest.mark.timeout(900)
