@@ -127,3 +127,48 @@ def test_two_replicas_striped_restore():
     assert res[0]["pull_flip"] == (1, g, 1, g)
     for r in range(world):
         assert res[r]["pull_clean"] == (0, 0, 1) and res[r]["pull_mem_equal"], r
+
+
+@pytest.mark.parametrize("kind", [1, 2])
+def test_fused_pull_in_process(kind):
+    """swap_pull_stripes with the peer replica as a second arena of this process (the same bytes at a
+    constant shift): every byte restored, and a corruption of the peer's HBM copy inside the pulled stripe
+    is reported by the pull kernel's fused check as exactly its chunk (the oracle's chunk of that byte)."""
+    import sys
+
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    import numpy as np
+    import torch
+
+    import oracle as orc
+    import workloads as W
+    from gpu_util import device_case, poison
+    from paper_conf_sc_stoyanovsracb25_b200 import swap
+
+    specs = W.config_a(5) + W.edge_tables(4096)["chunk_pm1"]
+    arena, host, base, offs, sw_regions, or_regions = device_case(specs, 5)
+    rc, ref, moff = orc.checkpoint(or_regions, host, base, kind, 4096, 4096, threads=4)
+    peer = arena.clone()
+    delta = peer.data_ptr() - base
+    s = torch.cuda.Stream()
+    with swap.Swapper(sw_regions, chunk_bytes=4096, checksum=kind, pipe_mib=2) as sw, torch.cuda.stream(s):
+        sw.checkpoint(s)
+        assert np.array_equal(sw.image(), ref)
+        poison(arena, specs, offs)
+        sw.restore_stripe(0, 2, s)
+        sw.pull_stripes(0, 2, [0, delta], s)
+        res = sw.verify(s)
+        assert (res["n_bad"], res["hbm_n_bad"]) == (0, 0)
+        assert np.array_equal(arena.cpu().numpy(), host)
+        # corrupt one byte of the peer copy inside a group of stripe 1
+        g1 = next(sp for sp in sw.restore_spans() if sp[0] % 2 == 1)
+        dev = g1[1] + g1[3] // 3
+        peer[dev - base] ^= 0x40
+        # the oracle's chunk of that byte: region i holding it, chunk (dev - addr_i) // C
+        i = next(k for k, (_, a, nb, _) in enumerate(or_regions) if a <= dev < a + nb)
+        chunk = sum(-(-r.nbytes // 4096) for r in specs[:i]) + (dev - or_regions[i][1]) // 4096
+        poison(arena, specs, offs)
+        sw.restore_stripe(0, 2, s)
+        sw.pull_stripes(0, 2, [0, delta], s)
+        res = sw.verify(s, raise_on_corrupt=False)
+        assert (res["n_bad"], res["first_bad_chunk"], res["hbm_n_bad"], res["hbm_first_bad"]) == (1, chunk, 1, chunk)

@@ -45,7 +45,8 @@ with swap.Swapper(regions, chunk_bytes=1024, checksum=2, mechanism="ce_region") 
     sw.restore(s)
     assert sw.verify(s)["status"] == 0
 # every XXH64 hash kernel, forced per launch through SWAP_XXH_KERNEL (the CE movers hash from HBM)
-for v in ("lane8", "bal", "bal8", "dyn", "coop", "coop16", "coop8", "ring"):
+for v in ("lane8", "bal", "bal8", "dyn", "coop", "coop16", "coop8", "ring", "quad", "quad1k", "quad4k", "quad_x",
+          "dyn_x", "quad2", "pair", "pair2", "quad3k"):
     os.environ["SWAP_XXH_KERNEL"] = v
     with swap.Swapper(regions, chunk_bytes=1024, checksum=2, mechanism="ce_region") as sw, torch.cuda.stream(s):
         sw.checkpoint(s)
@@ -53,6 +54,36 @@ for v in ("lane8", "bal", "bal8", "dyn", "coop", "coop16", "coop8", "ring"):
         sw.restore(s)
         assert sw.verify(s)["status"] == 0, v
 os.environ.pop("SWAP_XXH_KERNEL")
+# the quad kernels' multi-stage rings: chunks of several stages (64 KiB) and a ragged tail
+for v in ("quad", "quad2", "quad3k"):
+    os.environ["SWAP_XXH_KERNEL"] = v
+    with swap.Swapper(regions, chunk_bytes=1 << 16, checksum=2, mechanism="ce_region") as sw, torch.cuda.stream(s):
+        sw.checkpoint(s)
+        poison(arena, specs, offs)
+        sw.restore(s)
+        assert sw.verify(s)["status"] == 0, v
+os.environ.pop("SWAP_XXH_KERNEL")
+# CRC-32C hash kernel variants (fixed shared layout at the 0x400 dynamic base)
+for v in ("base", "b0f", "zb", "zbb0f"):
+    os.environ["SWAP_CRC_KERNEL"] = v
+    with swap.Swapper(regions, chunk_bytes=1 << 16, checksum=1, mechanism="ce_region") as sw, torch.cuda.stream(s):
+        sw.checkpoint(s)
+        poison(arena, specs, offs)
+        sw.restore(s)
+        assert sw.verify(s)["status"] == 0, v
+os.environ.pop("SWAP_CRC_KERNEL")
+# DP replicas in one process: stripe restore of replica A, then the fused pull of the other stripe from
+# replica B (a second arena with the same bytes at a constant shift)
+arena_b = arena.clone()
+delta = arena_b.data_ptr() - arena.data_ptr()
+for kind in (1, 2):
+    with swap.Swapper(regions, chunk_bytes=4096, checksum=kind, pipe_mib=1) as sw, torch.cuda.stream(s):
+        sw.checkpoint(s)
+        poison(arena, specs, offs)
+        sw.restore_stripe(0, 2, s)
+        sw.pull_stripes(0, 2, [0, delta], s)
+        assert sw.verify(s)["status"] == 0, kind
+del arena_b
 # VMM arenas + full-duplex exchange
 def engine(seed):
     sp = W.scaled(W.config_b(), 48 << 20)
