@@ -672,6 +672,7 @@ def run_ours(args):
                         "how": "same sample and threads, CRC-32C by the SSE4.2 crc32 instruction"},
                **cpu_context(my_cpus)}
 
+    clk_all = gather_obj({k: clk.get(k) for k in ("sm_mhz", "samples", "reasons")})
     numa = sw.numa()
     placement = gather_obj({"rank": rank, "gpu": local_dev, "gpu_numa_node": node, "cpus": len(my_cpus),
                             "image_numa_node": numa["node"], "image_local_fraction": numa["local_fraction"]})
@@ -769,6 +770,7 @@ def run_ours(args):
                                  "events); value uses the mean over steps of the per-step max over ranks"},
             "swap_in_latency_s": round(swapin_ms * 1e-3, 5),
             "swap_in_latency_s_range": [round(min(swapin_steps) * 1e-3, 5), round(max(swapin_steps) * 1e-3, 5)],
+            "swap_in_latency_s_median": round(statistics.median(swapin_steps) * 1e-3, 5),
             "restore_GBps_per_gpu": round(achieved, 3),
             "restore_GBps_per_gpu_slowest": round(payload / (max(restore_steps) * 1e-3) / GB, 3),
             "checkpoint_GBps_per_gpu": round(payload / (ckpt_ms * 1e-3) / GB, 3),
@@ -803,6 +805,7 @@ def run_ours(args):
                            "because the device-timed metric is itself the host-to-device transfer"},
             "gpu_launches": int(launches),
             "clocks": clk,
+            "clocks_all_ranks": clk_all if world > 1 else None,
             "placement": placement,
             "topology": topology(),
             "cpu_baseline": cpu,
