@@ -172,3 +172,54 @@ def test_fused_pull_in_process(kind):
         sw.pull_stripes(0, 2, [0, delta], s)
         res = sw.verify(s, raise_on_corrupt=False)
         assert (res["n_bad"], res["first_bad_chunk"], res["hbm_n_bad"], res["hbm_first_bad"]) == (1, chunk, 1, chunk)
+
+
+def test_stripe_pull_with_policies_masks_and_released_arena():
+    """Replica A in a released, bound VMM arena with a DISCARD region and a touched-chunk mask: the stripe
+    restore re-acquires HBM for *every* group (the pulled ones included), zero-fills the zero chunks in full,
+    and the fused pull from replica B (a cudaMalloc copy) fills the rest -- equal to the oracle's
+    policy_view, the image equal to the oracle's checkpoint of that view."""
+    import sys
+
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    import numpy as np
+    import torch
+
+    import oracle as orc
+    import workloads as W
+    from paper_conf_sc_stoyanovsracb25_b200 import swap
+
+    C = 1 << 16
+    specs = W.scaled(W.config_b(), 96 << 20)
+    offs, total = W.place(specs)
+    arena = swap.Arena(total)
+    base, view = arena.alloc(total)
+    W.fill_device_arena(view, specs, offs, seed=9)
+    peer = view.clone()  # replica B: the same bytes, cudaMalloc'd
+    host = view.cpu().numpy()
+    regions = [(base + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs, offs))]
+    or_regions = [(i, a, n, k) for (a, n, k, i) in regions]
+    big = max(range(len(specs)), key=lambda i: specs[i].nbytes)
+    disc = next(i for i in range(len(specs)) if i != big and specs[i].nbytes > C)
+    keep = (np.arange(-(-specs[big].nbytes // C)) % 3 != 1).astype(np.uint8)
+    s = torch.cuda.Stream()
+    with swap.Swapper(regions, chunk_bytes=C, pipe_mib=4) as sw, torch.cuda.stream(s):
+        sw.set_region_policy(disc, "discard")
+        sw.set_chunk_mask(big, keep)
+        sw.bind_arena(arena)
+        sw.checkpoint(s)
+        pol = [orc.SAVE] * len(specs)
+        pol[disc] = orc.DISCARD
+        want = orc.policy_view(or_regions, pol, host, host, base, C, {big: keep})
+        rc, ref, _ = orc.checkpoint(or_regions, want, base, orc.CRC32C, C, 4096, threads=8)
+        assert rc == 0 and np.array_equal(sw.image(), ref)
+        arena.release()
+        sw.restore_stripe(1, 2, s)
+        sw.pull_stripes(1, 2, [peer.data_ptr() - base, 0], s)
+        res = sw.verify(s)
+        assert (res["n_bad"], res["hbm_n_bad"]) == (0, 0) and arena.resident
+        back = arena.tensor(0, total).cpu().numpy()
+        for r, o in zip(specs, offs):
+            assert np.array_equal(back[o:o + r.nbytes], want[o:o + r.nbytes]), r.name
+        sw.bind_arena(None)
+    arena.close()

@@ -55,7 +55,7 @@ def host_free() -> int:
     return 0
 
 
-def check_records(man: np.ndarray, plan, specs, regions, kind: int):
+def check_records(man: np.ndarray, plan, specs, regions, kind: int, C: int = C):
     """Header, region records and chunk records (all but c_g) against oracle.plan + §8(c) step 3."""
     n, m = len(specs), plan.n_chunks
     magic, ver, k, c, a, nn, mm, payload, rank, world = HDR.unpack_from(man, 0)
@@ -95,7 +95,7 @@ def poison_restore_verify(sw, arena, specs, offs, stream):
     return res
 
 
-def flip_check(swp, sw, plan, specs, stream, g, img):
+def flip_check(swp, sw, plan, specs, stream, g, img, C: int = C):
     """One flipped image bit in chunk g is reported as exactly chunk g; then a clean restore."""
     i = int(np.searchsorted(np.asarray(plan.first), g, side="right") - 1)
     j = g - plan.first[i]
@@ -112,8 +112,11 @@ def flip_check(swp, sw, plan, specs, stream, g, img):
     assert sw.verify(stream, hbm_pass=True)["status"] == 0
 
 
-@pytest.mark.parametrize("cfg,kind", [("B", 1), ("B", 2), ("D", 2)], ids=["B-crc32c", "B-xxh64", "D-xxh64"])
-def test_full_size_every_chunk(swp, orc, cfg, kind):
+@pytest.mark.parametrize("cfg,kind,C", [("B", 1, C), ("B", 2, C), ("D", 2, C), ("B", 2, 4 << 20), ("B", 2, 16 << 20)],
+                         ids=["B-crc32c", "B-xxh64", "D-xxh64", "B-xxh64-4MiB", "B-xxh64-16MiB"])
+def test_full_size_every_chunk(swp, orc, cfg, kind, C):
+    """4 / 16 MiB XXH64 chunks: the round-2 quad-per-chunk kernels (2 x 3 KiB / 2 x 4 KiB rings) at full size;
+    16 MiB restores take AUTO's coalesced copies + one hash pass (CE_BATCH)."""
     specs = W.config_b() if cfg == "B" else W.config_d(0)
     payload = sum(r.nbytes for r in specs)
     if host_free() < 2.3 * payload:
@@ -125,12 +128,14 @@ def test_full_size_every_chunk(swp, orc, cfg, kind):
     stream = torch.cuda.Stream()
     sw = swp.Swapper(regions, chunk_bytes=C, checksum=kind, mechanism="auto")
     try:
-        assert sw.mechanism() == "ce_pipe"  # the bench's launch configuration at this size
+        # the bench's launch configuration at this size (XXH64 with chunks > 4 MiB restores with CE_BATCH)
+        assert sw.mechanism() == ("ce_batch" if C > (4 << 20) else "ce_pipe")
+        assert sw.mechanism("checkpoint") == "ce_pipe"
         with torch.cuda.stream(stream):
             sw.checkpoint(stream)
             img, man = sw.image(), sw.manifest()
             assert img.size == plan.image_bytes and man.size == plan.image_bytes - plan.manifest_off
-            cg = check_records(man, plan, specs, regions, kind)
+            cg = check_records(man, plan, specs, regions, kind, C)
             assert orc.manifest_ok(man)
             rc, nbad, fbad = orc.verify(man, mem, base, threads=THREADS)
             assert (rc, nbad, fbad) == (0, 0, U64_MAX), "GPU chunk checksums differ from the oracle"
@@ -147,7 +152,7 @@ def test_full_size_every_chunk(swp, orc, cfg, kind):
                 assert np.array_equal(arena[lo:lo + step].cpu().numpy(), mem[lo:lo + step]), f"arena at {lo}"
             rng = np.random.default_rng(5)
             g = int(rng.integers(0, plan.n_chunks))
-            flip_check(swp, sw, plan, specs, stream, g, img)
+            flip_check(swp, sw, plan, specs, stream, g, img, C)
     finally:
         sw.close()
         del arena
