@@ -336,10 +336,13 @@ SWAP_API swap_status swap_bind_arena(swap_ctx_t* ctx, swap_arena_t* a);
 
 /* NVLink-assisted restore (NEXT-2): with SWAP_MECH_CE_PIPE, restore groups are striped round-robin over
  * this device and the `n` helper devices; a helper copies its groups' image range from the pinned host
- * image into its own HBM staging buffer over its own PCIe link, then to this device's regions with
- * peer copies (NVLink via NVSwitch), and this device's side stream checks each group as usual. Helpers
- * should be idle GPUs of the node; peer access to this device is enabled on each. A helper equal to this
- * device degenerates to an on-device staging copy (used by the one-GPU tests). n = 0 removes them.
+ * image into its own HBM staging buffer over its own PCIe link, and then this device's SM mover kernel
+ * pulls the group from the helper's staging over NVLink (peer access this device -> helper) into the
+ * regions and checks every chunk from the same registers (the transfer and the check are one kernel).
+ * With SWAP_ASSIST=copy in the environment (read when the helpers are set) the helper instead copies the
+ * group to this device with peer copies (copy engines) and this device re-reads it for the hash check.
+ * Helpers should be idle GPUs of the node; peer access is enabled both ways. A helper equal to this
+ * device degenerates to an on-device staging buffer (used by the one-GPU tests). n = 0 removes them.
  * Needs REGISTERED+ (staging is sized from the restore groups). The checkpoint path is unchanged. */
 SWAP_API swap_status swap_set_helpers(swap_ctx_t* ctx, const int* devices, int n);
 

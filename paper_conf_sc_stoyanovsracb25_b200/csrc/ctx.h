@@ -95,11 +95,16 @@ struct swap_ctx {
   struct Helper {
     int dev = -1;
     cudaStream_t s = nullptr;
-    uint8_t* staging = nullptr;
+    uint8_t* staging[2] = {nullptr, nullptr};  // ping-pong: the helper's i-th group of a restore uses slot i % 2
     uint64_t staging_bytes = 0;  // the largest restore group's image range when the helpers were set
     cudaEvent_t ev = nullptr, done = nullptr;
+    cudaEvent_t consumed[2] = {nullptr, nullptr};  // this device has finished reading the slot (fused pull)
   };
   std::vector<Helper> helpers;
+  // fused helper pull: s_move's descriptors with the sources of helper groups rewritten to the helper's
+  // staging (read over NVLink by this device's SM mover); assist_copy = use copy-engine peer copies + hash
+  swk::SegDesc* d_assist = nullptr;
+  bool assist_copy = false;
   uint32_t stripe = 0, n_stripes = 1;  // CE_PIPE restore groups this restore moves (swap_restore_stripe)
   swk::SegDesc* d_pull = nullptr;      // descriptors of the last swap_pull_stripes (sources in peer HBM)
   size_t pull_cap = 0;

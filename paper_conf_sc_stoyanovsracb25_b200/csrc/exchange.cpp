@@ -6,6 +6,7 @@
 #include <cuda.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -218,10 +219,40 @@ swap_status swap_set_helpers(swap_ctx_t* c, const int* devices, int n) {
     CUDA_TRY(c, cudaEventCreateWithFlags(&h.ev, cudaEventDisableTiming));
     CUDA_TRY(c, cudaEventCreateWithFlags(&h.done, cudaEventDisableTiming));
     h.staging_bytes = std::max<uint64_t>(stage, 16);
-    CUDA_TRY(c, cudaMalloc(&h.staging, h.staging_bytes));
-    c->helpers.push_back(h);
+    c->helpers.push_back(h);  // owned by the ctx from here on (free_helpers releases whatever was made)
+    auto& hh = c->helpers.back();
+    for (int k = 0; k < 2; ++k) CUDA_TRY(c, cudaMalloc(&hh.staging[k], hh.staging_bytes));
   }
   CUDA_TRY(c, cudaSetDevice(c->cfg.device));
+  for (auto& h : c->helpers)  // recorded on this device's side stream, so created on this device
+    for (int k = 0; k < 2; ++k) CUDA_TRY(c, cudaEventCreateWithFlags(&h.consumed[k], cudaEventDisableTiming));
+  if (n == 0) return SWAP_OK;
+  // the fused pull: this device reads the helpers' staging (peer access target -> helper), with s_move's
+  // descriptors of every helper group rewritten to source from the staging copy of its image range
+  for (const auto& h : c->helpers)
+    if (h.dev != c->cfg.device) {
+      cudaError_t e = cudaDeviceEnablePeerAccess(h.dev, 0);
+      if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return cuda_fail(c, e, "peer access to helper");
+      cudaGetLastError();
+    }
+  const DescSet& S = c->s_move;
+  std::vector<swk::SegDesc> d = S.h_desc;
+  const size_t H = c->helpers.size();
+  for (size_t gi = 0; gi < S.groups.size(); ++gi) {
+    const size_t k = gi % (H + 1);
+    if (k == 0) continue;
+    const Group& G = S.groups[gi];
+    const uint64_t lo_dev = reinterpret_cast<uint64_t>(c->image_dev + (G.spans.front().host - c->image));
+    const int slot = (int)((gi / (H + 1)) % 2);  // ping-pong staging (movers.cpp ce_pipe)
+    for (uint32_t i = G.d0; i < G.d1; ++i)
+      d[i].host = reinterpret_cast<uint64_t>(c->helpers[k - 1].staging[slot]) + (d[i].host - lo_dev);
+  }
+  if (!d.empty()) {
+    CUDA_TRY(c, cudaMalloc(&c->d_assist, d.size() * sizeof(swk::SegDesc)));
+    CUDA_TRY(c, cudaMemcpy(c->d_assist, d.data(), d.size() * sizeof(swk::SegDesc), cudaMemcpyHostToDevice));
+  }
+  const char* mode = getenv("SWAP_ASSIST");
+  c->assist_copy = mode && !strcmp(mode, "copy");
   return SWAP_OK;
 }
 

@@ -188,6 +188,7 @@ swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, c
       // helper k-1: H2D of the group's image range into its staging over its own PCIe link, then
       // NVLink peer copies of each span to this device; the side stream checks it as usual
       auto& h = c->helpers[k - 1];
+      const int slot = (int)((g / (H + 1)) % 2);  // the same slot the fused descriptors were built for
       uint8_t* lo = G.spans.front().host;
       uint8_t* hi = G.spans.back().host + G.spans.back().bytes;
       if ((uint64_t)(hi - lo) > h.staging_bytes) {  // groups rebuilt without re-sizing the helpers
@@ -195,18 +196,29 @@ swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, c
         return SWAP_EINTERNAL;
       }
       CUDA_TRY(c, cudaSetDevice(h.dev));
-      CUDA_TRY(c, cudaMemcpyAsync(h.staging, lo, (size_t)(hi - lo), cudaMemcpyHostToDevice, h.s));
-      for (const Span& sp : G.spans)
-        CUDA_TRY(c, cudaMemcpyPeerAsync(reinterpret_cast<void*>(sp.dev), c->cfg.device, h.staging + (sp.host - lo), h.dev,
-                                        sp.bytes, h.s));
+      // the slot is free once this device has pulled the group that used it before (fused mode; in copy
+      // mode the helper's own stream orders the reuse)
+      CUDA_TRY(c, cudaStreamWaitEvent(h.s, h.consumed[slot], 0));
+      CUDA_TRY(c, cudaMemcpyAsync(h.staging[slot], lo, (size_t)(hi - lo), cudaMemcpyHostToDevice, h.s));
+      if (c->assist_copy || !c->d_assist)  // copy-engine peer copies, then the usual HBM hash check
+        for (const Span& sp : G.spans)
+          CUDA_TRY(c, cudaMemcpyPeerAsync(reinterpret_cast<void*>(sp.dev), c->cfg.device,
+                                          h.staging[slot] + (sp.host - lo), h.dev, sp.bytes, h.s));
       CUDA_TRY(c, cudaEventRecord(h.ev, h.s));
       CUDA_TRY(c, cudaSetDevice(c->cfg.device));
       CUDA_TRY(c, cudaStreamWaitEvent(c->side, h.ev, 0));
       swk::Params p = base;
-      p.desc = base.desc + G.d0;
       p.partial = base.partial + G.d0;
       p.n_desc = G.d1 - G.d0;
-      if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, c->side)) != SWAP_OK) return st;
+      if (c->assist_copy || !c->d_assist) {
+        p.desc = base.desc + G.d0;
+        if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, c->side)) != SWAP_OK) return st;
+      } else {  // fused: this device's SM mover pulls the group from the helper's staging over NVLink and
+                // checks every chunk from the same registers (no peer copy, no HBM re-read)
+        p.desc = c->d_assist + G.d0;
+        if ((st = launch(c, swk::SCATTER, hash_kind(c), p, c->side)) != SWAP_OK) return st;
+        CUDA_TRY(c, cudaEventRecord(h.consumed[slot], c->side));
+      }
       continue;
     }
     if ((st = copy_spans(c, G.spans, dir, s)) != SWAP_OK) return st;
@@ -264,28 +276,39 @@ swap_status upload_tables(swap_ctx* c) {
   return SWAP_OK;
 }
 
-// Auto segment size: enough CRC work items to give every warp slot of the GPU (SMs x 32) one, between
-// 4 KiB and 256 KiB (large images keep 256 KiB; a 64 MiB image gets 8 KiB).
+// Auto segment size: the smallest power of 2 that gives every warp slot of the GPU (SMs x 32) at most one
+// CRC work item -- one round of the hash kernel -- between 4 KiB and 256 KiB (large images keep 256 KiB; a
+// 64 MiB image gets 16 KiB: its verify pass 45 us vs 50 us with 8 KiB, 74 / 54 / 80 us with 4 / 32 / 64 KiB,
+// tools/seg_ab.py).
 uint32_t auto_seg(const swap_ctx* c, uint64_t payload) {
   const uint64_t per = payload / ((uint64_t)c->sm_count * 32 + 1);
   uint64_t s = 4096;
-  while (s * 2 <= per && s < (256u << 10)) s *= 2;
+  while (s < per && s < (256u << 10)) s *= 2;
   return (uint32_t)s;
 }
 
 void free_helpers(swap_ctx* c) {
   int cur = -1;
   cudaGetDevice(&cur);
+  if (c->side) {  // the side stream may still be pulling from the staging buffers
+    cudaSetDevice(c->cfg.device);
+    cudaStreamSynchronize(c->side);
+  }
   for (auto& h : c->helpers) {
     cudaSetDevice(h.dev);
     if (h.s) cudaStreamSynchronize(h.s);
-    if (h.staging) cudaFree(h.staging);
+    for (int k = 0; k < 2; ++k) {
+      if (h.staging[k]) cudaFree(h.staging[k]);
+      if (h.consumed[k]) cudaEventDestroy(h.consumed[k]);
+    }
     if (h.ev) cudaEventDestroy(h.ev);
     if (h.done) cudaEventDestroy(h.done);
     if (h.s) cudaStreamDestroy(h.s);
   }
   c->helpers.clear();
   if (cur >= 0) cudaSetDevice(cur);
+  if (c->d_assist) cudaFree(c->d_assist);
+  c->d_assist = nullptr;
 }
 
 void release(swap_ctx* c) {

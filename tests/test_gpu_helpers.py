@@ -1,6 +1,7 @@
 """NEXT-2 NVLink-assisted restore, degenerate one-GPU form: helper "peers" equal to the target device,
-so every helper group goes host -> HBM staging -> peer copy (here on-device) -> regions. The striping,
-staging offsets, cross-stream ordering and checks must give a bit-exact restore."""
+so every helper group goes host -> HBM staging -> regions, either pulled by the target's SM mover with the
+fused check (default) or by peer copies + the HBM hash check (SWAP_ASSIST=copy). The striping, staging
+offsets, cross-stream ordering and checks must give a bit-exact restore."""
 import numpy as np
 import pytest
 
@@ -19,9 +20,14 @@ def swp():
     return swap
 
 
+@pytest.mark.parametrize("mode", ["fused", "copy"])
 @pytest.mark.parametrize("n_helpers", [1, 2])
 @pytest.mark.parametrize("kind", [1, 2], ids=["crc32c", "xxh64"])
-def test_assisted_restore_bit_exact(swp, orc, n_helpers, kind):
+def test_assisted_restore_bit_exact(swp, orc, n_helpers, kind, mode, monkeypatch):
+    if mode == "copy":
+        monkeypatch.setenv("SWAP_ASSIST", "copy")
+    else:
+        monkeypatch.delenv("SWAP_ASSIST", raising=False)
     specs = W.scaled(W.config_b(), 160 << 20)
     arena, host, base, offs, sw_regions, or_regions = device_case(specs, 41)
     rc, ref, moff = orc.checkpoint(or_regions, host, base, kind, 1 << 20, 4096, threads=8)
@@ -70,3 +76,32 @@ def test_assisted_restore_with_bound_arena_and_policies(swp, orc):
             assert np.array_equal(back[o:o + r.nbytes], want)
         sw.bind_arena(None)
     arena.close()
+
+
+def test_helpers_with_mask_and_import(swp, orc):
+    """a chunk mask shrinks the restore groups (the helpers' staging is re-sized at the
+    checkpoint); swap_import then rebuilds full groups, larger than that staging -- it must re-size the
+    helpers again, and the CE_PIPE restore through the helpers stays bit-exact."""
+    C = 1 << 20
+    specs = W.scaled(W.config_b(), 300 << 20)
+    arena, host, base, offs, sw_regions, or_regions = device_case(specs, 17)
+    big = max(range(len(specs)), key=lambda i: specs[i].nbytes)
+    n = -(-specs[big].nbytes // C)
+    keep = (np.arange(n) % 8 == 0).astype(np.uint8)
+    s = torch.cuda.Stream()
+    with swp.Swapper(sw_regions, chunk_bytes=C, mechanism="ce_pipe", pipe_mib=16) as sw, torch.cuda.stream(s):
+        sw.set_helpers([0])
+        sw.set_chunk_mask(big, keep)
+        sw.checkpoint(s)  # masked groups; helpers re-sized for them
+        want = orc.policy_view(or_regions, [orc.SAVE] * len(specs), host, host, base, C, {big: keep})
+        rc, ref, moff = orc.checkpoint(or_regions, want, base, 1, C, 4096, threads=8)
+        assert np.array_equal(sw.image(), ref)
+        sw.import_image()  # the image "came from elsewhere": full groups again
+        poison(arena, specs, offs)
+        sw.restore(s)
+        res = sw.verify(s)
+        assert res["status"] == 0 and res["n_bad"] == 0 and res["hbm_n_bad"] == 0
+        back = arena.cpu().numpy()
+        for r, o in zip(specs, offs):
+            assert np.array_equal(back[o:o + r.nbytes], want[o:o + r.nbytes]), r.name
+        sw.set_helpers([])
