@@ -625,32 +625,40 @@ def run_ours(args):
             barrier()
             if rank == 0:
                 helpers = [(local_dev + i) % ndev for i in range(1, k + 1)]
-                try:
-                    sw.set_mechanism("ce_pipe")
-                    sw.set_helpers(helpers)
-                    ts = []
-                    for _ in range(3):
-                        poison()
-                        stream.synchronize()
-                        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                        e0.record(stream)
-                        sw.restore(stream)
-                        res = sw.verify(stream, hbm_pass=True)
-                        e1.record(stream)
-                        e1.synchronize()
-                        assert res["status"] == 0 and res["n_bad"] == 0 and res["hbm_n_bad"] == 0, res
-                        ts.append(e0.elapsed_time(e1) * 1e-3)
-                    t = statistics.median(ts[1:])
-                    assisted[str(k)] = {"helpers": helpers, "swap_in_s": round(t, 4), "GBps": round(payload / t / GB, 2),
-                                        "frac_of_k_plus_1_links": round(payload / t / GB / ((k + 1) * ce["h2d"]), 3)}
-                except Exception as ex:  # noqa: BLE001 - an informational leg must not sink the line
-                    assisted[str(k)] = {"helpers": helpers, "error": f"{type(ex).__name__}: {ex}"[:300]}
-                finally:
+                rec_k = {"helpers": helpers}
+                for mode in ("fused", "copy"):  # SM pull over NVLink with the fused check / peer copies + hash
                     try:
-                        sw.set_helpers([])
-                        sw.set_mechanism(args.mechanism)
-                    except Exception:  # noqa: BLE001
-                        pass
+                        if mode == "copy":
+                            os.environ["SWAP_ASSIST"] = "copy"
+                        else:
+                            os.environ.pop("SWAP_ASSIST", None)
+                        sw.set_mechanism("ce_pipe")
+                        sw.set_helpers(helpers)
+                        ts = []
+                        for _ in range(3):
+                            poison()
+                            stream.synchronize()
+                            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                            e0.record(stream)
+                            sw.restore(stream)
+                            res = sw.verify(stream, hbm_pass=True)
+                            e1.record(stream)
+                            e1.synchronize()
+                            assert res["status"] == 0 and res["n_bad"] == 0 and res["hbm_n_bad"] == 0, res
+                            ts.append(e0.elapsed_time(e1) * 1e-3)
+                        t = statistics.median(ts[1:])
+                        rec_k[mode] = {"swap_in_s": round(t, 4), "GBps": round(payload / t / GB, 2),
+                                       "frac_of_k_plus_1_links": round(payload / t / GB / ((k + 1) * ce["h2d"]), 3)}
+                    except Exception as ex:  # noqa: BLE001 - an informational leg must not sink the line
+                        rec_k[mode] = {"error": f"{type(ex).__name__}: {ex}"[:300]}
+                    finally:
+                        os.environ.pop("SWAP_ASSIST", None)
+                        try:
+                            sw.set_helpers([])
+                            sw.set_mechanism(args.mechanism)
+                        except Exception:  # noqa: BLE001
+                            pass
+                assisted[str(k)] = rec_k
             barrier()
 
     cpu = None
