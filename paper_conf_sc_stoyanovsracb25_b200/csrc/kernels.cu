@@ -316,37 +316,55 @@ __device__ __forceinline__ void move_segment(const Params& p, const SegDesc& d, 
   constexpr bool COPY = (MODE == GATHER || MODE == SCATTER);
 
   if (KIND == KIND_XXH64) {
-    // acc lanes 0..3 hold v1..v4 (seed 0).
-    uint64_t acc = lane == 0 ? P1 + P2 : lane == 1 ? P2 : lane == 2 ? 0ull : 0ull - P1;
+    // acc lanes 0..3 carry the chains v1..v4 in t-form (xt_step). Software pipeline: the loads of the next
+    // UX blocks are issued before the current blocks are stored and hashed, so the chunk's serial round
+    // chain overlaps its host-link latency (round 1 loaded, stored, then hashed: the warp idled on each).
+    constexpr int UX = 8;
+    uint64_t acc = xt_init(lane & 3);
     const int half = (lane & 3) >> 1;
-    uint32_t b = 0;
-    for (; b < nblk; b += U) {
-      const uint32_t nb = nblk - b < (uint32_t)U ? nblk - b : (uint32_t)U;
-      int4 v[U];
+    auto load = [&](int4 (&v)[UX], uint32_t b, uint32_t nb) {
 #pragma unroll
-      for (int u = 0; u < U; ++u)
+      for (int u = 0; u < UX; ++u)
         if (u < (int)nb) v[u] = ld_stream(src + (size_t)(b + u) * 512 + lane * 16);
+    };
+    auto consume = [&](const int4 (&v)[UX], uint32_t b, uint32_t nb) {
       if (COPY) {
 #pragma unroll
-        for (int u = 0; u < U; ++u)
+        for (int u = 0; u < UX; ++u)
           if (u < (int)nb) st_stream(dst + (size_t)(b + u) * 512 + lane * 16, v[u]);
       }
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
+      for (int u = 0; u < UX; ++u) {
         if (u < (int)nb) {
           const uint64_t lo = (uint64_t)(uint32_t)v[u].x | ((uint64_t)(uint32_t)v[u].y << 32);
           const uint64_t hi = (uint64_t)(uint32_t)v[u].z | ((uint64_t)(uint32_t)v[u].w << 32);
 #pragma unroll
-          for (int s = 0; s < 16; ++s) {
+          for (int s = 0; s < 16; ++s) {  // stripe s of the block: lanes 2s, 2s+1 hold its 4 words
             const int srcl = 2 * s + half;
             const uint64_t wlo = __shfl_sync(0xffffffffu, lo, srcl);
             const uint64_t whi = __shfl_sync(0xffffffffu, hi, srcl);
             const uint64_t w = (lane & 1) ? whi : wlo;
-            if (lane < 4) acc = xround(acc, w);
+            if (lane < 4) acc = xt_step(acc, w);
           }
         }
       }
+    };
+    int4 va[UX], vb[UX];
+    uint32_t b = 0, nb = nblk < (uint32_t)UX ? nblk : (uint32_t)UX;
+    load(va, 0, nb);
+    while (b < nblk) {  // two batches per iteration: va / vb ping-pong, no register copies
+      uint32_t b2 = b + nb, nb2 = b2 < nblk ? min((uint32_t)UX, nblk - b2) : 0u;
+      load(vb, b2, nb2);
+      consume(va, b, nb);
+      if (!nb2) break;
+      const uint32_t b3 = b2 + nb2, nb3 = b3 < nblk ? min((uint32_t)UX, nblk - b3) : 0u;
+      load(va, b3, nb3);
+      consume(vb, b2, nb2);
+      b = b3;
+      nb = nb3;
+      if (!nb) break;
     }
+    acc = xt_final(acc);
     const uint32_t r = len - nblk * 512u;
     const uint64_t base = (uint64_t)nblk * 512u;
     stage_tail<MODE>(src + base, COPY ? dst + base : nullptr, r, tail, lane);
@@ -445,8 +463,10 @@ struct SmemLayout {
   static constexpr size_t bytes = off_tail + (size_t)WARPS * TAIL_BYTES;
 };
 
+// XXH64 movers run one CTA per SM (launch_mover / movers.cpp size their grid to the SM count): a warp
+// per chunk, and the software-pipelined register double buffer of move_segment needs up to 128 registers.
 template <int MODE, int KIND>
-__global__ void __launch_bounds__(THREADS, 2) mover_kernel(const Params p) {
+__global__ void __launch_bounds__(THREADS, KIND == KIND_XXH64 ? 1 : 2) mover_kernel(const Params p) {
   using L = SmemLayout<KIND>;
   extern __shared__ __align__(128) uint8_t smem[];
   uint32_t* sT = reinterpret_cast<uint32_t*>(smem);
@@ -457,6 +477,17 @@ __global__ void __launch_bounds__(THREADS, 2) mover_kernel(const Params p) {
 
   if (KIND == KIND_CRC32C)
     for (int i = tid; i < L::tab_words; i += THREADS) sT[i] = __ldg(p.tables + i);
+
+  if (KIND == KIND_XXH64) {
+    // a descriptor is a whole chunk, one warp's long serial job: warps take chunks interleaved across
+    // CTAs (chunk w * grid + cta first), so a few chunks spread over as many SMs as possible, and no CTA
+    // barrier ties a warp to the slowest one of its round; the descriptor is read directly (no staging)
+    for (uint32_t idx = warp * gridDim.x + blockIdx.x; idx < p.n_desc; idx += gridDim.x * WARPS) {
+      const SegDesc d = p.desc[idx];
+      move_segment<MODE, KIND>(p, d, idx, sT, tail, lane);
+    }
+    return;
+  }
 
   const uint32_t per_round = gridDim.x * WARPS;
   const uint32_t first0 = blockIdx.x * WARPS;
