@@ -2,6 +2,7 @@
 // the ABI (swap_abi.cpp), the movers (movers.cpp) and the exchange / assisted restore (exchange.cpp).
 #pragma once
 #include <cstdint>
+#include <memory>
 #include <string>
 #include <vector>
 
@@ -46,7 +47,8 @@ struct DescSet {
   std::vector<size_t> ce_bytes;
   std::vector<Group> groups;              // CE_PIPE
   std::vector<cudaEvent_t> group_ev;
-  std::vector<swk::SegDesc> h_desc;       // host copy of d_desc (the fused peer pull rewrites sources)
+  // host copy of d_desc (the fused pulls rewrite sources); shared, so aliases of a set do not copy it
+  std::shared_ptr<const std::vector<swk::SegDesc>> h_desc;
   bool owned = false;                     // false: an alias of another set
 };
 

@@ -236,7 +236,7 @@ swap_status swap_set_helpers(swap_ctx_t* c, const int* devices, int n) {
       cudaGetLastError();
     }
   const DescSet& S = c->s_move;
-  std::vector<swk::SegDesc> d = S.h_desc;
+  std::vector<swk::SegDesc> d = S.h_desc ? *S.h_desc : std::vector<swk::SegDesc>();
   const size_t H = c->helpers.size();
   for (size_t gi = 0; gi < S.groups.size(); ++gi) {
     const size_t k = gi % (H + 1);
@@ -272,12 +272,13 @@ swap_status swap_pull_stripes(swap_ctx_t* c, uint32_t stripe, uint32_t n_stripes
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
   const DescSet& S = c->s_move;
   std::vector<swk::SegDesc> d;
-  d.reserve(S.h_desc.size());
+  if (!S.h_desc) return SWAP_OK;
+  d.reserve(S.h_desc->size());
   for (size_t gi = 0; gi < S.groups.size(); ++gi) {
     const uint32_t o = (uint32_t)(gi % n_stripes);
     if (o == stripe) continue;
     for (uint32_t i = S.groups[gi].d0; i < S.groups[gi].d1; ++i) {
-      swk::SegDesc x = S.h_desc[i];
+      swk::SegDesc x = (*S.h_desc)[i];
       x.host = (uint64_t)((int64_t)x.dev + peer_delta[o]);
       d.push_back(x);
     }

@@ -418,7 +418,7 @@ static swap_status build_set(swap_ctx* c, DescSet* S, Pick pick, bool zero_src) 
     CUDA_TRY(c, cudaMemcpy(S->d_desc, desc.data(), desc.size() * sizeof(swk::SegDesc), cudaMemcpyHostToDevice));
   S->group_ev.assign(S->groups.size(), nullptr);
   for (auto& e : S->group_ev) CUDA_TRY(c, cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-  S->h_desc = std::move(desc);
+  S->h_desc = std::make_shared<const std::vector<swk::SegDesc>>(std::move(desc));
   return SWAP_OK;
 }
 
