@@ -782,7 +782,17 @@ def run_ours(args):
             "restore_GBps_per_gpu": round(achieved, 3),
             "restore_GBps_per_gpu_slowest": round(payload / (max(restore_steps) * 1e-3) / GB, 3),
             "checkpoint_GBps_per_gpu": round(payload / (ckpt_ms * 1e-3) / GB, 3),
-            "roofline": {"bound": "host_link", "kernel": RESTORE_KERNEL[eff_mech],
+            # the dominant kernel of the timed region (ncu launch list, profiles/r02_ncu_launches_bench_B.md) is the
+            # HBM hash kernel: per-group restore checks + the a8 verify pass; its launch is timed live as the verify
+            "roofline": {"bound": "hbm", "kernel": VERIFY_KERNEL[args.checksum],
+                         "achieved": round(payload / (verify_ms * 1e-3) / GB, 1), "peak": hbm_peak,
+                         "unit": "GB/s", "frac": round(payload / (verify_ms * 1e-3) / GB / hbm_peak, 4),
+                         "traffic": (ncu_traffic(name, args.checksum, payload) or {}).get("bytes"),
+                         "algorithmic_bytes_per_launch": payload,
+                         "how": "payload bytes (1 B HBM read per image byte) / the verify launch's mean duration "
+                                "(CUDA events on the ctx stream over the timed steps)",
+                         "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy; a read-only stream can exceed it)"},
+            "roofline_link": {"bound": "host_link", "kernel": RESTORE_KERNEL[eff_mech],
                          "achieved": round(achieved, 3), "peak": PCIE_GEN5_X16_GBPS, "unit": "GB/s",
                          "frac": round(achieved / PCIE_GEN5_X16_GBPS, 4), "traffic": None,
                          "traffic_note": "copy-engine / link transfer: no kernel DRAM counters (see roofline_verify.traffic)",
