@@ -110,6 +110,7 @@ struct swap_ctx {
   uint32_t stripe = 0, n_stripes = 1;  // CE_PIPE restore groups this restore moves (swap_restore_stripe)
   swk::SegDesc* d_pull = nullptr;      // descriptors of the last swap_pull_stripes (sources in peer HBM)
   size_t pull_cap = 0;
+  cudaEvent_t ev_pull = nullptr;       // recorded after the last pull kernel (d_pull reuse waits for it)
   int numa_node = -1;         // NUMA node the image placement targeted (-1: none)
   double numa_local = 1.0;    // sampled share of image pages on numa_node
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;

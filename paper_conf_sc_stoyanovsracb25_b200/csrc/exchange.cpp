@@ -284,8 +284,12 @@ swap_status swap_pull_stripes(swap_ctx_t* c, uint32_t stripe, uint32_t n_stripes
     }
   }
   if (d.empty()) return SWAP_OK;
+  if (c->ev_pull) CUDA_TRY(c, cudaStreamWaitEvent(s, c->ev_pull, 0));  // a previous pull may still read d_pull
   if (d.size() > c->pull_cap) {
-    if (c->d_pull) cudaFree(c->d_pull);
+    if (c->d_pull) {
+      CUDA_TRY(c, cudaStreamSynchronize(s));
+      cudaFree(c->d_pull);
+    }
     c->d_pull = nullptr;
     c->pull_cap = 0;
     CUDA_TRY(c, cudaMalloc(&c->d_pull, d.size() * sizeof(swk::SegDesc)));
@@ -296,7 +300,11 @@ swap_status swap_pull_stripes(swap_ctx_t* c, uint32_t stripe, uint32_t n_stripes
   swk::Params p = base_params(c, S);
   p.desc = c->d_pull;
   p.n_desc = (uint32_t)d.size();
-  return launch(c, swk::SCATTER, hash_kind(c), p, s);
+  swap_status st = launch(c, swk::SCATTER, hash_kind(c), p, s);
+  if (st != SWAP_OK) return st;
+  if (!c->ev_pull) CUDA_TRY(c, cudaEventCreateWithFlags(&c->ev_pull, cudaEventDisableTiming));
+  CUDA_TRY(c, cudaEventRecord(c->ev_pull, s));
+  return SWAP_OK;
 }
 
 namespace {

@@ -336,6 +336,8 @@ void release(swap_ctx* c) {
   if (c->d_pull) cudaFree(c->d_pull);
   c->d_pull = nullptr;
   c->pull_cap = 0;
+  if (c->ev_pull) cudaEventDestroy(c->ev_pull);
+  c->ev_pull = nullptr;
   if (c->d_arrive) cudaFree(c->d_arrive);
   if (c->d_status) cudaFree(c->d_status);
   if (c->h_status) cudaFreeHost(c->h_status);
