@@ -89,6 +89,15 @@ def test_null_args(swp):
     assert L.swap_restore(None, None) == swp.SWAP_EINVAL
     assert L.swap_verify(None, None, 1, None) == swp.SWAP_EINVAL
     assert L.swap_sync(None, None) == swp.SWAP_EINVAL
+    # round-2 entry points: argument checks come first and need no device
+    assert L.swap_get_mechanism_dir(None, 0, None) == swp.SWAP_EINVAL
+    assert L.swap_get_numa(None, None, None) == swp.SWAP_EINVAL
+    assert L.swap_restore_stripe(None, 0, 2, None) == swp.SWAP_EINVAL
+    assert L.swap_pull_stripes(None, 0, 2, None, None) == swp.SWAP_EINVAL
+    assert L.swap_get_restore_spans(None, None, 0, None) == swp.SWAP_EINVAL
+    assert L.swap_ipc_export(0, None, None, None) == swp.SWAP_EINVAL
+    assert L.swap_ipc_import(0, None, 0, None, None) == swp.SWAP_EINVAL
+    assert L.swap_ipc_close(0, None) == swp.SWAP_EINVAL
 
 
 SUM = struct.Struct("<IIIIQQQQQQ")
