@@ -55,7 +55,7 @@ def _worker(rank, world, init_file, q):
             # flips in replica 1's image: one in a group replica 1 owns, one in a group replica 0 owns
             img = sw.image()
             own1 = next(sp for sp in spans if sp[0] % world == 1)
-            own0 = next(sp for sp in spans if sp[0] % world == 0)
+            own0 = next(sp for sp in spans if sp[0] % world == 0)  # replica 0's stripe
             p1, p0 = own1[2] + own1[3] // 2, own0[2] + own0[3] // 2
             chunk_of = {}
             for pos in (p1, p0):  # the chunk holding image offset pos, from the oracle manifest
@@ -99,9 +99,9 @@ def _worker(rank, world, init_file, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.timeout(300)
-def test_two_replicas_striped_restore():
-    world = 2
+@pytest.mark.timeout(400)
+@pytest.mark.parametrize("world", [2, 3])
+def test_replicas_striped_restore(world):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     with tempfile.TemporaryDirectory() as d:
@@ -115,16 +115,18 @@ def test_two_replicas_striped_restore():
             assert p.exitcode == 0
     for r in range(world):
         assert "error" not in res[r], res[r].get("error")
-        assert res[r]["image_equal"] and res[r]["spans_cover"] and res[r]["n_groups"] >= 4
+        assert res[r]["image_equal"] and res[r]["spans_cover"] and res[r]["n_groups"] >= 2 * world
         assert res[r]["clean"] == (0, 0, 1) and res[r]["mem_equal"]
     g = res[1]["flip_chunk"]
-    # replica 1 moved the flipped chunk itself (fused check) and broadcast it: both HBM passes see it;
+    # replica 1 moved the flipped chunk itself (fused check) and broadcast it: every HBM pass sees it;
     # the flip in replica 0's stripe was never read
     assert res[1]["flip"] == (1, g, 1, g)
-    assert res[0]["flip"] == (0, (1 << 64) - 1, 1, g)
-    # fused pull: replica 0's pull kernel checks the chunk it read from replica 1's HBM
+    for r in range(world):
+        if r != 1:
+            assert res[r]["flip"] == (0, (1 << 64) - 1, 1, g), r
+            # fused pull: replica r's pull kernel checks the chunk it read from replica 1's HBM
+            assert res[r]["pull_flip"] == (1, g, 1, g), r
     assert res[1]["pull_flip"] == (1, g, 1, g)
-    assert res[0]["pull_flip"] == (1, g, 1, g)
     for r in range(world):
         assert res[r]["pull_clean"] == (0, 0, 1) and res[r]["pull_mem_equal"], r
 
