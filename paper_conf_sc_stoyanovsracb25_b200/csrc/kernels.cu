@@ -538,25 +538,53 @@ __global__ void __launch_bounds__(THREADS, KIND == KIND_XXH64 ? 1 : 2) mover_ker
 // wavefronts (the r1 contiguous-run layout needed 32 + 32).
 constexpr int HT_THREADS = 1024;
 constexpr int HT_WARPS = HT_THREADS / 32;
-// Shared layout, in absolute shared-window addresses. Dynamic shared memory starts at 0x400 on sm_100 (the
-// first KiB of the CTA window is reserved; tools/probe_smem_base.cu measures it) and the kernel traps if it
-// does not, so the tables' alignment costs no padding: descriptors + mbarriers at 0x400, the Z^96 nibble
-// tables at 0x1000 (8 x 16 entries x 32 lanes, 16 KiB, 2-KiB aligned), the four slicing tables at 0x8000
-// (table k at 0x8000 + k*32 KiB, entry e of lane l at + e*128 + l*4: 32-KiB aligned, so a lookup address
-// is (index << 7) | (0x8000 + 4*lane) plus an immediate table offset: one shift + one LOP3). Variant ZB
-// adds Z^96 *byte* tables at 0x28000 (4 x 256 entries x 16 copies, lanes l and l+16 share copy l&15:
-// entry e of copy c at word e*16 + c, 16-KiB aligned) and drops the nibble tables.
-constexpr uint32_t HT_SMEM_BASE = 0x400;
-constexpr uint32_t HT_A_DESC = 0x400;
-constexpr uint32_t HT_A_BAR = HT_A_DESC + 2 * HT_WARPS * 32;  // 2 rounds x 32 descriptors x 32 B
-constexpr uint32_t HT_A_ZN = 0x1000;
-constexpr uint32_t HT_A_TAB = 0x8000;
-constexpr uint32_t HT_TAB_BYTES = 4 * 256 * 128;
-constexpr uint32_t HT_A_ZB = HT_A_TAB + HT_TAB_BYTES;          // 0x28000
-constexpr uint32_t HT_ZB_BYTES = 4 * 256 * 16 * 4;              // 64 KiB
-template <bool ZB>
-constexpr size_t ht_smem() { return (ZB ? HT_A_ZB + HT_ZB_BYTES : HT_A_TAB + HT_TAB_BYTES) - HT_SMEM_BASE; }
-static_assert(HT_A_BAR + 16 <= HT_A_ZN && HT_A_ZN + 8 * 16 * 128 <= HT_A_TAB, "hash kernel shared layout");
+// Shared layout, in shared-window addresses derived from the dynamic-shared-memory base R (measured once per
+// device by smem_base_probe; 0x400 on sm_100, the first KiB of the CTA window being reserved): descriptors +
+// mbarriers at R, the Z^96 nibble tables (8 x 16 entries x 32 lanes, 16 KiB) at the next 2-KiB boundary, the
+// four slicing tables at the next 32-KiB boundary (table k at +k*32 KiB, entry e of lane l at + e*128 + l*4,
+// so a lookup address is (index << 7) | (base + 4*lane) plus an immediate table offset: one shift + one
+// LOP3). Variant ZB adds Z^96 *byte* tables after the slicing tables (4 x 256 entries x 16 copies, lanes l
+// and l+16 share copy l&15: entry e of copy c at word e*16 + c) instead of the nibble tables. With R = 0x400
+// nothing is padded: nibble tables at 0x1000, slicing tables at 0x8000.
+struct HtLayout {
+  uint32_t desc, bar, zn, tab, zb, end;
+};
+__host__ __device__ constexpr uint32_t ht_align(uint32_t v, uint32_t a) { return (v + a - 1) / a * a; }
+__host__ __device__ inline HtLayout ht_layout(uint32_t R, bool zb) {
+  HtLayout L{};
+  L.desc = R;
+  L.bar = R + 2 * HT_WARPS * 32;  // 2 rounds x 32 descriptors x 32 B
+  L.zn = ht_align(L.bar + 16, 2048);
+  L.tab = ht_align(L.zn + 8 * 16 * 128, 32768);
+  L.zb = L.tab + 4 * 256 * 128;
+  L.end = zb ? L.zb + 4 * 256 * 16 * 4 : L.zb;
+  return L;
+}
+__global__ void smem_base_probe(uint32_t* out) {
+  extern __shared__ __align__(128) uint8_t s[];
+  if (threadIdx.x == 0) *out = static_cast<uint32_t>(__cvta_generic_to_shared(s));
+}
+// The dynamic-shared-memory base of this device's kernels (cached per device; swap_create probes it so
+// that no launch pays the probe's synchronising cudaMalloc / cudaFree).
+static cudaError_t smem_base(uint32_t* R) {
+  static uint32_t cache[64] = {};
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (!cache[dev & 63]) {
+    uint32_t* d = nullptr;
+    if ((e = cudaMalloc(&d, 4)) != cudaSuccess) return e;
+    smem_base_probe<<<1, 32, 128>>>(d);
+    uint32_t h = 0;
+    e = cudaMemcpy(&h, d, 4, cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    if (e != cudaSuccess) return e;
+    cache[dev & 63] = h ? h : 1;  // 0 (no reservation) stored as 1 (a 0 base aligns to itself)
+  }
+  *R = cache[dev & 63] == 1 ? 0 : cache[dev & 63];
+  return cudaSuccess;
+}
+static_assert(ht_align(0x400 + 2 * HT_WARPS * 32 + 16, 2048) == 0x1000, "hash kernel shared layout at R = 0x400");
 
 __device__ __forceinline__ void ld32(const uint8_t* p, uint32_t (&w)[8]) {
   asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
@@ -690,11 +718,11 @@ template <int MODE, bool ZB, bool B0F>
 __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
-  if (raw != HT_SMEM_BASE) __trap();  // the layout below assumes dynamic shared memory at 0x400
-  uint8_t* smem = smem_raw - HT_SMEM_BASE;  // generic pointer of shared address 0
-  uint32_t* sT = reinterpret_cast<uint32_t*>(smem + HT_A_TAB);
-  SegDesc* sDesc = reinterpret_cast<SegDesc*>(smem + HT_A_DESC);
-  uint64_t* sBar = reinterpret_cast<uint64_t*>(smem + HT_A_BAR);
+  const HtLayout HL = ht_layout(raw, ZB);  // the host sized the allocation for this base (smem_base)
+  uint8_t* smem = smem_raw - raw;  // generic pointer of shared address 0
+  uint32_t* sT = reinterpret_cast<uint32_t*>(smem + HL.tab);
+  SegDesc* sDesc = reinterpret_cast<SegDesc*>(smem + HL.desc);
+  uint64_t* sBar = reinterpret_cast<uint64_t*>(smem + HL.bar);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 
   // replicate T0..T3 (the first four slicing tables) once per lane, and the Z^96 tables
@@ -705,7 +733,7 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
     for (int r = 0; r < 8; ++r) dst[r] = make_uint4(v, v, v, v);
   }
   if (ZB) {
-    uint32_t* sZ = reinterpret_cast<uint32_t*>(smem + HT_A_ZB);
+    uint32_t* sZ = reinterpret_cast<uint32_t*>(smem + HL.zb);
     for (int i = tid; i < 4 * 256; i += HT_THREADS) {
       const uint32_t v = __ldg(p.tables + TAB_Z96B + i);
       uint4* dst = reinterpret_cast<uint4*>(sZ + (size_t)i * 16);
@@ -713,7 +741,7 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
       for (int r = 0; r < 4; ++r) dst[r] = make_uint4(v, v, v, v);
     }
   } else {
-    uint32_t* sZ = reinterpret_cast<uint32_t*>(smem + HT_A_ZN);
+    uint32_t* sZ = reinterpret_cast<uint32_t*>(smem + HL.zn);
     for (int i = tid; i < 8 * 16; i += HT_THREADS) {
       const uint32_t v = __ldg(p.tables + TAB_Z96N + i);
       uint4* dst = reinterpret_cast<uint4*>(sZ + (size_t)i * 32);
@@ -740,8 +768,8 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
     if (rounds > 1) issue(1);
   }
   __syncthreads();
-  const uint32_t lb = HT_A_TAB + 4u * lane;
-  const uint32_t lz = ZB ? HT_A_ZB + 4u * (lane & 15) : HT_A_ZN + 4u * lane;
+  const uint32_t lb = HL.tab + 4u * lane;
+  const uint32_t lz = ZB ? HL.zb + 4u * (lane & 15) : HL.zn + 4u * lane;
   const uint32_t m128 = blockDim.x >> 3;  // = 128 (HT_THREADS = 1024), opaque to ptxas
   const uint32_t* x2n = p.tables + TAB_X2N;
 
@@ -777,18 +805,26 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
   }
 }
 
+cudaError_t probe_smem_base() {
+  uint32_t R = 0;
+  return smem_base(&R);
+}
+
 template <int MODE, bool ZB, bool B0F>
 static cudaError_t launch_hash_t(const Params& p, int grid, cudaStream_t s) {
   static unsigned long long attr_set = 0;
-  int dev = 0;
-  cudaError_t e = cudaGetDevice(&dev);
+  uint32_t R = 0;
+  cudaError_t e = smem_base(&R);
   if (e != cudaSuccess) return e;
+  const size_t bytes = ht_layout(R, ZB).end - R;
+  int dev = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
   if (!((attr_set >> (dev & 63)) & 1ull)) {
-    e = cudaFuncSetAttribute(hash_kernel<MODE, ZB, B0F>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ht_smem<ZB>());
+    e = cudaFuncSetAttribute(hash_kernel<MODE, ZB, B0F>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
     if (e != cudaSuccess) return e;
     attr_set |= 1ull << (dev & 63);
   }
-  hash_kernel<MODE, ZB, B0F><<<grid, HT_THREADS, ht_smem<ZB>(), s>>>(p);
+  hash_kernel<MODE, ZB, B0F><<<grid, HT_THREADS, bytes, s>>>(p);
   return cudaGetLastError();
 }
 

@@ -86,6 +86,9 @@ uint32_t host_multmodp(uint32_t a, uint32_t b);
 // Launch mover kernel <mode, kind> with `grid` CTAs on `stream`.
 cudaError_t launch_mover(int mode, int kind, const Params& p, int grid, cudaStream_t stream);
 int mover_threads();
+// Measures (once per device) where kernels' dynamic shared memory starts; the CRC hash kernel's table
+// layout is derived from it. Called by swap_create.
+cudaError_t probe_smem_base();
 // Grid for the CRC HBM hash kernel (1 CTA of 1024 threads per SM, 128 KB tables).
 int hash_grid(int sm_count, uint32_t n_desc);
 size_t mover_smem_bytes(int kind);

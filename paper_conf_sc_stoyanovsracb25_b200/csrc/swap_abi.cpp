@@ -69,7 +69,8 @@ swap_status swap_create(const swap_config_t* cfg_in, swap_ctx_t** out) {
       (e = cudaHostAlloc(&c->h_status, sizeof(swk::DevStatus), cudaHostAllocDefault)) != cudaSuccess ||
       (e = cudaEventCreate(&c->ev[0])) != cudaSuccess || (e = cudaEventCreate(&c->ev[1])) != cudaSuccess ||
       (e = cudaEventCreate(&c->ev[2])) != cudaSuccess || (e = cudaEventCreate(&c->ev[3])) != cudaSuccess ||
-      (e = cudaEventCreate(&c->ev[4])) != cudaSuccess || (e = cudaEventCreate(&c->ev[5])) != cudaSuccess) {
+      (e = cudaEventCreate(&c->ev[4])) != cudaSuccess || (e = cudaEventCreate(&c->ev[5])) != cudaSuccess ||
+      (e = swk::probe_smem_base()) != cudaSuccess) {
     cuda_fail(c, e, "swap_create");
     fprintf(stderr, "libswap: %s\n", c->err.c_str());
     release(c);
