@@ -213,7 +213,8 @@ SWAP_API swap_status swap_get_mechanism_dir(const swap_ctx_t* ctx, int direction
  * collective: dist.restore_replicas broadcasts each span from its owner with NCCL). Until that exchange
  * the other stripes' bytes on this device are stale; swap_verify(hbm_pass = 1) afterwards checks every
  * chunk against this ctx's manifest. Zero chunks (DISCARD, masks) are zero-filled in full on every replica.
- * n_stripes == 1 is swap_restore with CE_PIPE. EINVAL: stripe >= n_stripes, or helper devices are set.
+ * n_stripes == 1 is exactly swap_restore (AUTO mechanism). EINVAL: stripe >= n_stripes, n_stripes == 0, or
+ * helper devices are set together with n_stripes > 1.
  * State as swap_restore (-> RESTORED). */
 SWAP_API swap_status swap_restore_stripe(swap_ctx_t* ctx, uint32_t stripe, uint32_t n_stripes, swap_stream_t stream);
 
