@@ -693,13 +693,14 @@ def run_ours(args):
     # NVLink, HBM verify of everything) vs every replica pulling the whole image over its own link
     dp = None
     if multi and not args.no_dp:
-        dp_err, swd, arena0 = "", None, None
+        dp_err, swd, arena0, vmm0 = "", None, None, None
         try:  # local setup first; collectives only if every rank got this far
             _, specs0, _ = workload(args.config, 0, world)
             offs0, bytes0 = W.place(specs0)
-            arena0 = torch.empty(bytes0, dtype=torch.uint8, device=dev)
+            vmm0 = swap.Arena(bytes0, device=local_dev)  # the product's releasable HBM
+            base0, arena0 = vmm0.alloc(bytes0)
             W.fill_device_arena(arena0, specs0, offs0, seed=0)  # identical bytes on every replica
-            regions0 = [(arena0.data_ptr() + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs0, offs0))]
+            regions0 = [(base0 + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs0, offs0))]
             payload0 = sum(r.nbytes for r in specs0)
             swd = swap.Swapper(regions0, chunk_bytes=args.chunk, checksum=kind, mechanism="ce_pipe", device=local_dev)
             with torch.cuda.stream(stream):
@@ -737,11 +738,8 @@ def run_ours(args):
             with torch.cuda.stream(stream):
                 t_striped = timed(lambda: sdist.restore_replicas(swd, None, stream))
                 t_indep = timed(independent)
-                try:  # fused NVLink pull: CUDA IPC maps of the other replicas' arenas
-                    deltas, bases = sdist.map_replicas(arena0.data_ptr(), local_dev, None)
-                    t_pull = timed(lambda: sdist.pull_replicas(swd, deltas, None, stream))
-                    for b_ in bases:
-                        swap.ipc_close(local_dev, b_)
+                try:  # fused NVLink pull: the other replicas' VMM arenas mapped here (slab fds over Unix sockets)
+                    t_pull = timed(lambda: sdist.pull_replicas(swd, None, None, stream, arena=vmm0))
                 except Exception as ex:  # noqa: BLE001
                     t_pull = f"{type(ex).__name__}: {ex}"[:200]
             dp = {"replicas": world, "image_bytes": payload0, "striped_swap_in_s": round(t_striped, 4),
@@ -752,10 +750,13 @@ def run_ours(args):
                   "how": "swap_restore_stripe (1/N of the CE_PIPE groups per replica over its own PCIe link) + in-place "
                          "NCCL broadcasts of every stripe span from its owner + HBM verify of all chunks, max over ranks; "
                          "fused pull: the other stripes read from the owners' HBM over NVLink by the SM mover with the "
-                         "chunk check from the same registers (swap_pull_stripes), then the HBM verify"}
+                         "chunk check from the same registers (swap_pull_stripes; the peers' VMM arenas mapped per "
+                         "swap-in via exported slab fds, included in the time), then the HBM verify"}
         if swd is not None:
             swd.close()
         del arena0
+        if vmm0 is not None:
+            vmm0.close()
 
     if rank == 0:
         value = total_payload / (swapin_ms * 1e-3) / GB

@@ -361,6 +361,19 @@ SWAP_API swap_status swap_exchange(swap_ctx_t* const* victims, size_t n_victims,
                                    uint64_t* peak_extra);
 SWAP_API const char* swap_arena_last_error(const swap_arena_t* a);
 SWAP_API void swap_arena_destroy(swap_arena_t* a);
+/* Peer mapping of arenas (data-parallel replicas, NEXT-2): swap_arena_export writes one POSIX file
+ * descriptor per slab (the caller owns them: pass them to another process, e.g. over a Unix socket with
+ * SCM_RIGHTS, then close them) and the slab size; with fds == NULL it only reports *n. Every slab must be
+ * mapped (ESTATE otherwise); the descriptors stay valid for the slabs' current physical memory, so a
+ * released and re-acquired arena must be exported again. swap_arena_import maps such a set of slabs (total
+ * bytes = the exporter's arena size) into a fresh VA range on `device` with read-write access and returns it
+ * (the fds may be closed afterwards); swap_arena_unimport unmaps it. This is how swap_pull_stripes reads a
+ * replica's VMM arena. */
+typedef struct swap_arena_view swap_arena_view_t;
+SWAP_API swap_status swap_arena_export(swap_arena_t* a, int* fds, size_t cap, size_t* n, uint64_t* slab_bytes);
+SWAP_API swap_status swap_arena_import(int device, const int* fds, size_t n, uint64_t slab_bytes, uint64_t total_bytes,
+                                       swap_arena_view_t** out, uint64_t* dev_addr);
+SWAP_API void swap_arena_unimport(swap_arena_view_t* v);
 
 /* ---------------------------------------------------------------------------------------------
  * Task manager (NEXT-1): memory reservations and demand-aware preemption, host-only.

@@ -12,6 +12,7 @@
 #include <cuda_runtime.h>
 
 #include <cstring>
+#include <unistd.h>
 #include <string>
 #include <vector>
 
@@ -29,6 +30,8 @@ struct Drv {
   decltype(&cuMemMap) map = nullptr;
   decltype(&cuMemUnmap) unmap = nullptr;
   decltype(&cuMemSetAccess) set_access = nullptr;
+  decltype(&cuMemExportToShareableHandle) export_h = nullptr;    // optional (peer import of arenas)
+  decltype(&cuMemImportFromShareableHandle) import_h = nullptr;  // optional
   bool ok = false;
 };
 
@@ -50,6 +53,8 @@ const Drv& drv() {
            resolve("cuMemAddressFree", &x.addr_free) && resolve("cuMemCreate", &x.create) &&
            resolve("cuMemRelease", &x.release) && resolve("cuMemMap", &x.map) && resolve("cuMemUnmap", &x.unmap) &&
            resolve("cuMemSetAccess", &x.set_access);
+    resolve("cuMemExportToShareableHandle", &x.export_h);
+    resolve("cuMemImportFromShareableHandle", &x.import_h);
     return x;
   }();
   return d;
@@ -86,6 +91,9 @@ swap_status map_slab(swap_arena* a, uint64_t i) {
   prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
   prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
   prop.location.id = a->device;
+  // slabs can be exported as POSIX file descriptors (swap_arena_export: data-parallel replicas map each
+  // other's arenas for the fused NVLink pull)
+  prop.requestedHandleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
   CUmemAccessDesc acc;
   std::memset(&acc, 0, sizeof(acc));
   acc.location = prop.location;
@@ -225,6 +233,106 @@ swap_status swap_arena_reacquire_range(swap_arena_t* a, uint64_t offset, uint64_
     if (st != SWAP_OK) return st;
   }
   return SWAP_OK;
+}
+
+swap_status swap_arena_export(swap_arena_t* a, int* fds, size_t cap, size_t* n, uint64_t* slab_bytes) {
+  if (!a || !n || (cap && !fds)) return SWAP_EINVAL;
+  *n = n_slabs(a);
+  if (slab_bytes) *slab_bytes = kSlab;
+  if (!fds) return SWAP_OK;
+  if (cap < *n) return SWAP_EINVAL;
+  if (!a->resident) {
+    a->err = "swap_arena_export needs every slab mapped (re-acquire first)";
+    return SWAP_ESTATE;
+  }
+  const Drv& D = drv();
+  if (!D.export_h) return SWAP_EUNSUPPORTED;
+  CtxGuard g(a->device);
+  for (uint64_t i = 0; i < *n; ++i) {
+    int fd = -1;
+    const CUresult r = D.export_h(&fd, a->slabs[i], CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR, 0);
+    if (r != CUDA_SUCCESS) {
+      for (uint64_t k = 0; k < i; ++k) close(fds[k]);
+      a->err = "cuMemExportToShareableHandle failed (" + std::to_string((int)r) + ")";
+      return SWAP_ECUDA;
+    }
+    fds[i] = fd;
+  }
+  return SWAP_OK;
+}
+
+// A peer arena mapped into this process: reserved VA + imported slabs.
+struct swap_arena_view {
+  int device = 0;
+  CUdeviceptr base = 0;
+  uint64_t bytes = 0;
+  struct Slab {
+    CUmemGenericAllocationHandle h;
+    uint64_t off, size;
+  };
+  std::vector<Slab> slabs;
+};
+
+void swap_arena_unimport(swap_arena_view_t* v);
+
+swap_status swap_arena_import(int device, const int* fds, size_t n, uint64_t slab_bytes, uint64_t total_bytes,
+                              swap_arena_view_t** out, uint64_t* dev_addr) {
+  if (!fds || !out || !dev_addr || n == 0 || slab_bytes == 0 || total_bytes == 0 ||
+      (total_bytes + slab_bytes - 1) / slab_bytes != n)
+    return SWAP_EINVAL;
+  *out = nullptr;
+  CtxGuard g(device);
+  const Drv& D = drv();
+  if (!D.ok || !D.import_h) return SWAP_EUNSUPPORTED;
+  auto* v = new (std::nothrow) swap_arena_view();
+  if (!v) return SWAP_ENOMEM;
+  v->device = device;
+  v->bytes = total_bytes;
+  if (D.reserve(&v->base, total_bytes, slab_bytes, 0, 0) != CUDA_SUCCESS) {
+    delete v;
+    return SWAP_ENOMEM;
+  }
+  CUmemAccessDesc acc;
+  std::memset(&acc, 0, sizeof(acc));
+  acc.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  acc.location.id = device;
+  acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+  for (size_t i = 0; i < n; ++i) {
+    const uint64_t off = i * slab_bytes, sz = total_bytes - off < slab_bytes ? total_bytes - off : slab_bytes;
+    CUmemGenericAllocationHandle h;
+    void* fd_as_handle = reinterpret_cast<void*>(static_cast<uintptr_t>(fds[i]));
+    if (D.import_h(&h, fd_as_handle, CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR) != CUDA_SUCCESS) {
+      swap_arena_unimport(v);
+      return SWAP_ECUDA;
+    }
+    if (D.map(v->base + off, sz, 0, h, 0) != CUDA_SUCCESS) {
+      D.release(h);
+      swap_arena_unimport(v);
+      return SWAP_ECUDA;
+    }
+    v->slabs.push_back(swap_arena_view::Slab{h, off, sz});
+    if (D.set_access(v->base + off, sz, &acc, 1) != CUDA_SUCCESS) {
+      swap_arena_unimport(v);
+      return SWAP_ECUDA;
+    }
+  }
+  *out = v;
+  *dev_addr = (uint64_t)v->base;
+  return SWAP_OK;
+}
+
+void swap_arena_unimport(swap_arena_view_t* v) {
+  if (!v) return;
+  {
+    CtxGuard g(v->device);
+    const Drv& D = drv();
+    for (const auto& sl : v->slabs) {
+      D.unmap(v->base + sl.off, sl.size);
+      D.release(sl.h);
+    }
+    if (v->base) D.addr_free(v->base, v->bytes);
+  }
+  delete v;
 }
 
 const char* swap_arena_last_error(const swap_arena_t* a) { return a ? a->err.c_str() : "null arena"; }

@@ -19,7 +19,12 @@ from __future__ import annotations
 import torch
 import torch.distributed as dist
 
-from .swap import SWAP_OK, SwapError, Swapper, ipc_export, ipc_import, swap_merge_global
+import os
+import socket
+import tempfile
+import threading
+
+from .swap import Arena, SWAP_OK, SwapError, Swapper, arena_import, ipc_export, ipc_import, swap_merge_global
 
 
 def _comm_device(group=None) -> torch.device:
@@ -106,20 +111,101 @@ def map_replicas(local_ptr: int, device: int, group=None) -> tuple[list[int], li
     return deltas, bases
 
 
-def pull_replicas(sw: Swapper, peer_delta: list[int], group=None, stream=None) -> dict:
+def _exchange_fds(my_fds: list[int], group=None) -> dict[int, list[int]]:
+    """Every rank sends its file descriptors to every other rank over Unix-domain sockets (SCM_RIGHTS;
+    the rendezvous paths travel through torch.distributed); returns {peer rank: its fds, now valid here}."""
+    k, r = dist.get_world_size(group), dist.get_rank(group)
+    path = os.path.join(tempfile.gettempdir(), f"swapserve-{os.getpid()}-{r}-{id(my_fds)}.sock")
+    srv = socket.socket(socket.AF_UNIX, socket.SOCK_STREAM)
+    srv.bind(path)
+    srv.listen(max(1, k - 1))
+    got: dict[int, list[int]] = {}
+
+    def accept_all():
+        for _ in range(k - 1):
+            conn, _ = srv.accept()
+            with conn:
+                fds, peer, expect = [], None, None
+                while expect is None or len(fds) < expect:
+                    msg, part, _, _ = socket.recv_fds(conn, 64, 253)
+                    if not msg:
+                        break
+                    peer, expect = (int(x) for x in msg.decode().split(":")[:2])
+                    fds.extend(part)
+                got[peer] = fds
+
+    t = threading.Thread(target=accept_all, daemon=True)
+    t.start()
+    paths = [None] * k
+    dist.all_gather_object(paths, path, group=group)
+    for o in range(k):
+        if o == r:
+            continue
+        with socket.socket(socket.AF_UNIX, socket.SOCK_STREAM) as c:
+            c.connect(paths[o])
+            for i in range(0, max(1, len(my_fds)), 200):  # SCM_RIGHTS carries at most 253 fds per message
+                socket.send_fds(c, [f"{r}:{len(my_fds)}:".encode()], my_fds[i:i + 200])
+    t.join()
+    srv.close()
+    os.unlink(path)
+    dist.barrier(group=group)
+    return got
+
+
+def map_replicas_arena(arena: Arena, group=None) -> tuple[list[int], list[int]]:
+    """map_replicas for VMM arenas (releasable HBM, swap.Arena): every replica exports its arena's slabs as
+    file descriptors (swap_arena_export), the descriptors are exchanged over Unix sockets, and each peer's
+    slabs are mapped here (swap_arena_import). The arena must be resident; after a release / re-acquire the
+    physical slabs are new, so map again. Returns (peer_delta, views to swap.arena_unimport)."""
+    k, r = dist.get_world_size(group), dist.get_rank(group)
+    fds, slab = arena.export()
+    try:
+        peers = _exchange_fds(fds, group)
+    finally:
+        for f in fds:
+            os.close(f)
+    sizes = [None] * k
+    dist.all_gather_object(sizes, arena.nbytes, group=group)
+    deltas, views = [], []
+    for o in range(k):
+        if o == r:
+            deltas.append(0)
+            continue
+        try:
+            view, addr = arena_import(arena.device, peers[o], slab, sizes[o])
+        finally:
+            for f in peers[o]:
+                os.close(f)
+        views.append(view)
+        deltas.append(addr - arena.base)
+    return deltas, views
+
+
+def pull_replicas(sw: Swapper, peer_delta: list[int] | None = None, group=None, stream=None,
+                  arena: Arena | None = None) -> dict:
     """Swap-in of k data-parallel replicas with the fused NVLink pull (NEXT-2): replica r restores its
     stripe over its own PCIe link (swap_restore_stripe); once every stripe has landed (barrier), one SM
     kernel per replica pulls the other stripes straight from the owners' HBM and checks every chunk from the
     registers that carried it (swap_pull_stripes); then the HBM verify pass. A closing barrier keeps any
-    replica from overwriting its stripe while a peer may still be reading it. Returns the verify result."""
+    replica from overwriting its stripe while a peer may still be reading it. With `arena` (the replicas'
+    regions live in VMM arenas, possibly released before the swap-in: the stripe restore re-acquires every
+    slab) the peers' arenas are mapped after the stripe restores (map_replicas_arena) and unmapped at the end;
+    otherwise `peer_delta` comes from map_replicas. Returns the verify result."""
+    from .swap import arena_unimport
+
     k, r = dist.get_world_size(group), dist.get_rank(group)
     s = stream if stream is not None else torch.cuda.current_stream(sw.device)
     sw.restore_stripe(r, k, s)
     s.synchronize()
     dist.barrier(group=group)
+    views = []
+    if arena is not None:
+        peer_delta, views = map_replicas_arena(arena, group)
     sw.pull_stripes(r, k, peer_delta, s)
     res = sw.verify(s, hbm_pass=True, raise_on_corrupt=False)
     dist.barrier(group=group)
+    for v in views:
+        arena_unimport(v)
     return res
 
 

@@ -35,7 +35,7 @@ EXPORTS = [
     "swap_get_launch_count", "swap_status_str", "swap_last_error", "swap_destroy",
     "swap_arena_create", "swap_arena_info", "swap_arena_release", "swap_arena_reacquire", "swap_arena_last_error",
     "swap_arena_reacquire_range", "swap_bind_arena", "swap_exchange", "swap_set_helpers",
-    "swap_arena_destroy", "swap_sched_create", "swap_sched_add_backend", "swap_sched_touch", "swap_sched_lock",
+    "swap_arena_destroy", "swap_arena_export", "swap_arena_import", "swap_arena_unimport", "swap_sched_create", "swap_sched_add_backend", "swap_sched_touch", "swap_sched_lock",
     "swap_sched_plan", "swap_sched_reserve", "swap_sched_cancel", "swap_sched_grant", "swap_sched_release",
     "swap_sched_query", "swap_sched_free", "swap_sched_destroy",
 ]
@@ -146,6 +146,10 @@ def load(build_if_missing: bool = True) -> ctypes.CDLL:
         "swap_exchange": (st, [P(vp), sz, vp, vp, vp, ctypes.c_uint64, P(ctypes.c_uint64)]),
         "swap_arena_last_error": (ctypes.c_char_p, [vp]),
         "swap_arena_destroy": (None, [vp]),
+        "swap_arena_export": (st, [vp, P(ctypes.c_int), ctypes.c_size_t, P(ctypes.c_size_t), P(ctypes.c_uint64)]),
+        "swap_arena_import": (st, [ctypes.c_int, P(ctypes.c_int), ctypes.c_size_t, ctypes.c_uint64, ctypes.c_uint64,
+                                   P(vp), P(ctypes.c_uint64)]),
+        "swap_arena_unimport": (None, [vp]),
         "swap_sched_create": (st, [u32, P(ctypes.c_uint64), P(vp)]),
         "swap_sched_add_backend": (st, [vp, u32, P(ctypes.c_uint64), ctypes.c_int]),
         "swap_sched_touch": (st, [vp, u32, u32, ctypes.c_double]),
@@ -209,6 +213,20 @@ def swap_verify(ctx, stream: int = 0, hbm_pass: bool = True):
     res = swap_verify_result_t()
     st = load().swap_verify(ctx, ctypes.c_void_p(stream), 1 if hbm_pass else 0, ctypes.byref(res))
     return st, res
+
+
+def arena_import(device: int, fds: list[int], slab_bytes: int, total_bytes: int) -> tuple[int, int]:
+    """Maps a peer's exported arena slabs on `device` (swap_arena_import): (view handle, device address)."""
+    arr = (ctypes.c_int * max(1, len(fds)))(*fds)
+    view, addr = ctypes.c_void_p(), ctypes.c_uint64()
+    st = load().swap_arena_import(device, arr, len(fds), slab_bytes, total_bytes, ctypes.byref(view), ctypes.byref(addr))
+    if st:
+        raise SwapError(st, "swap_arena_import failed")
+    return view.value, addr.value
+
+
+def arena_unimport(view: int):
+    load().swap_arena_unimport(ctypes.c_void_p(view))
 
 
 def ipc_export(device: int, ptr: int) -> tuple[bytes, int]:
@@ -557,6 +575,16 @@ class Arena:
 
         assert 0 <= offset and offset + nbytes <= self.nbytes
         return torch.as_tensor(_CudaArray(self.base + offset, nbytes), device=f"cuda:{self.device}")
+
+    def export(self) -> tuple[list[int], int]:
+        """POSIX file descriptors of the arena's slabs (the caller owns and must close them) and the slab
+        size -- swap_arena_export; pass them to a peer process (dist.map_replicas_arena does, over a Unix
+        socket) for arena_import."""
+        n, slab = ctypes.c_size_t(), ctypes.c_uint64()
+        self._check(load().swap_arena_export(self._h, None, 0, ctypes.byref(n), ctypes.byref(slab)))
+        fds = (ctypes.c_int * max(1, n.value))()
+        self._check(load().swap_arena_export(self._h, fds, n.value, ctypes.byref(n), ctypes.byref(slab)))
+        return list(fds[:n.value]), slab.value
 
     def alloc(self, nbytes: int, align: int = 256):
         """Bump-allocates `nbytes` (aligned) and returns (dev_addr, torch view)."""

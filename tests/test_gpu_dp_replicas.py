@@ -225,3 +225,72 @@ def test_stripe_pull_with_policies_masks_and_released_arena():
             assert np.array_equal(back[o:o + r.nbytes], want[o:o + r.nbytes]), r.name
         sw.bind_arena(None)
     arena.close()
+
+
+def _arena_worker(rank, world, init_file, q):
+    import sys
+
+    sys.path.insert(0, ROOT)
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import workloads as W
+    from paper_conf_sc_stoyanovsracb25_b200 import dist as sdist
+    from paper_conf_sc_stoyanovsracb25_b200 import swap
+
+    dist.init_process_group("gloo", init_method=f"file://{init_file}", rank=rank, world_size=world)
+    try:
+        torch.cuda.set_device(0)
+        specs = W.scaled(W.config_b(), 2300 << 20)  # > 2 slabs
+        offs, total = W.place(specs)
+        arena = swap.Arena(total)
+        base, view = arena.alloc(total)
+        W.fill_device_arena(view, specs, offs, seed=4)  # the same engine on every replica
+        host = view.cpu().numpy()
+        regions = [(base + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs, offs))]
+        s = torch.cuda.Stream()
+        out = {}
+        with swap.Swapper(regions, pipe_mib=64) as sw, torch.cuda.stream(s):
+            sw.bind_arena(arena)
+            for it in range(2):  # swap out (HBM released), then the cooperative swap-in; twice
+                sw.swap_out(arena, s)
+                assert not arena.resident
+                res = sdist.pull_replicas(sw, None, None, s, arena=arena)
+                out[f"res{it}"] = (res["status"], res["n_bad"], res["hbm_n_bad"])
+                back = arena.tensor(0, total).cpu().numpy()  # guards are fresh HBM after the release: regions only
+                out[f"eq{it}"] = all(np.array_equal(back[o:o + r.nbytes], host[o:o + r.nbytes]) for r, o in zip(specs, offs))
+            sw.bind_arena(None)
+        arena.close()
+        q.put((rank, out))
+    except Exception:
+        import traceback
+
+        q.put((rank, {"error": traceback.format_exc()}))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.timeout(400)
+def test_replicas_fused_pull_released_vmm_arenas():
+    """DP replicas whose regions live in released VMM arenas (NEXT-1 + NEXT-2): the stripe restore
+    re-acquires every slab, the replicas exchange their arenas' slab file descriptors over Unix sockets and
+    map each other (swap_arena_export / swap_arena_import), the fused pull fills the other stripes, and the
+    regions equal the original bytes on every replica, twice."""
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    with tempfile.TemporaryDirectory() as d:
+        init_file = os.path.join(d, "pg")
+        procs = [ctx.Process(target=_arena_worker, args=(r, world, init_file, q)) for r in range(world)]
+        for p in procs:
+            p.start()
+        res = dict(q.get(timeout=360) for _ in range(world))
+        for p in procs:
+            p.join(60)
+            assert p.exitcode == 0
+    for r in range(world):
+        assert "error" not in res[r], res[r].get("error")
+        for it in range(2):
+            assert res[r][f"res{it}"] == (0, 0, 0) and res[r][f"eq{it}"], (r, it, res[r])
