@@ -143,6 +143,15 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       : "memory");
 }
 
+// shared -> global bulk copy (TMA store, bulk-group completion; the global side may be host-mapped memory)
+__device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(smem_u32(src)), "r"(bytes)
+               : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read_all() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
 // a * b mod P (reflected), branch-free.
 __device__ __forceinline__ uint32_t multmodp(uint32_t a, uint32_t b) {
   uint32_t p = 0;
@@ -218,13 +227,25 @@ __device__ __forceinline__ uint64_t ld_u64_smem(const uint8_t* p) {  // 8-aligne
   return v;
 }
 
-// The result of chunk g: store (checkpoint / hash pass) or compare (restore / verify).
+// The expected checksum of chunk g for the compare modes, loaded when the chunk's work starts: the manifest
+// lives in mapped host memory, so the load is a PCIe round trip that must overlap the hashing, not follow it
+// (CRC-32C verify with 4-KiB chunks: one such stall per chunk). A volatile load is issued where it is
+// written (the kernels' main loops are volatile asm too). 0 for the store modes.
 template <int MODE>
-__device__ __forceinline__ void chunk_result(const Params& p, uint32_t g, uint64_t c) {
+__device__ __forceinline__ uint64_t expect_early(const Params& p, uint32_t g) {
+  if (MODE == GATHER || MODE == HASH_STORE) return 0;
+  uint64_t v;
+  asm volatile("ld.global.u64 %0, [%1];" : "=l"(v) : "l"(p.cs_exp + 4ull * g));
+  return v;
+}
+
+// The result of chunk g: store (checkpoint / hash pass) or compare (restore / verify) with the expected
+// value e (expect_early).
+template <int MODE>
+__device__ __forceinline__ void chunk_result(const Params& p, uint32_t g, uint64_t c, uint64_t e) {
   if (MODE == GATHER || MODE == HASH_STORE) {
     p.cs_out[4ull * g] = c;
   } else {
-    uint64_t e = p.cs_exp[4ull * g];
     if (e != c) {
       atomicAdd(p.n_bad, 1ull);
       atomicMin(p.first_bad, static_cast<unsigned long long>(g));
@@ -238,13 +259,14 @@ __device__ __forceinline__ void chunk_result(const Params& p, uint32_t g, uint64
 // Horner steps (crc(A||B) = Z^|B|(crc A) ^ crc B), shifts it past the segments that follow (a table of
 // x^(8*m*seg) for m whole segments, then the last one), and an XOR shuffle tree sums the lanes.
 template <int MODE>
-__device__ __forceinline__ void crc_segment_done(const Params& p, const SegDesc& d, uint32_t idx, uint32_t S, int lane) {
+__device__ __forceinline__ void crc_segment_done(const Params& p, const SegDesc& d, uint32_t idx, uint32_t S, int lane,
+                                                 uint64_t e) {
   const uint32_t* x2n = p.tables + TAB_X2N;
   if (d.nseg == 1) {
     if (lane == 0) {
       const uint64_t len = d.bytes;
       const uint32_t zi = (len == p.chunk_bytes) ? p.zinit_c : crc_shift(0xFFFFFFFFu, len, x2n);
-      chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ S)));
+      chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ S)), e);
     }
     return;
   }
@@ -283,7 +305,7 @@ __device__ __forceinline__ void crc_segment_done(const Params& p, const SegDesc&
     p.arrive[d.chunk] = 0;
     const uint64_t L = (uint64_t)(nseg - 1) * p.seg_bytes + last_len;
     const uint32_t zi = (L == p.chunk_bytes) ? p.zinit_c : crc_shift(0xFFFFFFFFu, L, x2n);
-    chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ X)));
+    chunk_result<MODE>(p, d.chunk, (uint64_t)(~(zi ^ X)), e);
   }
 }
 
@@ -314,6 +336,7 @@ __device__ __forceinline__ void move_segment(const Params& p, const SegDesc& d, 
   const uint32_t len = d.bytes;
   const uint32_t nblk = len / 512u;
   constexpr bool COPY = (MODE == GATHER || MODE == SCATTER);
+  const uint64_t e = lane == 0 ? expect_early<MODE>(p, d.chunk) : 0;  // used by lane 0 only
 
   if (KIND == KIND_XXH64) {
     // acc lanes 0..3 carry the chains v1..v4 in t-form (xt_step). Software pipeline: the loads of the next
@@ -410,7 +433,7 @@ __device__ __forceinline__ void move_segment(const Params& p, const SegDesc& d, 
       h ^= h >> 29;
       h *= P3;
       h ^= h >> 32;
-      chunk_result<MODE>(p, d.chunk, h);
+      chunk_result<MODE>(p, d.chunk, h, e);
     }
     return;
   }
@@ -450,7 +473,7 @@ __device__ __forceinline__ void move_segment(const Params& p, const SegDesc& d, 
   uint32_t S = X;  // lane 0 continues the register through the tail: F(X, tail) = F(0, full || tail)
   if (lane == 0)
     for (uint32_t i = 0; i < r; ++i) S = sT[(S ^ tail[i]) & 0xFFu] ^ (S >> 8);
-  crc_segment_done<MODE>(p, d, idx, S, lane);
+  crc_segment_done<MODE>(p, d, idx, S, lane, e);
 }
 
 // ------------------------------------------------------------------ the persistent kernel
@@ -778,6 +801,7 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
     const uint32_t idx = r * per_round + first0 + warp;
     if (idx < p.n_desc) {
       const SegDesc d = sDesc[(r & 1) * HT_WARPS + warp];
+      const uint64_t e = lane == 0 ? expect_early<MODE>(p, d.chunk) : 0;
       const uint64_t len = d.bytes;
       const uint64_t Ls = hash_strand(len);
       const uint64_t q = (uint64_t)(lane >> 2), jj = (uint64_t)(lane & 3);
@@ -795,7 +819,7 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
       }
 #pragma unroll
       for (int s = 16; s > 0; s >>= 1) X ^= __shfl_xor_sync(0xffffffffu, X, s);
-      crc_segment_done<MODE>(p, d, idx, X, lane);
+      crc_segment_done<MODE>(p, d, idx, X, lane, e);
     }
     __syncthreads();
     if (tid == 0 && r + 2 < rounds) {
@@ -881,6 +905,7 @@ __global__ void __launch_bounds__(XR_WARPS * 32) xxh_ring_kernel(const Params p)
   uint32_t seq = 0;  // stages issued by this warp so far (buffer = seq % STAGES, parity = seq / STAGES & 1)
   for (uint32_t idx = blockIdx.x * XR_WARPS + warp; idx < p.n_desc; idx += gridDim.x * XR_WARPS) {
     const SegDesc d = p.desc[idx];
+    const uint64_t e = lane == 0 ? expect_early<MODE>(p, d.chunk) : 0;
     const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
     const uint64_t len = d.bytes, len16 = len & ~15ull;
     const uint32_t nst = (uint32_t)((len16 + XR_STAGE - 1) / XR_STAGE);
@@ -953,7 +978,7 @@ __global__ void __launch_bounds__(XR_WARPS * 32) xxh_ring_kernel(const Params p)
       h ^= h >> 29;
       h *= P3;
       h ^= h >> 32;
-      chunk_result<MODE>(p, d.chunk, h);
+      chunk_result<MODE>(p, d.chunk, h, e);
     }
     seq += nst;
     __syncwarp();
@@ -1030,8 +1055,9 @@ __device__ __forceinline__ void xxh_stripes(const uint8_t* src, uint64_t end, ui
 // The end of one chunk's XXH64 once its whole 32-B stripes are in v (xxHash spec): merge, the tail
 // [stripes_end, len) read from device memory at src, avalanche; then store / compare its c_g.
 template <int MODE>
-__device__ __forceinline__ void xxh_finish(const Params& p, const SegDesc& d, const uint64_t (&v)[4]) {
-  const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
+__device__ __forceinline__ void xxh_finish(const Params& p, const SegDesc& d, const uint64_t (&v)[4], uint64_t e,
+                                           const uint8_t* src_override = nullptr) {
+  const uint8_t* src = src_override ? src_override : reinterpret_cast<const uint8_t*>(d.dev);
   const uint64_t len = d.bytes;
   uint64_t o = len / 32 * 32;
   uint64_t h;
@@ -1065,12 +1091,13 @@ __device__ __forceinline__ void xxh_finish(const Params& p, const SegDesc& d, co
   h ^= h >> 29;
   h *= P3;
   h ^= h >> 32;
-  chunk_result<MODE>(p, d.chunk, h);
+  chunk_result<MODE>(p, d.chunk, h, e);
 }
 
 // One whole chunk (descriptor d) by one lane.
 template <int MODE, int U, bool TF = true>
 __device__ __forceinline__ void xxh_chunk(const Params& p, const SegDesc& d) {
+  const uint64_t e = expect_early<MODE>(p, d.chunk);
   const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
   uint64_t v[4] = {P1 + P2, P2, 0, 0ull - P1};
   if (TF) {
@@ -1083,7 +1110,7 @@ __device__ __forceinline__ void xxh_chunk(const Params& p, const SegDesc& d) {
 #pragma unroll
     for (int i = 0; i < 4; ++i) v[i] = xt_final(v[i]);
   }
-  xxh_finish<MODE>(p, d, v);
+  xxh_finish<MODE>(p, d, v, e);
 }
 
 template <int MODE, int U, int MAXT>
@@ -1172,6 +1199,7 @@ __global__ void __launch_bounds__(W * 32) xxh_coop_kernel(const Params p) {
     const bool mine = lane < K && idx < p.n_desc;
     SegDesc d{};
     if (mine) d = p.desc[idx];
+    const uint64_t e = mine ? expect_early<MODE>(p, d.chunk) : 0;
     const uint64_t len = mine ? d.bytes : 0;
     uint64_t maxlen = len;
 #pragma unroll
@@ -1241,7 +1269,7 @@ __global__ void __launch_bounds__(W * 32) xxh_coop_kernel(const Params p) {
     }
     asm volatile("cp.async.wait_group 0;" ::: "memory");
     __syncwarp();
-    if (mine) xxh_finish<MODE>(p, d, v);
+    if (mine) xxh_finish<MODE>(p, d, v, e);
     batch = next;
   }
 }
@@ -1295,8 +1323,15 @@ __global__ void __launch_bounds__(W * 32) xxh_quad_kernel(const Params p) {
     const bool mine = idx < p.n_desc;
     SegDesc d{};
     if (mine) d = p.desc[idx];
+    const uint64_t e = (mine && j == 0) ? expect_early<MODE>(p, d.chunk) : 0;
     const uint64_t len = mine ? d.bytes : 0, len16 = len & ~15ull;
     const uint32_t nst_max = __reduce_max_sync(0xffffffffu, (uint32_t)((len16 + STG - 1) / STG));
+    // the mover modes copy as they hash: SCATTER reads the image (host-mapped, or a peer replica's HBM for
+    // swap_pull_stripes) and writes the regions, GATHER the reverse; each stage is stored from the ring by
+    // the quad leader with a TMA bulk store once the quad has hashed it
+    constexpr bool COPY = (MODE == GATHER || MODE == SCATTER);
+    const uint8_t* src = reinterpret_cast<const uint8_t*>(MODE == SCATTER ? d.host : d.dev);
+    uint8_t* dst = reinterpret_cast<uint8_t*>(MODE == SCATTER ? d.dev : d.host);
     // stage k of all the warp's chunks: lane 0 arms the barrier with their byte total, group leaders copy
     auto issue = [&](uint32_t k) {
       const uint32_t b = (seq + k) % S;
@@ -1308,7 +1343,7 @@ __global__ void __launch_bounds__(W * 32) xxh_quad_kernel(const Params p) {
         mbar_expect_tx(bars + b, tot);
       }
       __syncwarp();
-      if (j == 0 && sz) bulk_g2s(ring + (size_t)b * STG, reinterpret_cast<const uint8_t*>(d.dev) + o, sz, bars + b);
+      if (j == 0 && sz) bulk_g2s(ring + (size_t)b * STG, src + o, sz, bars + b);
     };
     for (uint32_t k = 0; k < nst_max && k < (uint32_t)S; ++k) issue(k);
     uint64_t v[NC];
@@ -1340,7 +1375,18 @@ __global__ void __launch_bounds__(W * 32) xxh_quad_kernel(const Params p) {
         }
       }
       __syncwarp();  // every lane is done with buffer b before it is refilled
+      if (COPY && j == 0) {  // store the stage, and let the TMA finish reading it before the refill
+        const uint64_t o = (uint64_t)k * STG;
+        if (o < len16) {
+          bulk_s2g(dst + o, ring + (size_t)b * STG, (uint32_t)(len16 - o < STG ? len16 - o : STG));
+          bulk_wait_read_all();
+        }
+      }
       if (k + S < nst_max) issue(k + S);
+    }
+    if (COPY && mine && j == 0) {
+      for (uint64_t o = len16; o < len; ++o) dst[o] = src[o];  // the < 16-B tail the bulk copies cannot carry
+      bulk_wait_all();  // the stores are complete before the chunk's result is published
     }
     uint64_t vv[4];
 #pragma unroll
@@ -1349,7 +1395,7 @@ __global__ void __launch_bounds__(W * 32) xxh_quad_kernel(const Params p) {
 #pragma unroll
       for (int x = 0; x < LPC; ++x) vv[x + c * LPC] = __shfl_sync(0xffffffffu, v[c], (lane & ~(LPC - 1)) + x);
     }
-    if (mine && j == 0) xxh_finish<MODE>(p, d, vv);
+    if (mine && j == 0) xxh_finish<MODE>(p, d, vv, e, src);
     seq += nst_max;
     batch = next;
     __syncwarp();
@@ -1527,6 +1573,22 @@ cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_
   if (p.chunk_bytes >= (8u << 20))
     return st ? launch_xxh_quad<HASH_STORE, 3, 2, 4096>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 3, 2, 4096>(p, sm_count, s);
   return st ? launch_xxh_quad<HASH_STORE, 4, 2, 3072>(p, sm_count, s) : launch_xxh_quad<HASH_CHECK, 4, 2, 3072>(p, sm_count, s);
+}
+
+// XXH64 GATHER / SCATTER through the quad-per-chunk kernel (copy + hash from the TMA ring), sized like the
+// verify kernels; SWAP_XXH_MOVER=warp keeps the warp-per-chunk mover (measurements).
+bool xxh_quad_mover_enabled() {
+  const char* e = getenv("SWAP_XXH_MOVER");
+  return !(e && !strcmp(e, "warp"));
+}
+cudaError_t launch_xxh_move(int mode, const Params& p, int sm_count, cudaStream_t s) {
+  if (p.n_desc == 0) return cudaSuccess;
+  const bool big = p.chunk_bytes >= (8u << 20);
+  if (mode == GATHER)
+    return big ? launch_xxh_quad<GATHER, 3, 2, 4096>(p, sm_count, s) : launch_xxh_quad<GATHER, 4, 2, 3072>(p, sm_count, s);
+  if (mode == SCATTER)
+    return big ? launch_xxh_quad<SCATTER, 3, 2, 4096>(p, sm_count, s) : launch_xxh_quad<SCATTER, 4, 2, 3072>(p, sm_count, s);
+  return cudaErrorInvalidValue;
 }
 
 cudaError_t launch_mover(int mode, int kind, const Params& p, int grid, cudaStream_t s) {

@@ -95,6 +95,9 @@ size_t mover_smem_bytes(int kind);
 // XXH64 HBM hash: one warp per chunk, chunk bytes TMA-streamed through a shared-memory ring.
 bool hash_xxh_lane_ok(int sm_count, uint32_t n_desc);
 cudaError_t launch_xxh_hash(int mode, const Params& p, int sm_count, cudaStream_t stream);
+// XXH64 GATHER / SCATTER with the quad-per-chunk kernel (needs p.ticket); enabled unless SWAP_XXH_MOVER=warp.
+bool xxh_quad_mover_enabled();
+cudaError_t launch_xxh_move(int mode, const Params& p, int sm_count, cudaStream_t stream);
 
 // Zero-fill of a span list (DISCARD regions and masked chunks on the device at restore; stale masked
 // chunks of the mapped host image at checkpoint): one launch instead of one cudaMemsetAsync per span.

@@ -53,18 +53,17 @@ int grid_of(swap_ctx* c) { return c->cfg.grid_ctas ? (int)c->cfg.grid_ctas : 2 *
 // one whole-image hash pass overlaps every D2H copy (config B, 16 MiB: CE_PIPE 57.2 vs SM 51.5 GB/s,
 // `profiles/r01_bench_B_xxh64_16MiB_v2.json`). Up to 4 MiB the restore rule is the CRC one too (config B,
 // 2 / 4 MiB: CE_PIPE 54.6 / 54.2 vs SM 50.8 / 50.6).
-// XXH64 with chunks of 1 MiB and more on images below the CRC crossover (round 2, config A 64 MiB, GB/s,
-// SM / CE_BATCH / CE_PIPE): a chunk is one serial hash job, so with few chunks the SM fused mover is bound
-// by the per-chunk round chain -- restore 27.9 / 33.9 / 21.3 at 1 MiB, 7.1 / 16.9 / 6.2 at 4 MiB, 2.3 / 7.5
-// / 3.3 at 16 MiB; checkpoint 30.1 / 34.8 / 53.8, 7.6 / 17.1 / 24.9, 2.4 / 7.9 / 9.2 -- so such restores take
-// the coalesced copies + one quad-kernel hash pass and such checkpoints CE_PIPE (the hash pass runs beside
-// the D2H copies).
+// XXH64 with chunks of 1 MiB and more on images below the CRC crossover (round 2, config A 64 MiB): a chunk
+// is one serial hash job, so with few chunks every path is bound by per-chunk round chains. Restores keep
+// the SM mover -- the quad-per-chunk kernel copies and hashes from its TMA ring: 1 MiB restore 50.7 GB/s,
+// swap-in 31.0 (CE_BATCH 23.1); 4 MiB 21.1 / 10.7 (9.0) -- checkpoints take CE_PIPE, whose hash pass runs
+// beside the D2H copies (1 MiB 53.5 vs SM 45.7 GB/s).
 uint32_t resolve_mech(const swap_ctx* c, int dir) {
   if (c->cfg.mechanism != SWAP_MECH_AUTO) return c->cfg.mechanism;
   const uint64_t S = c->plan.payload_bytes;
-  const bool xxh_big = c->plan.kind == SWAP_CHECKSUM_XXH64 && c->plan.C >= (1ull << 20);
-  if (dir == 1 && c->plan.kind == SWAP_CHECKSUM_XXH64 && c->plan.C > (4ull << 20)) return SWAP_MECH_CE_BATCH;
-  if (xxh_big && S < (2ull << 30)) return dir == 0 ? SWAP_MECH_CE_PIPE : SWAP_MECH_CE_BATCH;
+  const bool xxh = c->plan.kind == SWAP_CHECKSUM_XXH64;
+  if (dir == 1 && xxh && c->plan.C > (4ull << 20) && S >= (2ull << 30)) return SWAP_MECH_CE_BATCH;
+  if (dir == 0 && xxh && c->plan.C >= (1ull << 20)) return SWAP_MECH_CE_PIPE;
   if (dir == 0) return S < (1ull << 30) ? SWAP_MECH_SM : SWAP_MECH_CE_PIPE;
   return S < (2ull << 30) ? SWAP_MECH_SM : SWAP_MECH_CE_PIPE;
 }
@@ -88,6 +87,9 @@ swap_status launch(swap_ctx* c, int mode, int kind, const swk::Params& p, cudaSt
   cudaError_t e;
   if ((mode == swk::HASH_STORE || mode == swk::HASH_CHECK) && kind == swk::KIND_XXH64 && !c->cfg.grid_ctas)
     e = swk::launch_xxh_hash(mode, p, c->sm_count, s);
+  else if ((mode == swk::GATHER || mode == swk::SCATTER) && kind == swk::KIND_XXH64 && !c->cfg.grid_ctas &&
+           p.ticket && swk::xxh_quad_mover_enabled())
+    e = swk::launch_xxh_move(mode, p, c->sm_count, s);
   else
     e = swk::launch_mover(mode, kind, p, std::max(1, want), s);
   if (e != cudaSuccess) return cuda_fail(c, e, "mover kernel launch");
