@@ -40,12 +40,14 @@ METRIC = "swap-in (restore + HBM verify) throughput, whole job"
 RESTORE_KERNEL = {
     "sm": "mover_kernel<SCATTER,CRC|XXH> (SM loads from mapped pinned image + fused checksum)",
     "sm_nocheck": "mover_kernel<SCATTER,NONE>",
-    "ce_pipe": "restore phase: cudaMemcpyAsync H2D groups (copy engine) + hash_kernel<HASH_CHECK> per group on a side stream",
+    "ce_pipe": "restore phase: cudaMemcpyAsync H2D groups (copy engine) + the HBM hash kernel <HASH_CHECK> per group on a side stream",
     "ce_region": "restore phase: cudaMemcpyAsync per region + HBM hash pass",
     "ce_chunk": "restore phase: cudaMemcpyAsync per chunk + HBM hash pass",
     "ce_batch": "restore phase: coalesced cudaMemcpyAsync runs + HBM hash pass",
 }
-VERIFY_KERNEL = {"crc32c": "hash_kernel<HASH_CHECK> (CRC-32C: quad-line 256-bit loads, per-lane replicated slice-by-4 + Z^96 tables)",
+VERIFY_KERNEL = {"crc32c": "crc_ts_kernel<HASH_CHECK> (CRC-32C strand-staged: one TMA tensor box of 32 lane strands x 80 B per "
+                           "stage, per-lane replicated slice-by-4 tables; the quad-line hash_kernel below 128 KiB "
+                           "segments or 16 segments per warp)",
                  "xxh64": "xxh_quad_kernel<HASH_CHECK> (XXH64: a lane quad per chunk, per-chunk TMA rings in shared memory; "
                           "lane kernels below 256 KiB chunks)"}
 PCIE_GEN5_X16_GBPS = 63.015  # 64 GB/s x 128/130 (nominal, per direction)

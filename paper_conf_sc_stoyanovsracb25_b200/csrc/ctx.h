@@ -80,6 +80,9 @@ struct swap_ctx {
   swk::DevStatus* d_status = nullptr;
   swk::DevStatus* h_status = nullptr;  // pinned
   uint32_t* d_tables = nullptr;
+  void* d_tmaps = nullptr;             // strand-staged CRC kernel: per-region tensor maps (null: none)
+  uint32_t* d_chunk_region = nullptr;  // [n_chunks] region index
+  ulonglong2* d_reg_span = nullptr;    // [n_regions] {device base, bytes}
   uint32_t zinit_c = 0, xseg = 0;
   uint32_t seg = 0;  // CRC-32C segment size in use (cfg.seg_bytes, or chosen at registration when 0)
   uint32_t cur_mech = SWAP_MECH_SM;  // mechanism of the call in progress (resolve_mech)

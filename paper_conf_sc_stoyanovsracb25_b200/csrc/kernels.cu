@@ -21,6 +21,9 @@
 #include <cstdlib>
 #include <cstring>
 
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
 #include "kernels.cuh"
 
 namespace swk {
@@ -86,6 +89,10 @@ void build_tables(uint32_t* tab, uint64_t L1, uint64_t seg) {
     const uint64_t end = hash_lane_end(L1, l);
     tab[TAB_HLANE + l] = end ? host_x2nmodp(L1 - end, 3, x2n) : 0u;
   }
+  for (int l = 0; l < 32; ++l) {  // strand-staged kernel: lane l's register after its strand
+    const uint64_t tend = ts_lane_end(L1, l);
+    tab[TAB_SLANE + l] = tend ? host_x2nmodp(L1 - tend, 3, x2n) : 0u;
+  }
   for (int m = 0; m < ZS_N; ++m) tab[TAB_ZS + m] = host_x2nmodp((uint64_t)m * seg, 3, x2n);
   // Z^96 (the gap between a lane's consecutive 32-B pieces) of nibble v at nibble position k
   for (int kk = 0; kk < 8; ++kk)
@@ -100,6 +107,38 @@ void build_tables(uint32_t* tab, uint64_t L1, uint64_t seg) {
       for (int z = 0; z < 96; ++z) r = t[r & 0xFFu] ^ (r >> 8);
       tab[TAB_Z96B + kk * 256 + e] = r;
     }
+}
+
+bool encode_tmaps(void* out, const uint64_t* base, const uint64_t* bytes, int n, uint64_t L1) {
+  constexpr int S = TS_S, strands = 32;
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    cudaDriverEntryPointQueryResult q{};
+    void* f = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess || !f)
+      return false;
+    fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
+  }
+  const uint64_t P = L1 / strands;
+  if (L1 % strands || P % 16) return false;
+  memset(out, 0, (size_t)n * 128);
+  for (int r = 0; r < n; ++r) {
+    const uint64_t rows = bytes[r] / P;
+    if (rows == 0 || rows > (1ull << 31) || base[r] % 16) continue;
+    const cuuint64_t dims[2] = {P, rows}, strides[1] = {P};
+    const cuuint32_t box[2] = {(cuuint32_t)S, (cuuint32_t)strands}, es[2] = {1, 1};
+    CUtensorMap* m = reinterpret_cast<CUtensorMap*>(static_cast<uint8_t*>(out) + 128ull * r);
+    if (fn(m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, reinterpret_cast<void*>(base[r]), dims, strides, box, es,
+           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS) {
+      if (getenv("SWAP_DEBUG_TMAP"))
+        fprintf(stderr, "encode_tmaps: region %d base %llx bytes %llu L1 %llu S %d strands %d failed\n", r,
+                (unsigned long long)base[r], (unsigned long long)bytes[r], (unsigned long long)L1, S, strands);
+      return false;
+    }
+  }
+  return true;
 }
 
 // ------------------------------------------------------------------ device helpers
@@ -852,18 +891,262 @@ static cudaError_t launch_hash_t(const Params& p, int grid, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-// CRC-32C hash-pass variant: b0f (default), or forced with SWAP_CRC_KERNEL (base | b0f | zb | zbb0f) for
-// A/B measurements (read at every launch). In-process on config B (profiles/r02_crc_variants.md): b0f
-// +0.9..1.7 % over base at 4 KiB / 1 MiB / 16 MiB chunks; the Z^96 byte tables (zb) -10 % -- their 2-way
-// conflicts cost more than the 4 lookups they save.
+// ------------------------------------------------------------------ HBM hash kernel (CRC-32C), strand-staged
+// The quad-line kernel above pays 8 nibble lookups (Z^96) per 32-B piece because a lane's bytes are 32-B
+// pieces 128 B apart: 40 lookup + 8 load L1 wavefronts per KiB per warp. Here a segment is cut into 32
+// contiguous strands (ts_strand), one per lane, streamed through a per-warp ring of NB stages in shared
+// memory: stage k holds bytes [k*S, (k+1)*S) of every strand, row = lane. A lane's bytes are then contiguous
+// across stages, so its register only takes slicing-by-4 word steps -- no Z shift until the final fold by
+// x^(8 * bytes after the strand) (TAB_SLANE for the common length L1): 32 lookup + 8 LDS.128 wavefronts per
+// KiB per warp. S is an odd multiple of 16 B, so the 8 lanes of an LDS.128 phase hit 8 distinct 16-B bank
+// groups. Standard segments (len == L1 at a multiple of L1 inside their region: every full segment) are
+// staged with ONE 2-D tensor copy per stage -- the region viewed as rows of P = L1/32 bytes, box {S, 32} at
+// column k*S, row offset/P; columns past P (a strand's last partial stage) are out of bounds, zero-filled,
+// never read from memory. Other segments (ragged region tails, DISCARD chunks hashed from the zero buffer)
+// take per-lane 1-D bulk copies: ptxas issues those through an ELECT loop (~10 issue slots per lane and
+// stage), half the speed if every segment took them (profiles/r02_crc_strand_staged.md), fine for the few
+// ragged ones. The producer (lane 0 on the tensor path) runs NB stages ahead across segment boundaries (the
+// warp's segments form one flat stage sequence). Throughput follows the resident warp count (dependent
+// lookup chains), which shared memory caps: the tables take 128 KiB, each warp's ring NB*32*S bytes.
+// Shared layout (window addresses, base R0): W*NB mbarriers at R0, rings below the 32-KiB-aligned slicing
+// tables and after them (the tables sit at a 32-KiB boundary for crc_word4's (index << 7) | lb addresses).
+template <int W, int NB, int S>
+struct TsLayout {
+  static_assert(S % 16 == 0 && (S / 16) % 2 == 1, "stage width: odd multiple of 16 B (conflict-free LDS.128)");
+  static_assert(S == TS_S, "the tensor maps are encoded for box {TS_S, 32}");
+  static constexpr uint32_t STAGE = 32u * S;
+  static constexpr uint32_t RING = (uint32_t)NB * STAGE;
+  uint32_t bar, low, tab, high, nlow, end;
+};
+constexpr uint32_t TS_SMEM_MAX = 227u * 1024u;  // opt-in dynamic shared memory per CTA
+template <int W, int NB, int S>
+__host__ __device__ inline TsLayout<W, NB, S> ts_layout(uint32_t R0) {
+  using LT = TsLayout<W, NB, S>;
+  LT L{};
+  L.bar = R0;
+  L.low = ht_align(R0 + W * NB * 8, 128);
+  L.tab = ht_align(L.low, 32768);
+  if (L.tab < L.low + LT::RING) L.tab = ht_align(L.low + 1, 32768);
+  L.nlow = (L.tab - L.low) / LT::RING;
+  if (L.nlow > (uint32_t)W) L.nlow = W;
+  L.high = L.tab + 4 * 256 * 128;
+  L.end = L.high + (uint32_t)(W - L.nlow) * LT::RING;
+  return L;
+}
+
+__device__ __forceinline__ uint4 lds128(uint32_t addr) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr));
+  return v;
+}
+__device__ __forceinline__ void bulk_g2s_a(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(bar)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx_a(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_a(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n}" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const void* tmap, int c0, int c1, uint32_t bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::
+          "r"(dst), "l"(tmap), "r"(c0), "r"(c1), "r"(bar)
+      : "memory");
+}
+
+template <int MODE, int W, int NB, int S>
+__global__ void __launch_bounds__(W * 32, 1) crc_ts_kernel(const Params p) {
+  using LT = TsLayout<W, NB, S>;
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  const LT L = ts_layout<W, NB, S>(raw);
+  uint8_t* smem = smem_raw - raw;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+
+  for (int i = tid; i < 4 * 256; i += W * 32) {  // slicing tables T0..T3, replicated once per lane
+    const uint32_t v = __ldg(p.tables + TAB_T16 + i);
+    uint4* dst = reinterpret_cast<uint4*>(smem + L.tab + (size_t)i * 128);
+#pragma unroll
+    for (int r = 0; r < 8; ++r) dst[r] = make_uint4(v, v, v, v);
+  }
+  const uint32_t bars = L.bar + (uint32_t)warp * NB * 8;
+  if (lane == 0) {
+    for (int b = 0; b < NB; ++b)
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bars + 8 * b), "r"(1) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  const uint32_t ring = (uint32_t)warp < L.nlow ? L.low + (uint32_t)warp * LT::RING
+                                                : L.high + ((uint32_t)warp - L.nlow) * LT::RING;
+  const uint32_t myrow = ring + (uint32_t)lane * S;
+  __syncthreads();
+
+  const uint32_t stride = gridDim.x * W;
+  const uint32_t L1 = p.hlane_len;
+  // producer cursor (this warp's copies): segment pidx, its stage pk of pnst; psrc = this lane's strand,
+  // pbytes = its bytes below len & ~15 (the bulk-copied part); ptm / prow: the tensor path
+  uint32_t pidx = blockIdx.x * W + warp, pk = 0, pnst = 0, pseq = 0, pbytes = 0;
+  const uint8_t* psrc = nullptr;
+  const void* ptm = nullptr;
+  int prow = 0;
+  auto p_load = [&]() {  // geometry of producer segment pidx (skipping empty ones)
+    for (; pidx < p.n_desc; pidx += stride) {
+      const uint64_t dev = __ldg(reinterpret_cast<const unsigned long long*>(&p.desc[pidx].dev));
+      const uint32_t len = __ldg(&p.desc[pidx].bytes);
+      const uint32_t Ls = (uint32_t)ts_strand(len);
+      pnst = (Ls + S - 1) / S;
+      if (pnst == 0) continue;
+      const uint32_t a0 = (uint32_t)lane * Ls, e16 = min(a0 + Ls, len & ~15u);
+      pbytes = e16 > a0 ? e16 - a0 : 0u;
+      psrc = reinterpret_cast<const uint8_t*>(dev) + a0;
+      pk = 0;
+      ptm = nullptr;
+      if (p.tmaps && len == L1) {
+        const uint32_t r = __ldg(p.chunk_region + __ldg(&p.desc[pidx].chunk));
+        const ulonglong2 rs = __ldg(p.reg_span + r);
+        const uint64_t off = dev - rs.x;
+        if (dev >= rs.x && off + len <= rs.y && off % L1 == 0) {
+          ptm = reinterpret_cast<const uint8_t*>(p.tmaps) + 128ull * r;
+          prow = (int)(off / (L1 / 32));
+        }
+      }
+      return;
+    }
+  };
+  auto p_issue = [&]() {  // next stage of the flat sequence into buffer pseq % NB
+    if (pidx >= p.n_desc) return;
+    const uint32_t off = pk * S;
+    const uint32_t b = pseq % NB;
+    const uint32_t bar = bars + 8 * b;
+    if (ptm) {
+      if (lane == 0) {
+        mbar_arrive_tx_a(bar, LT::STAGE);
+        tma_load_2d(ring + b * LT::STAGE, ptm, (int)off, prow, bar);
+      }
+    } else {
+      const uint32_t n = pbytes > off ? min(pbytes - off, (uint32_t)S) : 0u;
+      const uint32_t tot = __reduce_add_sync(0xffffffffu, n);
+      if (lane == 0) mbar_arrive_tx_a(bar, tot);
+      if (n) bulk_g2s_a(myrow + b * LT::STAGE, psrc + off, n, bar);
+    }
+    ++pseq;
+    if (++pk == pnst) {
+      pidx += stride;
+      p_load();
+    }
+  };
+  p_load();
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+#pragma unroll 1
+  for (int k = 0; k < NB; ++k) p_issue();
+
+  const uint32_t lb = L.tab + 4u * lane;
+  const uint32_t m128 = 128u * gridDim.y;  // = 128 (gridDim.y == 1), opaque to ptxas
+  const uint32_t* x2n = p.tables + TAB_X2N;
+  uint32_t cseq = 0;
+  for (uint32_t idx = blockIdx.x * W + warp; idx < p.n_desc; idx += stride) {
+    const SegDesc d = p.desc[idx];
+    const uint64_t e = lane == 0 ? expect_early<MODE>(p, d.chunk) : 0;
+    const uint32_t len = d.bytes, Ls = (uint32_t)ts_strand(len), nst = (Ls + S - 1) / S;
+    const uint32_t a0 = (uint32_t)lane * Ls, aend = min(a0 + Ls, len), e16 = min(aend, len & ~15u);
+    const uint32_t mine = e16 > a0 ? e16 - a0 : 0u;
+    uint32_t c = 0;
+#pragma unroll 1
+    for (uint32_t k = 0; k < nst; ++k) {
+      const uint32_t b = cseq % NB;
+      mbar_wait_a(bars + 8 * b, (cseq / NB) & 1u);
+      const uint32_t row = myrow + b * LT::STAGE;
+      const uint32_t off = k * S;
+      const uint32_t n = mine > off ? min(mine - off, (uint32_t)S) : 0u;
+      if (n == (uint32_t)S) {
+        uint4 v[S / 16];
+#pragma unroll
+        for (int u = 0; u < S / 16; ++u) v[u] = lds128(row + 16 * u);
+#pragma unroll
+        for (int u = 0; u < S / 16; ++u) {
+          c = crc_word4<true>(c, v[u].x, lb, m128);
+          c = crc_word4<true>(c, v[u].y, lb, m128);
+          c = crc_word4<true>(c, v[u].z, lb, m128);
+          c = crc_word4<true>(c, v[u].w, lb, m128);
+        }
+      } else {
+#pragma unroll 1
+        for (uint32_t u = 0; u < n; u += 16) {
+          const uint4 v = lds128(row + u);
+          c = crc_word4<true>(c, v.x, lb, m128);
+          c = crc_word4<true>(c, v.y, lb, m128);
+          c = crc_word4<true>(c, v.z, lb, m128);
+          c = crc_word4<true>(c, v.w, lb, m128);
+        }
+      }
+      ++cseq;
+      __syncwarp();  // every lane's reads of this stage precede its refill (one tensor copy fills all rows)
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      p_issue();
+    }
+    uint32_t X = 0;
+    if (a0 < len) {
+      // the segment's last len & 15 bytes (the strand that ends at len), from HBM
+      const uint8_t* src = reinterpret_cast<const uint8_t*>(d.dev);
+      for (uint32_t s = max(e16, a0); s < aend; ++s) c = lds_at((((c ^ src[s]) & 0xFFu) << 7) | lb) ^ (c >> 8);
+      const uint32_t kz = (len == L1) ? __ldg(p.tables + TAB_SLANE + lane) : x2nmodp(len - aend, 3, x2n);
+      X = multmodp(kz, c);
+    }
+#pragma unroll
+    for (int s = 16; s > 0; s >>= 1) X ^= __shfl_xor_sync(0xffffffffu, X, s);
+    crc_segment_done<MODE>(p, d, idx, X, lane, e);
+  }
+}
+
+template <int MODE, int W, int NB, int S>
+static cudaError_t launch_ts_t(const Params& p, int grid_cap, cudaStream_t s) {
+  static unsigned long long attr_set = 0;
+  uint32_t R0 = 0;
+  cudaError_t e = smem_base(&R0);
+  if (e != cudaSuccess) return e;
+  const TsLayout<W, NB, S> L = ts_layout<W, NB, S>(R0);
+  const size_t bytes = L.end - R0;
+  if (bytes > TS_SMEM_MAX) return cudaErrorInvalidConfiguration;
+  int dev = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  if (!((attr_set >> (dev & 63)) & 1ull)) {
+    e = cudaFuncSetAttribute(crc_ts_kernel<MODE, W, NB, S>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+    if (e != cudaSuccess) return e;
+    attr_set |= 1ull << (dev & 63);
+  }
+  const int grid = (int)std::max<uint32_t>(1, std::min<uint32_t>((uint32_t)grid_cap, (p.n_desc + W - 1) / W));
+  crc_ts_kernel<MODE, W, NB, S><<<grid, W * 32, bytes, s>>>(p);
+  return cudaGetLastError();
+}
+
+// CRC-32C hash-pass kernel. Default: the strand-staged kernel (19 warps, 2 x 80-B stages) when the tensor
+// maps exist, the common segment length L1 is at least 128 KiB and there are at least 16 segments per warp
+// of the grid -- +2.4..7.1 % (mean +4.7 %) over the quad-line b0f kernel on config B (1 MiB chunks) in six
+// in-process A/B blocks, +4.7 / +5.0 % with 16 / 4 MiB chunks (profiles/r02_crc_strand_staged.md) -- else
+// the quad-line b0f kernel: with short segments (a 16-KiB-segment 64 MiB image 48 vs 66 us; 4-KiB chunks
+// 2.8 vs 1.8 TB/s) or few segments per warp (1 GiB, 4096 x 256 KiB: 0.25 vs 0.39 ms, the static segment
+// deal leaves whole segments of tail) the quad-line kernel wins. SWAP_CRC_KERNEL (base | b0f | zb | zbb0f | ts | ts16; read at every launch) forces one for
+// A/B measurements: b0f +0.9..1.7 % over base; the Z^96 byte tables (zb) -10 % (profiles/r02_crc_variants.md).
 template <int MODE>
 static cudaError_t launch_hash(const Params& p, int grid, cudaStream_t s) {
-  int v = 1;
-  if (const char* e = getenv("SWAP_CRC_KERNEL")) v = !strcmp(e, "base") ? 0 : !strcmp(e, "zb") ? 2 : !strcmp(e, "zbb0f") ? 3 : 1;
+  int v = (p.tmaps && p.hlane_len >= (128u << 10) && p.n_desc >= 16u * 19u * (uint32_t)grid) ? 10 : 1;
+  if (const char* e = getenv("SWAP_CRC_KERNEL"))
+    v = !strcmp(e, "base") ? 0 : !strcmp(e, "zb") ? 2 : !strcmp(e, "zbb0f") ? 3 : !strcmp(e, "ts") ? 10
+      : !strcmp(e, "ts16") ? 11 : 1;
   switch (v) {
     case 0: return launch_hash_t<MODE, false, false>(p, grid, s);
     case 2: return launch_hash_t<MODE, true, false>(p, grid, s);
     case 3: return launch_hash_t<MODE, true, true>(p, grid, s);
+    case 10: return launch_ts_t<MODE, 19, 2, TS_S>(p, grid, s);
+    case 11: return launch_ts_t<MODE, 16, 2, TS_S>(p, grid, s);
     default: return launch_hash_t<MODE, false, true>(p, grid, s);
   }
 }

@@ -45,7 +45,8 @@ constexpr int TAB_Z96N = TAB_HLANE + 32;       // [8][16] hash kernel: Z^96 of n
 constexpr int ZS_N = 1024;
 constexpr int TAB_ZS = TAB_Z96N + 128;         // [ZS_N] x^(8*m*seg) mod P: shift by m whole segments
 constexpr int TAB_Z96B = TAB_ZS + ZS_N;        // [4][256] hash kernel (ZB variant): Z^96 of byte e at position k
-constexpr int TAB_WORDS = TAB_Z96B + 4 * 256;
+constexpr int TAB_SLANE = TAB_Z96B + 4 * 256;  // [32] strand-staged hash kernel: Z^(L1 - ts_lane_end(L1, l))
+constexpr int TAB_WORDS = TAB_SLANE + 32;
 constexpr int TAB_SMEM_WORDS = TAB_LANE + 32;  // the part staged in shared memory
 
 struct Params {
@@ -64,6 +65,9 @@ struct Params {
   uint32_t xseg;                 // x^(8*seg_bytes) mod P
   uint32_t hlane_len;            // L1: the segment length TAB_HLANE was built for
   unsigned int* ticket;          // dynamic XXH64 lane kernel: chunk counter, zeroed before each launch
+  const void* tmaps;             // [n_regions] CUtensorMap of the strand-staged CRC kernel's tensor path, or null
+  const uint32_t* chunk_region;  // [n_chunks] region index of chunk g
+  const ulonglong2* reg_span;    // [n_regions] {device base, bytes}
 };
 
 void build_tables(uint32_t* tab /* TAB_WORDS */, uint64_t common_seg_len, uint64_t seg_bytes);
@@ -80,6 +84,21 @@ __host__ __device__ inline uint64_t hash_lane_end(uint64_t len, int lane) {
   const uint64_t last = s0 + (strand_end - 1 - s0) / 128 * 128;
   return last + 32 < strand_end ? last + 32 : strand_end;
 }
+// Strand geometry of the strand-staged CRC-32C hash kernel: a segment of `len` bytes is cut into 32
+// contiguous strands of ts_strand(len) bytes (a multiple of 16), one per lane; lane l owns
+// [l*Ls, min((l+1)*Ls, len)). ts_lane_end = one past the lane's last byte (0 if it owns none).
+__host__ __device__ inline uint64_t ts_strand(uint64_t len) { return ((len + 31) / 32 + 15) / 16 * 16; }
+__host__ __device__ inline uint64_t ts_lane_end(uint64_t len, int lane) {
+  const uint64_t Ls = ts_strand(len), a0 = (uint64_t)lane * Ls;
+  if (a0 >= len) return 0;
+  return a0 + Ls < len ? a0 + Ls : len;
+}
+// Its tensor path: region r viewed as rows of L1/32 bytes (u8, row pitch L1/32), box {TS_S, 32}; map r at
+// tmaps + 128 * r. out: n * 128 bytes (host); a region smaller than one row gets a zeroed map (never used:
+// its segments are not standard). Returns false if the driver entry point is missing or an encode fails
+// (the kernel then takes per-lane bulk copies, or launch_hash the quad-line kernel).
+constexpr int TS_S = 80;
+bool encode_tmaps(void* out, const uint64_t* base, const uint64_t* bytes, int n, uint64_t L1);
 uint32_t host_x2nmodp(uint64_t n, unsigned k, const uint32_t* x2n);
 uint32_t host_multmodp(uint32_t a, uint32_t b);
 

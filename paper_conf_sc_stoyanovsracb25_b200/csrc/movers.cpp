@@ -36,6 +36,9 @@ swk::Params base_params(swap_ctx* c, const DescSet& S) {
   p.xseg = c->xseg;
   p.hlane_len = (uint32_t)std::min<uint64_t>(c->plan.C, c->seg);
   p.ticket = &c->d_status->ticket;
+  p.tmaps = c->d_tmaps;
+  p.chunk_region = c->d_chunk_region;
+  p.reg_span = c->d_reg_span;
   return p;
 }
 
@@ -286,6 +289,31 @@ swap_status upload_tables(swap_ctx* c) {
   const uint32_t* x2n = tab.data() + swk::TAB_X2N;
   c->zinit_c = swk::host_multmodp(swk::host_x2nmodp(c->cfg.chunk_bytes, 3, x2n), 0xFFFFFFFFu);
   c->xseg = swk::host_x2nmodp(c->seg, 3, x2n);
+  // strand-staged CRC kernel's tensor path: a map per region, the region of every chunk
+  const size_t nr = c->plan.regions.size();
+  if (c->plan.kind == SWAP_CHECKSUM_CRC32C && nr && !c->d_tmaps) {
+    std::vector<uint64_t> base(nr), bytes(nr);
+    std::vector<ulonglong2> span(nr);
+    std::vector<uint32_t> creg(c->plan.n_chunks);
+    for (size_t r = 0; r < nr; ++r) {
+      const auto& R = c->plan.regions[r];
+      base[r] = R.r.dev_addr;
+      bytes[r] = R.r.bytes;
+      span[r] = make_ulonglong2(R.r.dev_addr, R.r.bytes);
+      for (uint64_t g = R.first; g < R.first + R.nchunks; ++g) creg[g] = (uint32_t)r;
+    }
+    std::vector<uint8_t> maps(nr * 128);
+    if (swk::encode_tmaps(maps.data(), base.data(), bytes.data(), (int)nr, std::min<uint64_t>(c->plan.C, c->seg))) {
+      CUDA_TRY(c, cudaMalloc(&c->d_tmaps, maps.size()));
+      CUDA_TRY(c, cudaMemcpy(c->d_tmaps, maps.data(), maps.size(), cudaMemcpyHostToDevice));
+      CUDA_TRY(c, cudaMalloc(&c->d_reg_span, nr * sizeof(ulonglong2)));
+      CUDA_TRY(c, cudaMemcpy(c->d_reg_span, span.data(), nr * sizeof(ulonglong2), cudaMemcpyHostToDevice));
+      if (!creg.empty()) {
+        CUDA_TRY(c, cudaMalloc(&c->d_chunk_region, creg.size() * 4));
+        CUDA_TRY(c, cudaMemcpy(c->d_chunk_region, creg.data(), creg.size() * 4, cudaMemcpyHostToDevice));
+      }
+    }
+  }
   return SWAP_OK;
 }
 
@@ -344,6 +372,9 @@ void release(swap_ctx* c) {
   if (c->d_status) cudaFree(c->d_status);
   if (c->h_status) cudaFreeHost(c->h_status);
   if (c->d_tables) cudaFree(c->d_tables);
+  if (c->d_tmaps) cudaFree(c->d_tmaps);
+  if (c->d_chunk_region) cudaFree(c->d_chunk_region);
+  if (c->d_reg_span) cudaFree(c->d_reg_span);
   for (auto& e : c->ev)
     if (e) cudaEventDestroy(e);
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
