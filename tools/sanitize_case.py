@@ -63,14 +63,18 @@ for v in ("quad", "quad2", "quad3k"):
         sw.restore(s)
         assert sw.verify(s)["status"] == 0, v
 os.environ.pop("SWAP_XXH_KERNEL")
-# CRC-32C hash kernel variants (fixed shared layout at the 0x400 dynamic base)
-for v in ("base", "b0f", "zb", "zbb0f"):
+# CRC-32C hash kernel variants (fixed shared layout at the 0x400 dynamic base; the strand-staged ts kernels
+# with their tensor-map path on standard segments and per-lane bulk copies on ragged ones, also with
+# 128 KiB segments of 1 MiB chunks)
+for v in ("base", "b0f", "zb", "zbb0f", "ts", "ts16"):
     os.environ["SWAP_CRC_KERNEL"] = v
-    with swap.Swapper(regions, chunk_bytes=1 << 16, checksum=1, mechanism="ce_region") as sw, torch.cuda.stream(s):
-        sw.checkpoint(s)
-        poison(arena, specs, offs)
-        sw.restore(s)
-        assert sw.verify(s)["status"] == 0, v
+    for C, seg in ((1 << 16, 0), (1 << 20, 1 << 17)):
+        with swap.Swapper(regions, chunk_bytes=C, checksum=1, mechanism="ce_region", seg_bytes=seg) as sw, \
+                torch.cuda.stream(s):
+            sw.checkpoint(s)
+            poison(arena, specs, offs)
+            sw.restore(s)
+            assert sw.verify(s)["status"] == 0, v
 os.environ.pop("SWAP_CRC_KERNEL")
 # DP replicas in one process: stripe restore of replica A, then the fused pull of the other stripe from
 # replica B (a second arena with the same bytes at a constant shift)
