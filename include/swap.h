@@ -296,7 +296,9 @@ typedef struct {
   float checkpoint_ms; /* gather kernel, or hash pass + copy-engine copies */
   float restore_ms;    /* scatter kernel, or copy-engine copies + hash pass */
   float verify_ms;     /* HBM verify pass */
-  float reserved;
+  float check_ms;      /* CE_PIPE restore: summed device time of its per-group HASH_CHECK launches on the side
+                        * stream (CUDA events around each launch; they overlap the copy engine's H2D copies,
+                        * off the critical path); 0 for other mechanisms and for helper groups */
 } swap_timings_t;
 SWAP_API swap_status swap_get_timings(const swap_ctx_t* ctx, swap_timings_t* out);
 

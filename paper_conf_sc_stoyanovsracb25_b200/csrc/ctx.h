@@ -117,6 +117,10 @@ struct swap_ctx {
   int numa_node = -1;         // NUMA node the image placement targeted (-1: none)
   double numa_local = 1.0;    // sampled share of image pages on numa_node
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  // per-group check timing of the last CE_PIPE restore (swap_timings_t.check_ms): event pairs, reused
+  std::vector<cudaEvent_t> chk_ev;
+  uint32_t n_chk = 0;
+  float chk_ms = 0.f;
 };
 
 namespace swc {

@@ -812,8 +812,13 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
     }
   }
   const uint32_t per_round = gridDim.x * HT_WARPS;
+  // fewer segments than warp slots (a CE_PIPE group's check): one round, segments dealt warp-major across the
+  // CTAs (segment w * grid + cta) so that every SM hashes, descriptors read directly; else rounds of
+  // HT_WARPS consecutive descriptors per CTA staged by TMA
+  const bool spread = p.n_desc < per_round;
   const uint32_t first0 = blockIdx.x * HT_WARPS;
-  const uint32_t rounds = p.n_desc > first0 ? (p.n_desc - first0 + per_round - 1) / per_round : 0u;
+  const uint32_t rounds = spread ? (blockIdx.x < p.n_desc ? 1u : 0u)
+                                 : p.n_desc > first0 ? (p.n_desc - first0 + per_round - 1) / per_round : 0u;
   auto issue = [&](uint32_t r) {
     const uint32_t first = r * per_round + first0;
     const uint32_t cnt = min((uint32_t)HT_WARPS, p.n_desc - first);
@@ -826,8 +831,8 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
     mbar_init(sBar + 1, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-    if (rounds > 0) issue(0);
-    if (rounds > 1) issue(1);
+    if (!spread && rounds > 0) issue(0);
+    if (!spread && rounds > 1) issue(1);
   }
   __syncthreads();
   const uint32_t lb = HL.tab + 4u * lane;
@@ -836,10 +841,10 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
   const uint32_t* x2n = p.tables + TAB_X2N;
 
   for (uint32_t r = 0; r < rounds; ++r) {
-    mbar_wait(sBar + (r & 1), (r >> 1) & 1u);
-    const uint32_t idx = r * per_round + first0 + warp;
+    if (!spread) mbar_wait(sBar + (r & 1), (r >> 1) & 1u);
+    const uint32_t idx = spread ? warp * gridDim.x + blockIdx.x : r * per_round + first0 + warp;
     if (idx < p.n_desc) {
-      const SegDesc d = sDesc[(r & 1) * HT_WARPS + warp];
+      const SegDesc d = spread ? p.desc[idx] : sDesc[(r & 1) * HT_WARPS + warp];
       const uint64_t e = lane == 0 ? expect_early<MODE>(p, d.chunk) : 0;
       const uint64_t len = d.bytes;
       const uint64_t Ls = hash_strand(len);
@@ -861,7 +866,7 @@ __global__ void __launch_bounds__(HT_THREADS, 1) hash_kernel(const Params p) {
       crc_segment_done<MODE>(p, d, idx, X, lane, e);
     }
     __syncthreads();
-    if (tid == 0 && r + 2 < rounds) {
+    if (!spread && tid == 0 && r + 2 < rounds) {
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       issue(r + 2);
     }
@@ -1151,9 +1156,10 @@ static cudaError_t launch_hash(const Params& p, int grid, cudaStream_t s) {
   }
 }
 
+// Every SM takes part even with few segments (hash_kernel deals them warp-major across CTAs then): a CE_PIPE
+// restore group's check (~1 K segments of 256 KiB) ran on 32 SMs before.
 int hash_grid(int sm_count, uint32_t n_desc) {
-  const uint32_t batches = (n_desc + HT_WARPS - 1) / HT_WARPS;
-  return (int)std::max<uint32_t>(1, std::min<uint32_t>((uint32_t)sm_count, batches));
+  return (int)std::max<uint32_t>(1, std::min<uint32_t>((uint32_t)sm_count, n_desc));
 }
 
 

@@ -108,7 +108,7 @@ int mover_threads();
 // Measures (once per device) where kernels' dynamic shared memory starts; the CRC hash kernel's table
 // layout is derived from it. Called by swap_create.
 cudaError_t probe_smem_base();
-// Grid for the CRC HBM hash kernel (1 CTA of 1024 threads per SM, 128 KB tables).
+// Grid for the CRC HBM hash kernels: one CTA per SM (never more CTAs than segments).
 int hash_grid(int sm_count, uint32_t n_desc);
 size_t mover_smem_bytes(int kind);
 // XXH64 HBM hash: one warp per chunk, chunk bytes TMA-streamed through a shared-memory ring.

@@ -193,6 +193,7 @@ swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, c
   swap_status st;
   if (dir == 0 && (st = launch(c, swk::HASH_STORE, hash_kind(c), base, c->side)) != SWAP_OK) return st;
   const size_t H = dir == 1 ? c->helpers.size() : 0;
+  if (dir == 1) c->n_chk = 0;
   for (auto& h : c->helpers)
     if (H) CUDA_TRY(c, cudaStreamWaitEvent(h.s, c->ev_fork, 0));
   for (size_t g = 0; g < S.groups.size(); ++g) {
@@ -245,7 +246,15 @@ swap_status ce_pipe(swap_ctx* c, DescSet& S, int dir, const swk::Params& base, c
       p.desc = base.desc + G.d0;
       p.partial = base.partial + G.d0;
       p.n_desc = G.d1 - G.d0;
+      while (c->chk_ev.size() < 2ull * (c->n_chk + 1)) {
+        cudaEvent_t e = nullptr;
+        CUDA_TRY(c, cudaEventCreate(&e));
+        c->chk_ev.push_back(e);
+      }
+      CUDA_TRY(c, cudaEventRecord(c->chk_ev[2 * c->n_chk], c->side));
       if ((st = launch(c, swk::HASH_CHECK, hash_kind(c), p, c->side)) != SWAP_OK) return st;
+      CUDA_TRY(c, cudaEventRecord(c->chk_ev[2 * c->n_chk + 1], c->side));
+      ++c->n_chk;
     }
   }
   for (auto& h : c->helpers) {
@@ -265,6 +274,15 @@ swap_status collect_timing(swap_ctx* c, int p) {
   if (!c->pending[p]) return SWAP_OK;
   CUDA_TRY(c, cudaEventElapsedTime(&c->ms[p], c->ev[2 * p], c->ev[2 * p + 1]));
   c->pending[p] = false;
+  if (p == 1) {  // the per-group checks of a CE_PIPE restore (n_chk = 0 for other movers)
+    c->chk_ms = 0.f;
+    for (uint32_t i = 0; i < c->n_chk; ++i) {
+      float ms = 0.f;
+      CUDA_TRY(c, cudaEventElapsedTime(&ms, c->chk_ev[2 * i], c->chk_ev[2 * i + 1]));
+      c->chk_ms += ms;
+    }
+    c->n_chk = 0;
+  }
   return SWAP_OK;
 }
 
@@ -377,6 +395,9 @@ void release(swap_ctx* c) {
   if (c->d_reg_span) cudaFree(c->d_reg_span);
   for (auto& e : c->ev)
     if (e) cudaEventDestroy(e);
+  for (auto& e : c->chk_ev)
+    if (e) cudaEventDestroy(e);
+  c->chk_ev.clear();
   if (c->ev_fork) cudaEventDestroy(c->ev_fork);
   if (c->ev_join) cudaEventDestroy(c->ev_join);
   if (c->side) cudaStreamDestroy(c->side);

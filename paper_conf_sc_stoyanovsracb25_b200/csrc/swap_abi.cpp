@@ -613,7 +613,7 @@ swap_status swap_get_timings(const swap_ctx_t* c, swap_timings_t* out) {
   out->checkpoint_ms = c->ms[0];
   out->restore_ms = c->ms[1];
   out->verify_ms = c->ms[2];
-  out->reserved = 0.f;
+  out->check_ms = c->ms[1] > 0.f ? c->chk_ms : 0.f;
   return SWAP_OK;
 }
 

@@ -76,7 +76,7 @@ class swap_shard_summary_t(ctypes.Structure):
 
 class swap_timings_t(ctypes.Structure):
     _fields_ = [("checkpoint_ms", ctypes.c_float), ("restore_ms", ctypes.c_float), ("verify_ms", ctypes.c_float),
-                ("reserved", ctypes.c_float)]
+                ("check_ms", ctypes.c_float)]
 
 
 assert ctypes.sizeof(swap_shard_summary_t) == 64 and ctypes.sizeof(swap_config_t) == 56
@@ -491,10 +491,12 @@ class Swapper:
         return d.value
 
     def timings(self) -> dict:
-        """Device ms of the last checkpoint / restore / HBM verify movers (CUDA events)."""
+        """Device ms of the last checkpoint / restore / HBM verify movers (CUDA events), and the summed
+        device ms of the last CE_PIPE restore's per-group check launches (check_ms)."""
         t = swap_timings_t()
         self._check(load().swap_get_timings(self._ctx, ctypes.byref(t)))
-        return {"checkpoint_ms": t.checkpoint_ms, "restore_ms": t.restore_ms, "verify_ms": t.verify_ms}
+        return {"checkpoint_ms": t.checkpoint_ms, "restore_ms": t.restore_ms, "verify_ms": t.verify_ms,
+                "check_ms": t.check_ms}
 
     def launch_count(self) -> int:
         n = ctypes.c_uint64()
