@@ -449,7 +449,7 @@ def run_ours(args):
     if world != args.gpus:
         print(f"warning: --gpus {args.gpus} but WORLD_SIZE={world}", file=sys.stderr)
     ndev = torch.cuda.device_count()
-    local_dev = local % ndev if args.dist_backend == "gloo" else local
+    local_dev = local % ndev if args.dist_backend == "gloo" or local >= ndev else local
     torch.cuda.set_device(local_dev)
     dev = torch.device("cuda", local_dev)
     node = gpu_numa_node(local_dev)

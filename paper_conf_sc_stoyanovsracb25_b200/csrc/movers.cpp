@@ -322,6 +322,9 @@ swap_status upload_tables(swap_ctx* c) {
     }
     std::vector<uint8_t> maps(nr * 128);
     if (swk::encode_tmaps(maps.data(), base.data(), bytes.data(), (int)nr, std::min<uint64_t>(c->plan.C, c->seg))) {
+      for (size_t r = 0; r < nr; ++r)  // a region without a map (smaller than one row, or > 2^31 rows) never
+        if (std::all_of(maps.begin() + r * 128, maps.begin() + (r + 1) * 128, [](uint8_t b) { return b == 0; }))
+          span[r].y = 0;  // takes the tensor path: its span is empty for the kernel's range check
       CUDA_TRY(c, cudaMalloc(&c->d_tmaps, maps.size()));
       CUDA_TRY(c, cudaMemcpy(c->d_tmaps, maps.data(), maps.size(), cudaMemcpyHostToDevice));
       CUDA_TRY(c, cudaMalloc(&c->d_reg_span, nr * sizeof(ulonglong2)));
