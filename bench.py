@@ -104,6 +104,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-assisted", action="store_true", help="skip the N>1 NVLink-assisted restore leg")
     ap.add_argument("--no-dp", action="store_true", help="skip the N>1 data-parallel replica leg")
+    ap.add_argument("--legs-timeout", type=float, default=480.0,
+                    help="N>1: seconds after the main measurement before the assisted / DP legs are abandoned "
+                         "(the line is printed with what they recorded)")
     ap.add_argument("--force-legs", action="store_true",
                     help="run the N>1 assisted and DP legs even over gloo / on one device (tests: degenerate helpers)")
     ap.add_argument("--sample-bytes", type=int, default=8 << 30, help="oracle sample size per step")
@@ -639,12 +642,139 @@ def run_ours(args):
     del h
     ce_all = gather_obj({k: round(v, 2) for k, v in ce.items()})
 
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:  # the oracle beside N=1 only
+        import oracle
+
+        sample, _ = oracle_sample_specs(specs, args.sample_bytes)
+        s_offs, s_total = W.place(sample)
+        s_host = arena[:s_total].cpu().numpy()  # same placement recipe: the arena prefix holds the sample
+        th = cpu_threads()
+        ref_rates, sbytes = time_oracle_restore(oracle, sample, s_host, s_offs, th, 3)
+        fast_rates, _ = time_oracle_restore(oracle, sample, s_host, s_offs, th, 3, fast=True)
+        del s_host
+        cpu = {"value": round(statistics.mean(ref_rates), 3), "unit": "GB/s", "cores": th, "kind": "oracle",
+               "sample": f"oracle_restore (memcpy + Sarwate CRC-32C per 1 MiB chunk) over the first {len(sample)} "
+                         f"regions of workload {name} ({sbytes} B = {sbytes / payload:.1%} of the image, contents "
+                         f"copied from the GPU arena), {th} OpenMP threads, mean of 3",
+               "fast": {"value": round(statistics.mean(fast_rates), 3), "unit": "GB/s",
+                        "how": "same sample and threads, CRC-32C by the SSE4.2 crc32 instruction"},
+               **cpu_context(my_cpus)}
+
+    clk_all = gather_obj({k: clk.get(k) for k in ("sm_mhz", "samples", "reasons")})
+    numa = sw.numa()
+    placement = gather_obj({"rank": rank, "gpu": local_dev, "gpu_numa_node": node, "cpus": len(my_cpus),
+                            "image_numa_node": numa["node"], "image_local_fraction": numa["local_fraction"]})
+    emitted = threading.Event()
+
+    def emit(assisted, dp, legs_note=None):
+        """Rank 0 prints the one JSON line (once: the normal end, or the legs watchdog)."""
+        if rank != 0 or emitted.is_set():
+            return
+        emitted.set()
+        value = total_payload / (swapin_ms * 1e-3) / GB
+        achieved = payload / (restore_ms * 1e-3) / GB
+        peaks = json.load(open(MEASURED_PEAKS)) if os.path.exists(MEASURED_PEAKS) else {}
+        hbm_peak = peaks.get("hbm_gbs", 6650.0)
+        workload_name = f"{name}: {desc}" + ("" if kv_scale == 1.0 else f" -- KV pool SHRUNK x{kv_scale} to fit host RAM (not the named config)")
+        line = {
+            "metric": METRIC if kv_scale == 1.0 else METRIC + " (KV pool shrunk)", "value": round(value, 3),
+            "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(step_ms, 3), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "u8", "data": "synthetic",
+            "config": {"workload": workload_name,
+                       "regions_per_rank": len(specs),
+                       "payload_bytes_per_rank": payload, "chunk_bytes": args.chunk, "seg_bytes": args.seg_bytes or "auto", "checksum": args.checksum,
+                       "mechanism": f"{args.mechanism} -> restore {eff_mech}, checkpoint {eff_mech_ckpt}",
+                       "l2": "no flush: every step moves the whole image (>> 126 MB L2)",
+                       "parallelism": "single GPU" if world == 1 else f"tp{world} shard per rank (no data collective)",
+                       "timing": "per step: barrier, then restore + HBM verify + K6 all-reduce on the ctx stream (CUDA "
+                                 "events); value uses the mean over steps of the per-step max over ranks"},
+            "swap_in_latency_s": round(swapin_ms * 1e-3, 5),
+            "swap_in_latency_s_range": [round(min(swapin_steps) * 1e-3, 5), round(max(swapin_steps) * 1e-3, 5)],
+            "swap_in_latency_s_median": round(statistics.median(swapin_steps) * 1e-3, 5),
+            "restore_GBps_per_gpu": round(achieved, 3),
+            "restore_GBps_per_gpu_slowest": round(payload / (max(restore_steps) * 1e-3) / GB, 3),
+            "checkpoint_GBps_per_gpu": round(payload / (ckpt_ms * 1e-3) / GB, 3),
+            # roofline = the HBM verify pass (a8), the kernel on the swap-in's critical path (~10 ms after the
+            # ~950 ms link transfer). In the serialised ncu launch list (profiles/r02_ncu_launches_bench_B_ts.md)
+            # the CE_PIPE restore's per-group checks hold the largest summed share, but they run on a side stream
+            # under the copy engine's H2D copies, off the critical path: roofline_group_checks times them live
+            "roofline": {"bound": "hbm", "kernel": VERIFY_KERNEL[args.checksum],
+                         "achieved": round(payload / (verify_ms * 1e-3) / GB, 1), "peak": hbm_peak,
+                         "unit": "GB/s", "frac": round(payload / (verify_ms * 1e-3) / GB / hbm_peak, 4),
+                         "traffic": (ncu_traffic(name, args.checksum, payload) or {}).get("bytes"),
+                         "algorithmic_bytes_per_launch": payload,
+                         "how": "payload bytes (1 B HBM read per image byte) / the verify launch's mean duration "
+                                "(CUDA events on the ctx stream over the timed steps)",
+                         "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy; a read-only stream can exceed it)"},
+            "roofline_link": {"bound": "host_link", "kernel": RESTORE_KERNEL[eff_mech],
+                         "achieved": round(achieved, 3), "peak": PCIE_GEN5_X16_GBPS, "unit": "GB/s",
+                         "frac": round(achieved / PCIE_GEN5_X16_GBPS, 4), "traffic": None,
+                         "traffic_note": "copy-engine / link transfer: no kernel DRAM counters (see roofline_verify.traffic)",
+                         "peak_source": "PCIe Gen5 x16 nominal per direction after 128b/130b (MEASURED_PEAKS.json has no host-link figure)",
+                         "frac_of_measured_ce_h2d": round(achieved / ce["h2d"], 4)},
+            "roofline_group_checks": group_checks(rec, payload, hbm_peak, eff_mech),
+            "roofline_verify": {"bound": "hbm", "kernel": VERIFY_KERNEL[args.checksum],
+                                "achieved": round(payload / (verify_ms * 1e-3) / GB, 1), "peak": hbm_peak,
+                                "unit": "GB/s", "frac": round(payload / (verify_ms * 1e-3) / GB / hbm_peak, 4),
+                                "traffic": (ncu_traffic(name, args.checksum, payload) or {}).get("bytes"),
+                                "traffic_detail": ncu_traffic(name, args.checksum, payload),
+                                "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)"},
+            "measured_ce_GBps": {k: round(v, 2) for k, v in ce.items()},
+            "measured_ce_GBps_all_ranks": ce_all,
+            "mechanisms": compare,
+            "fused_checksum_overhead": overhead(compare, achieved, ce),
+            "assisted_swap_in": assisted,
+            "dp_replicas": dp,
+            "setup_s": {"fill": round(t_fill, 2), "register_pin": round(t_register, 2)},
+            "swap_in_with_hbm_reacquire_s": round(statistics.mean(x[1] for x in reacq), 4),
+            "hbm_reacquire_s": round(statistics.mean(x[0] for x in reacq), 4),
+            "swap_in_with_overlapped_reacquire_s": round(statistics.mean(lazy), 4),
+            "e2e": {"value": round(total_payload / (host_ms * 1e-3) / GB, 3), "unit": "GB/s",
+                    "h2d_bytes_per_step": payload, "d2h_bytes_per_step": 32,
+                    "how": "host wall clock (perf_counter) around swap_restore + swap_verify (+ the K6 all-reduce) "
+                           "called through the C ABI (ctypes), image in pinned host DRAM: the H2D copy of every payload "
+                           "byte and the D2H read of the 32-B verify status are inside; per-step max over ranks. The "
+                           "harness poison is finished before the clock starts. It lands near the device-timed value "
+                           "because the device-timed metric is itself the host-to-device transfer"},
+            "gpu_launches": int(launches),
+            "clocks": clk,
+            "clocks_all_ranks": clk_all if world > 1 else None,
+            "placement": placement,
+            "topology": topology(),
+            "cpu_baseline": cpu,
+        }
+        if legs_note:
+            line["legs_note"] = legs_note
+        s = json.dumps(line)
+        print(s, flush=True)
+        if args.out:
+            with open(args.out, "a") as f:
+                f.write(s + "\n")
+
+    # The N>1 legs below run code paths (peer helpers, NCCL stripe broadcasts, VMM fd exchange) that only a
+    # multi-GPU box exercises; a hang there must not cost the measured line: after --legs-timeout seconds
+    # every rank gives up on them, rank 0 prints the line with what the legs recorded so far, and all exit 0.
+    legs = {"assisted": None, "dp": None}
+
+    def legs_timeout():
+        emit(legs["assisted"], legs["dp"], f"N>1 legs abandoned after {args.legs_timeout:.0f} s (timeout)")
+        sys.stdout.flush()
+        os._exit(0)
+
+    dog = threading.Timer(args.legs_timeout, legs_timeout) if world > 1 else None
+    if dog is not None:
+        dog.daemon = True
+        dog.start()
+
     # NEXT-2: rank 0's swap-in assisted by k idle peers (their PCIe links into HBM staging, then NVLink),
     # the other ranks idle in a barrier (outside the timed region)
     assisted = None
     multi = world > 1 and ((args.dist_backend == "nccl" and ndev > 1) or args.force_legs)
     if multi and not args.no_assisted:
         assisted = {}
+        legs["assisted"] = assisted
         for k in (1, 3, 7):
             if k > (world - 1 if args.force_legs else min(world, ndev) - 1):  # helpers: the job's own GPUs
                 break
@@ -687,29 +817,6 @@ def run_ours(args):
                 assisted[str(k)] = rec_k
             barrier()
 
-    cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:  # the oracle beside N=1 only
-        import oracle
-
-        sample, _ = oracle_sample_specs(specs, args.sample_bytes)
-        s_offs, s_total = W.place(sample)
-        s_host = arena[:s_total].cpu().numpy()  # same placement recipe: the arena prefix holds the sample
-        th = cpu_threads()
-        ref_rates, sbytes = time_oracle_restore(oracle, sample, s_host, s_offs, th, 3)
-        fast_rates, _ = time_oracle_restore(oracle, sample, s_host, s_offs, th, 3, fast=True)
-        del s_host
-        cpu = {"value": round(statistics.mean(ref_rates), 3), "unit": "GB/s", "cores": th, "kind": "oracle",
-               "sample": f"oracle_restore (memcpy + Sarwate CRC-32C per 1 MiB chunk) over the first {len(sample)} "
-                         f"regions of workload {name} ({sbytes} B = {sbytes / payload:.1%} of the image, contents "
-                         f"copied from the GPU arena), {th} OpenMP threads, mean of 3",
-               "fast": {"value": round(statistics.mean(fast_rates), 3), "unit": "GB/s",
-                        "how": "same sample and threads, CRC-32C by the SSE4.2 crc32 instruction"},
-               **cpu_context(my_cpus)}
-
-    clk_all = gather_obj({k: clk.get(k) for k in ("sm_mhz", "samples", "reasons")})
-    numa = sw.numa()
-    placement = gather_obj({"rank": rank, "gpu": local_dev, "gpu_numa_node": node, "cpus": len(my_cpus),
-                            "image_numa_node": numa["node"], "image_local_fraction": numa["local_fraction"]})
     sw.close()
     vmm.close()
     del arena
@@ -784,85 +891,10 @@ def run_ours(args):
         if vmm0 is not None:
             vmm0.close()
 
-    if rank == 0:
-        value = total_payload / (swapin_ms * 1e-3) / GB
-        achieved = payload / (restore_ms * 1e-3) / GB
-        peaks = json.load(open(MEASURED_PEAKS)) if os.path.exists(MEASURED_PEAKS) else {}
-        hbm_peak = peaks.get("hbm_gbs", 6650.0)
-        workload_name = f"{name}: {desc}" + ("" if kv_scale == 1.0 else f" -- KV pool SHRUNK x{kv_scale} to fit host RAM (not the named config)")
-        line = {
-            "metric": METRIC if kv_scale == 1.0 else METRIC + " (KV pool shrunk)", "value": round(value, 3),
-            "unit": "GB/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": round(step_ms, 3), "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
-            "dtype": "u8", "data": "synthetic",
-            "config": {"workload": workload_name,
-                       "regions_per_rank": len(specs),
-                       "payload_bytes_per_rank": payload, "chunk_bytes": args.chunk, "seg_bytes": args.seg_bytes or "auto", "checksum": args.checksum,
-                       "mechanism": f"{args.mechanism} -> restore {eff_mech}, checkpoint {eff_mech_ckpt}",
-                       "l2": "no flush: every step moves the whole image (>> 126 MB L2)",
-                       "parallelism": "single GPU" if world == 1 else f"tp{world} shard per rank (no data collective)",
-                       "timing": "per step: barrier, then restore + HBM verify + K6 all-reduce on the ctx stream (CUDA "
-                                 "events); value uses the mean over steps of the per-step max over ranks"},
-            "swap_in_latency_s": round(swapin_ms * 1e-3, 5),
-            "swap_in_latency_s_range": [round(min(swapin_steps) * 1e-3, 5), round(max(swapin_steps) * 1e-3, 5)],
-            "swap_in_latency_s_median": round(statistics.median(swapin_steps) * 1e-3, 5),
-            "restore_GBps_per_gpu": round(achieved, 3),
-            "restore_GBps_per_gpu_slowest": round(payload / (max(restore_steps) * 1e-3) / GB, 3),
-            "checkpoint_GBps_per_gpu": round(payload / (ckpt_ms * 1e-3) / GB, 3),
-            # roofline = the HBM verify pass (a8), the kernel on the swap-in's critical path (~10 ms after the
-            # ~950 ms link transfer). In the serialised ncu launch list (profiles/r02_ncu_launches_bench_B_ts.md)
-            # the CE_PIPE restore's per-group checks hold the largest summed share, but they run on a side stream
-            # under the copy engine's H2D copies, off the critical path: roofline_group_checks times them live
-            "roofline": {"bound": "hbm", "kernel": VERIFY_KERNEL[args.checksum],
-                         "achieved": round(payload / (verify_ms * 1e-3) / GB, 1), "peak": hbm_peak,
-                         "unit": "GB/s", "frac": round(payload / (verify_ms * 1e-3) / GB / hbm_peak, 4),
-                         "traffic": (ncu_traffic(name, args.checksum, payload) or {}).get("bytes"),
-                         "algorithmic_bytes_per_launch": payload,
-                         "how": "payload bytes (1 B HBM read per image byte) / the verify launch's mean duration "
-                                "(CUDA events on the ctx stream over the timed steps)",
-                         "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy; a read-only stream can exceed it)"},
-            "roofline_link": {"bound": "host_link", "kernel": RESTORE_KERNEL[eff_mech],
-                         "achieved": round(achieved, 3), "peak": PCIE_GEN5_X16_GBPS, "unit": "GB/s",
-                         "frac": round(achieved / PCIE_GEN5_X16_GBPS, 4), "traffic": None,
-                         "traffic_note": "copy-engine / link transfer: no kernel DRAM counters (see roofline_verify.traffic)",
-                         "peak_source": "PCIe Gen5 x16 nominal per direction after 128b/130b (MEASURED_PEAKS.json has no host-link figure)",
-                         "frac_of_measured_ce_h2d": round(achieved / ce["h2d"], 4)},
-            "roofline_group_checks": group_checks(rec, payload, hbm_peak, eff_mech),
-            "roofline_verify": {"bound": "hbm", "kernel": VERIFY_KERNEL[args.checksum],
-                                "achieved": round(payload / (verify_ms * 1e-3) / GB, 1), "peak": hbm_peak,
-                                "unit": "GB/s", "frac": round(payload / (verify_ms * 1e-3) / GB / hbm_peak, 4),
-                                "traffic": (ncu_traffic(name, args.checksum, payload) or {}).get("bytes"),
-                                "traffic_detail": ncu_traffic(name, args.checksum, payload),
-                                "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured)"},
-            "measured_ce_GBps": {k: round(v, 2) for k, v in ce.items()},
-            "measured_ce_GBps_all_ranks": ce_all,
-            "mechanisms": compare,
-            "fused_checksum_overhead": overhead(compare, achieved, ce),
-            "assisted_swap_in": assisted,
-            "dp_replicas": dp,
-            "setup_s": {"fill": round(t_fill, 2), "register_pin": round(t_register, 2)},
-            "swap_in_with_hbm_reacquire_s": round(statistics.mean(x[1] for x in reacq), 4),
-            "hbm_reacquire_s": round(statistics.mean(x[0] for x in reacq), 4),
-            "swap_in_with_overlapped_reacquire_s": round(statistics.mean(lazy), 4),
-            "e2e": {"value": round(total_payload / (host_ms * 1e-3) / GB, 3), "unit": "GB/s",
-                    "h2d_bytes_per_step": payload, "d2h_bytes_per_step": 32,
-                    "how": "host wall clock (perf_counter) around swap_restore + swap_verify (+ the K6 all-reduce) "
-                           "called through the C ABI (ctypes), image in pinned host DRAM: the H2D copy of every payload "
-                           "byte and the D2H read of the 32-B verify status are inside; per-step max over ranks. The "
-                           "harness poison is finished before the clock starts. It lands near the device-timed value "
-                           "because the device-timed metric is itself the host-to-device transfer"},
-            "gpu_launches": int(launches),
-            "clocks": clk,
-            "clocks_all_ranks": clk_all if world > 1 else None,
-            "placement": placement,
-            "topology": topology(),
-            "cpu_baseline": cpu,
-        }
-        s = json.dumps(line)
-        print(s, flush=True)
-        if args.out:
-            with open(args.out, "a") as f:
-                f.write(s + "\n")
+    legs["dp"] = dp
+    if dog is not None:
+        dog.cancel()
+    emit(assisted, dp)
     if world > 1:
         tdist.barrier()
         tdist.destroy_process_group()

@@ -57,3 +57,21 @@ def test_bench_two_ranks_gloo_config_d():
     assert rec["topology"]["numa_nodes"] and rec["clocks"]["samples"] > 0
     lo, hi = rec["swap_in_latency_s_range"]
     assert lo <= rec["swap_in_latency_s"] <= hi
+
+
+@pytest.mark.timeout(600)
+def test_bench_two_ranks_legs_watchdog():
+    """A hang in the N>1 legs must not cost the measured line: with a legs timeout shorter than the legs, every
+    rank abandons them, rank 0 prints the line (with a legs_note and what the legs had recorded) and the job
+    exits 0."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr=127.0.0.1", "--master-port=29537", os.path.join(ROOT, "bench.py"), "--gpus", "2",
+           "--config", "A", "--steps", "2", "--warmup", "1", "--no-compare", "--no-cpu-baseline",
+           "--dist-backend", "gloo", "--force-legs", "--legs-timeout", "0.5"]
+    out = subprocess.run(cmd, capture_output=True, text=True, timeout=540, cwd=ROOT)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, out.stdout
+    rec = json.loads(lines[0])
+    assert rec["n_gpus"] == 2 and rec["value"] > 0
+    assert "timeout" in rec["legs_note"]
