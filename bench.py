@@ -759,6 +759,8 @@ def run_ours(args):
     legs = {"assisted": None, "dp": None}
 
     def legs_timeout():
+        if rank != 0:  # let rank 0 print first: its main thread may be in a collective with this rank
+            time.sleep(10)
         emit(legs["assisted"], legs["dp"], f"N>1 legs abandoned after {args.legs_timeout:.0f} s (timeout)")
         sys.stdout.flush()
         os._exit(0)
@@ -868,13 +870,18 @@ def run_ours(args):
                 swd.restore(stream)
                 return swd.verify(stream, hbm_pass=True)
 
-            with torch.cuda.stream(stream):
-                t_striped = timed(lambda: sdist.restore_replicas(swd, None, stream))
-                t_indep = timed(independent)
-                try:  # fused NVLink pull: the other replicas' VMM arenas mapped here (slab fds over Unix sockets)
-                    t_pull = timed(lambda: sdist.pull_replicas(swd, None, None, stream, arena=vmm0))
-                except Exception as ex:  # noqa: BLE001
-                    t_pull = f"{type(ex).__name__}: {ex}"[:200]
+            try:
+                with torch.cuda.stream(stream):
+                    t_striped = timed(lambda: sdist.restore_replicas(swd, None, stream))
+                    t_indep = timed(independent)
+                    try:  # fused NVLink pull: the other replicas' VMM arenas mapped here (slab fds over Unix sockets)
+                        t_pull = timed(lambda: sdist.pull_replicas(swd, None, None, stream, arena=vmm0))
+                    except Exception as ex:  # noqa: BLE001
+                        t_pull = f"{type(ex).__name__}: {ex}"[:200]
+            except Exception as ex:  # noqa: BLE001 - an informational leg must not sink the line
+                t_striped = None
+                dp = {"error": f"rank {rank}: {type(ex).__name__}: {ex}"[:300]}
+        if dp is None and swd is not None and t_striped is not None:
             dp = {"replicas": world, "image_bytes": payload0, "striped_swap_in_s": round(t_striped, 4),
                   "independent_swap_in_s": round(t_indep, 4), "speedup": round(t_indep / t_striped, 3),
                   "striped_GBps_per_replica": round(payload0 / t_striped / GB, 2),
