@@ -665,13 +665,18 @@ def run_ours(args):
     numa = sw.numa()
     placement = gather_obj({"rank": rank, "gpu": local_dev, "gpu_numa_node": node, "cpus": len(my_cpus),
                             "image_numa_node": numa["node"], "image_local_fraction": numa["local_fraction"]})
-    emitted = threading.Event()
+    emit_lock = threading.Lock()
+    emitted = []
 
     def emit(assisted, dp, legs_note=None):
         """Rank 0 prints the one JSON line (once: the normal end, or the legs watchdog)."""
-        if rank != 0 or emitted.is_set():
-            return
-        emitted.set()
+        with emit_lock:
+            if rank != 0 or emitted:
+                return
+            emitted.append(True)
+            emit_locked(assisted, dp, legs_note)
+
+    def emit_locked(assisted, dp, legs_note):
         value = total_payload / (swapin_ms * 1e-3) / GB
         achieved = payload / (restore_ms * 1e-3) / GB
         peaks = json.load(open(MEASURED_PEAKS)) if os.path.exists(MEASURED_PEAKS) else {}
@@ -758,9 +763,12 @@ def run_ours(args):
     # every rank gives up on them, rank 0 prints the line with what the legs recorded so far, and all exit 0.
     legs = {"assisted": None, "dp": None}
 
+    fired = threading.Event()
+
     def legs_timeout():
-        if rank != 0:  # let rank 0 print first: its main thread may be in a collective with this rank
-            time.sleep(10)
+        fired.set()
+        if rank != 0:  # let rank 0 print first (its main thread may be in a collective with this rank)
+            time.sleep(2)
         emit(legs["assisted"], legs["dp"], f"N>1 legs abandoned after {args.legs_timeout:.0f} s (timeout)")
         sys.stdout.flush()
         os._exit(0)
@@ -770,133 +778,140 @@ def run_ours(args):
         dog.daemon = True
         dog.start()
 
-    # NEXT-2: rank 0's swap-in assisted by k idle peers (their PCIe links into HBM staging, then NVLink),
-    # the other ranks idle in a barrier (outside the timed region)
-    assisted = None
-    multi = world > 1 and ((args.dist_backend == "nccl" and ndev > 1) or args.force_legs)
-    if multi and not args.no_assisted:
-        assisted = {}
-        legs["assisted"] = assisted
-        for k in (1, 3, 7):
-            if k > (world - 1 if args.force_legs else min(world, ndev) - 1):  # helpers: the job's own GPUs
-                break
-            barrier()
-            if rank == 0:
-                helpers = [(local_dev + i) % ndev for i in range(1, k + 1)]
-                rec_k = {"helpers": helpers}
-                for mode in ("fused", "copy"):  # SM pull over NVLink with the fused check / peer copies + hash
-                    try:
-                        if mode == "copy":
-                            os.environ["SWAP_ASSIST"] = "copy"
-                        else:
-                            os.environ.pop("SWAP_ASSIST", None)
-                        sw.set_mechanism("ce_pipe")
-                        sw.set_helpers(helpers)
-                        ts = []
-                        for _ in range(3):
-                            poison()
-                            stream.synchronize()
-                            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                            e0.record(stream)
-                            sw.restore(stream)
-                            res = sw.verify(stream, hbm_pass=True)
-                            e1.record(stream)
-                            e1.synchronize()
-                            assert res["status"] == 0 and res["n_bad"] == 0 and res["hbm_n_bad"] == 0, res
-                            ts.append(e0.elapsed_time(e1) * 1e-3)
-                        t = statistics.median(ts[1:])
-                        rec_k[mode] = {"swap_in_s": round(t, 4), "GBps": round(payload / t / GB, 2),
-                                       "frac_of_k_plus_1_links": round(payload / t / GB / ((k + 1) * ce["h2d"]), 3)}
-                    except Exception as ex:  # noqa: BLE001 - an informational leg must not sink the line
-                        rec_k[mode] = {"error": f"{type(ex).__name__}: {ex}"[:300]}
-                    finally:
-                        os.environ.pop("SWAP_ASSIST", None)
+    try:
+        # NEXT-2: rank 0's swap-in assisted by k idle peers (their PCIe links into HBM staging, then NVLink),
+        # the other ranks idle in a barrier (outside the timed region)
+        assisted = None
+        multi = world > 1 and ((args.dist_backend == "nccl" and ndev > 1) or args.force_legs)
+        if multi and not args.no_assisted:
+            assisted = {}
+            legs["assisted"] = assisted
+            for k in (1, 3, 7):
+                if k > (world - 1 if args.force_legs else min(world, ndev) - 1):  # helpers: the job's own GPUs
+                    break
+                barrier()
+                if rank == 0:
+                    helpers = [(local_dev + i) % ndev for i in range(1, k + 1)]
+                    rec_k = {"helpers": helpers}
+                    for mode in ("fused", "copy"):  # SM pull over NVLink with the fused check / peer copies + hash
                         try:
-                            sw.set_helpers([])
-                            sw.set_mechanism(args.mechanism)
-                        except Exception:  # noqa: BLE001
-                            pass
-                assisted[str(k)] = rec_k
-            barrier()
+                            if mode == "copy":
+                                os.environ["SWAP_ASSIST"] = "copy"
+                            else:
+                                os.environ.pop("SWAP_ASSIST", None)
+                            sw.set_mechanism("ce_pipe")
+                            sw.set_helpers(helpers)
+                            ts = []
+                            for _ in range(3):
+                                poison()
+                                stream.synchronize()
+                                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                                e0.record(stream)
+                                sw.restore(stream)
+                                res = sw.verify(stream, hbm_pass=True)
+                                e1.record(stream)
+                                e1.synchronize()
+                                assert res["status"] == 0 and res["n_bad"] == 0 and res["hbm_n_bad"] == 0, res
+                                ts.append(e0.elapsed_time(e1) * 1e-3)
+                            t = statistics.median(ts[1:])
+                            rec_k[mode] = {"swap_in_s": round(t, 4), "GBps": round(payload / t / GB, 2),
+                                           "frac_of_k_plus_1_links": round(payload / t / GB / ((k + 1) * ce["h2d"]), 3)}
+                        except Exception as ex:  # noqa: BLE001 - an informational leg must not sink the line
+                            rec_k[mode] = {"error": f"{type(ex).__name__}: {ex}"[:300]}
+                        finally:
+                            os.environ.pop("SWAP_ASSIST", None)
+                            try:
+                                sw.set_helpers([])
+                                sw.set_mechanism(args.mechanism)
+                            except Exception:  # noqa: BLE001
+                                pass
+                    assisted[str(k)] = rec_k
+                barrier()
 
-    sw.close()
-    vmm.close()
-    del arena
+        sw.close()
+        vmm.close()
+        del arena
 
-    # NEXT-2, data-parallel replicas (outside the timed region): every rank holds a replica of rank 0's
-    # engine image; striped swap-in (each replica pulls 1/N over its own link, stripes broadcast over
-    # NVLink, HBM verify of everything) vs every replica pulling the whole image over its own link
-    dp = None
-    if multi and not args.no_dp:
-        dp_err, swd, arena0, vmm0 = "", None, None, None
-        try:  # local setup first; collectives only if every rank got this far
-            _, specs0, _ = workload(args.config, 0, world)
-            offs0, bytes0 = W.place(specs0)
-            vmm0 = swap.Arena(bytes0, device=local_dev)  # the product's releasable HBM
-            base0, arena0 = vmm0.alloc(bytes0)
-            W.fill_device_arena(arena0, specs0, offs0, seed=0)  # identical bytes on every replica
-            regions0 = [(base0 + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs0, offs0))]
-            payload0 = sum(r.nbytes for r in specs0)
-            swd = swap.Swapper(regions0, chunk_bytes=args.chunk, checksum=kind, mechanism="ce_pipe", device=local_dev)
-            with torch.cuda.stream(stream):
-                swd.checkpoint(stream, sync=True)
-        except Exception as ex:  # noqa: BLE001
-            dp_err = f"rank {rank}: {type(ex).__name__}: {ex}"[:300]
-        if allreduce([1.0 if dp_err else 0.0], tdist.ReduceOp.MAX)[0] > 0:
-            dp = {"error": dp_err or "setup failed on another rank"}
-        else:
-            def poison0():
+        # NEXT-2, data-parallel replicas (outside the timed region): every rank holds a replica of rank 0's
+        # engine image; striped swap-in (each replica pulls 1/N over its own link, stripes broadcast over
+        # NVLink, HBM verify of everything) vs every replica pulling the whole image over its own link
+        dp = None
+        if multi and not args.no_dp:
+            dp_err, swd, arena0, vmm0 = "", None, None, None
+            try:  # local setup first; collectives only if every rank got this far
+                _, specs0, _ = workload(args.config, 0, world)
+                offs0, bytes0 = W.place(specs0)
+                vmm0 = swap.Arena(bytes0, device=local_dev)  # the product's releasable HBM
+                base0, arena0 = vmm0.alloc(bytes0)
+                W.fill_device_arena(arena0, specs0, offs0, seed=0)  # identical bytes on every replica
+                regions0 = [(base0 + o, r.nbytes, r.kind, i) for i, (r, o) in enumerate(zip(specs0, offs0))]
+                payload0 = sum(r.nbytes for r in specs0)
+                swd = swap.Swapper(regions0, chunk_bytes=args.chunk, checksum=kind, mechanism="ce_pipe", device=local_dev)
                 with torch.cuda.stream(stream):
-                    for r, o in zip(specs0, offs0):
-                        if r.nbytes:
-                            arena0[o:o + r.nbytes].fill_(W.POISON_BYTE)
-                stream.synchronize()
+                    swd.checkpoint(stream, sync=True)
+            except Exception as ex:  # noqa: BLE001
+                dp_err = f"rank {rank}: {type(ex).__name__}: {ex}"[:300]
+            if allreduce([1.0 if dp_err else 0.0], tdist.ReduceOp.MAX)[0] > 0:
+                dp = {"error": dp_err or "setup failed on another rank"}
+            else:
+                def poison0():
+                    with torch.cuda.stream(stream):
+                        for r, o in zip(specs0, offs0):
+                            if r.nbytes:
+                                arena0[o:o + r.nbytes].fill_(W.POISON_BYTE)
+                    stream.synchronize()
 
-            def timed(fn):
-                ts = []
-                for _ in range(3):
-                    poison0()
-                    barrier()
-                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                    e0.record(stream)
-                    res = fn()
-                    e1.record(stream)
-                    e1.synchronize()
-                    assert res["status"] == 0 and res["n_bad"] == 0 and res["hbm_n_bad"] == 0, res
-                    ts.append(e0.elapsed_time(e1) * 1e-3)
-                return statistics.median(allreduce(ts, tdist.ReduceOp.MAX)[1:])
+                def timed(fn):
+                    ts = []
+                    for _ in range(3):
+                        poison0()
+                        barrier()
+                        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                        e0.record(stream)
+                        res = fn()
+                        e1.record(stream)
+                        e1.synchronize()
+                        assert res["status"] == 0 and res["n_bad"] == 0 and res["hbm_n_bad"] == 0, res
+                        ts.append(e0.elapsed_time(e1) * 1e-3)
+                    return statistics.median(allreduce(ts, tdist.ReduceOp.MAX)[1:])
 
-            def independent():
-                swd.restore(stream)
-                return swd.verify(stream, hbm_pass=True)
+                def independent():
+                    swd.restore(stream)
+                    return swd.verify(stream, hbm_pass=True)
 
-            try:
-                with torch.cuda.stream(stream):
-                    t_striped = timed(lambda: sdist.restore_replicas(swd, None, stream))
-                    t_indep = timed(independent)
-                    try:  # fused NVLink pull: the other replicas' VMM arenas mapped here (slab fds over Unix sockets)
-                        t_pull = timed(lambda: sdist.pull_replicas(swd, None, None, stream, arena=vmm0))
-                    except Exception as ex:  # noqa: BLE001
-                        t_pull = f"{type(ex).__name__}: {ex}"[:200]
-            except Exception as ex:  # noqa: BLE001 - an informational leg must not sink the line
-                t_striped = None
-                dp = {"error": f"rank {rank}: {type(ex).__name__}: {ex}"[:300]}
-        if dp is None and swd is not None and t_striped is not None:
-            dp = {"replicas": world, "image_bytes": payload0, "striped_swap_in_s": round(t_striped, 4),
-                  "independent_swap_in_s": round(t_indep, 4), "speedup": round(t_indep / t_striped, 3),
-                  "striped_GBps_per_replica": round(payload0 / t_striped / GB, 2),
-                  "striped_fused_pull_swap_in_s": round(t_pull, 4) if isinstance(t_pull, float) else t_pull,
-                  "host_link_bytes_per_replica": payload0 // world,
-                  "how": "swap_restore_stripe (1/N of the CE_PIPE groups per replica over its own PCIe link) + in-place "
-                         "NCCL broadcasts of every stripe span from its owner + HBM verify of all chunks, max over ranks; "
-                         "fused pull: the other stripes read from the owners' HBM over NVLink by the SM mover with the "
-                         "chunk check from the same registers (swap_pull_stripes; the peers' VMM arenas mapped per "
-                         "swap-in via exported slab fds, included in the time), then the HBM verify"}
-        if swd is not None:
-            swd.close()
-        del arena0
-        if vmm0 is not None:
-            vmm0.close()
+                try:
+                    with torch.cuda.stream(stream):
+                        t_striped = timed(lambda: sdist.restore_replicas(swd, None, stream))
+                        t_indep = timed(independent)
+                        try:  # fused NVLink pull: the other replicas' VMM arenas mapped here (slab fds over Unix sockets)
+                            t_pull = timed(lambda: sdist.pull_replicas(swd, None, None, stream, arena=vmm0))
+                        except Exception as ex:  # noqa: BLE001
+                            t_pull = f"{type(ex).__name__}: {ex}"[:200]
+                except Exception as ex:  # noqa: BLE001 - an informational leg must not sink the line
+                    t_striped = None
+                    dp = {"error": f"rank {rank}: {type(ex).__name__}: {ex}"[:300]}
+            if dp is None and swd is not None and t_striped is not None:
+                dp = {"replicas": world, "image_bytes": payload0, "striped_swap_in_s": round(t_striped, 4),
+                      "independent_swap_in_s": round(t_indep, 4), "speedup": round(t_indep / t_striped, 3),
+                      "striped_GBps_per_replica": round(payload0 / t_striped / GB, 2),
+                      "striped_fused_pull_swap_in_s": round(t_pull, 4) if isinstance(t_pull, float) else t_pull,
+                      "host_link_bytes_per_replica": payload0 // world,
+                      "how": "swap_restore_stripe (1/N of the CE_PIPE groups per replica over its own PCIe link) + in-place "
+                             "NCCL broadcasts of every stripe span from its owner + HBM verify of all chunks, max over ranks; "
+                             "fused pull: the other stripes read from the owners' HBM over NVLink by the SM mover with the "
+                             "chunk check from the same registers (swap_pull_stripes; the peers' VMM arenas mapped per "
+                             "swap-in via exported slab fds, included in the time), then the HBM verify"}
+            if swd is not None:
+                swd.close()
+            del arena0
+            if vmm0 is not None:
+                vmm0.close()
+    except BaseException:
+        # a leg died (e.g. a peer that the watchdog already ended): let the watchdog print the line and exit
+        if dog is not None and (fired.is_set() or fired.wait(args.legs_timeout + 5)):
+            while True:
+                time.sleep(1)
+        raise
 
     legs["dp"] = dp
     if dog is not None:

@@ -67,7 +67,7 @@ def test_bench_two_ranks_legs_watchdog():
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr=127.0.0.1", "--master-port=29537", os.path.join(ROOT, "bench.py"), "--gpus", "2",
            "--config", "A", "--steps", "2", "--warmup", "1", "--no-compare", "--no-cpu-baseline",
-           "--dist-backend", "gloo", "--force-legs", "--legs-timeout", "0.5"]
+           "--dist-backend", "gloo", "--force-legs", "--legs-timeout", "0.01"]
     out = subprocess.run(cmd, capture_output=True, text=True, timeout=540, cwd=ROOT)
     assert out.returncode == 0, out.stderr[-3000:]
     lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
