@@ -80,6 +80,10 @@ struct swap_ctx {
   swk::DevStatus* d_status = nullptr;
   swk::DevStatus* h_status = nullptr;  // pinned
   uint32_t* d_tables = nullptr;
+  // device copy of the manifest's chunk records, staged by copy-engine restores so that the hash kernels
+  // read the expected checksums from HBM, not over a host link saturated by the restore's own copies
+  uint8_t* d_exp = nullptr;
+  bool exp_valid = false;  // d_exp matches the manifest (cleared by checkpoint / import)
   void* d_tmaps = nullptr;             // strand-staged CRC kernel: per-region tensor maps (null: none)
   uint32_t* d_chunk_region = nullptr;  // [n_chunks] region index
   ulonglong2* d_reg_span = nullptr;    // [n_regions] {device base, bytes}
@@ -137,6 +141,7 @@ swk::Params base_params(swap_ctx* c, const DescSet& S);
 int grid_of(swap_ctx* c);
 uint32_t resolve_mech(const swap_ctx* c, int dir);
 uint32_t mech(const swap_ctx* c);
+swap_status stage_expected(swap_ctx* c, cudaStream_t s);
 int kind_of(swap_ctx* c);
 int hash_kind(swap_ctx* c);
 swap_status launch(swap_ctx* c, int mode, int kind, const swk::Params& p, cudaStream_t s);

@@ -96,6 +96,7 @@ swap_status swap_exchange(swap_ctx_t* const* victims, size_t nv, swap_ctx_t* in,
     note_gathered(v, S);
     v->first_ckpt_done = true;
     v->st = St::CKPT_PENDING;
+    v->exp_valid = false;
   }
   const uint64_t budget = held + headroom;
   uint64_t acquired = 0, peak = 0;
@@ -189,6 +190,7 @@ swap_status swap_exchange(swap_ctx_t* const* victims, size_t nv, swap_ctx_t* in,
     if (ts != SWAP_OK) return ts;
     swp::seal_manifest(v->plan, manifest_ptr(v));
     v->st = St::CHECKPOINTED;
+    v->exp_valid = false;
   }
   if (peak_extra) *peak_extra = peak;
   return SWAP_OK;

@@ -27,7 +27,7 @@ swk::Params base_params(swap_ctx* c, const DescSet& S) {
   p.arrive = c->d_arrive;
   const uint64_t cs_off = c->plan.manifest_off + swp::kHeaderBytes + swp::kRegionRecBytes * c->plan.regions.size() + 24;
   p.cs_out = reinterpret_cast<uint64_t*>(c->image_dev + cs_off);
-  p.cs_exp = p.cs_out;
+  p.cs_exp = c->exp_valid ? reinterpret_cast<const uint64_t*>(c->d_exp + 24) : p.cs_out;
   p.n_bad = &c->d_status->n_bad;
   p.first_bad = &c->d_status->first_bad;
   p.tables = c->d_tables;
@@ -71,6 +71,18 @@ uint32_t resolve_mech(const swap_ctx* c, int dir) {
   return S < (2ull << 30) ? SWAP_MECH_SM : SWAP_MECH_CE_PIPE;
 }
 uint32_t mech(const swap_ctx* c) { return c->cur_mech; }
+
+// Stages the manifest's chunk records (expected checksums at +24 of each 32-B record) into HBM on `s`, at
+// every copy-engine restore (after its manifest check); the verify that follows reads the same copy.
+swap_status stage_expected(swap_ctx* c, cudaStream_t s) {
+  const uint64_t n = c->plan.n_chunks;
+  if (n == 0) return SWAP_OK;
+  if (!c->d_exp) CUDA_TRY(c, cudaMalloc(&c->d_exp, n * swp::kChunkRecBytes));
+  const uint64_t off = c->plan.manifest_off + swp::kHeaderBytes + swp::kRegionRecBytes * c->plan.regions.size();
+  CUDA_TRY(c, cudaMemcpyAsync(c->d_exp, c->image + off, n * swp::kChunkRecBytes, cudaMemcpyHostToDevice, s));
+  c->exp_valid = true;
+  return SWAP_OK;
+}
 int kind_of(swap_ctx* c) {
   if (mech(c) == SWAP_MECH_SM_NOCHECK) return swk::KIND_NONE;
   return c->plan.kind == SWAP_CHECKSUM_XXH64 ? swk::KIND_XXH64 : swk::KIND_CRC32C;
@@ -393,6 +405,7 @@ void release(swap_ctx* c) {
   if (c->d_status) cudaFree(c->d_status);
   if (c->h_status) cudaFreeHost(c->h_status);
   if (c->d_tables) cudaFree(c->d_tables);
+  if (c->d_exp) cudaFree(c->d_exp);
   if (c->d_tmaps) cudaFree(c->d_tmaps);
   if (c->d_chunk_region) cudaFree(c->d_chunk_region);
   if (c->d_reg_span) cudaFree(c->d_reg_span);

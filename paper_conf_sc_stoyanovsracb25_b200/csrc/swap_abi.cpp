@@ -241,6 +241,7 @@ swap_status swap_checkpoint(swap_ctx_t* c, swap_stream_t stream) {
   }
   DeviceGuard g(c->cfg.device);
   cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+  c->exp_valid = false;  // the chunk records are rewritten
   c->cur_mech = resolve_mech(c, 0);
   CUDA_TRY(c, cudaEventRecord(c->ev[0], s));
   bool hash_zero = false;
@@ -301,6 +302,8 @@ static swap_status restore_impl(swap_ctx* c, swap_stream_t stream, uint32_t stri
   c->stripe = stripe;
   c->n_stripes = n_stripes;
   DescSet& S = c->s_move;
+  if (mech(c) == SWAP_MECH_CE_PIPE || is_ce(mech(c)))  // the copies will saturate the host link
+    if ((st = stage_expected(c, s)) != SWAP_OK) return st;
   swk::Params p = base_params(c, S);
   CUDA_TRY(c, cudaMemsetAsync(&c->d_status->n_bad, 0, 8, s));
   CUDA_TRY(c, cudaMemsetAsync(&c->d_status->first_bad, 0xFF, 8, s));
@@ -496,6 +499,7 @@ swap_status swap_import(swap_ctx_t* c) {
   swap_status st = swp::check_manifest(c->plan, manifest_ptr(c), &c->err);
   if (st != SWAP_OK) return st;
   c->st = St::CHECKPOINTED;
+  c->exp_valid = false;
   c->first_ckpt_done = true;  // the imported image already holds SAVE_ONCE bytes and DISCARD checksums
   // the image came from elsewhere: its zero chunks are unknown, so restores move every chunk a mask
   // does not force to zero by policy, and the next checkpoint re-applies any pending mask in full
