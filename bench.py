@@ -76,8 +76,8 @@ def group_checks(rec: dict, payload: int, hbm_peak: float, mech: str):
         return None
     n = statistics.mean(rec["restore_launches"])
     t = statistics.mean(ms)
-    return {"bound": "hbm", "kernel": "HBM hash kernel <HASH_CHECK> per restore group (quad-line hash_kernel: a group "
-                                      "has too few segments per warp for the strand-staged kernel)",
+    return {"bound": "hbm", "kernel": "HBM hash kernel <HASH_CHECK> per restore group (CRC-32C: the strand-staged "
+                                      "crc_ts_kernel, one round of its warps per group)",
             "launches_per_restore": round(n, 1), "algorithmic_bytes_per_launch": round(payload / n),
             "achieved": round(payload / (t * 1e-3) / GB, 1), "peak": hbm_peak, "unit": "GB/s",
             "frac": round(payload / (t * 1e-3) / GB / hbm_peak, 4),

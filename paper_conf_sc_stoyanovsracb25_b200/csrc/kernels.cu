@@ -910,8 +910,10 @@ static cudaError_t launch_hash_t(const Params& p, int grid, cudaStream_t s) {
 // never read from memory. Other segments (ragged region tails, DISCARD chunks hashed from the zero buffer)
 // take per-lane 1-D bulk copies: ptxas issues those through an ELECT loop (~10 issue slots per lane and
 // stage), half the speed if every segment took them (profiles/r02_crc_strand_staged.md), fine for the few
-// ragged ones. The producer (lane 0 on the tensor path) runs NB stages ahead across segment boundaries (the
-// warp's segments form one flat stage sequence). Throughput follows the resident warp count (dependent
+// ragged ones. Segments are dealt warp-major across the CTAs (w * grid + cta, then + W * grid), so that a
+// launch with few segments (a CE_PIPE restore group's check) still spreads over every SM. The producer (lane 0
+// on the tensor path) runs NB stages ahead across segment boundaries (the warp's segments form one flat
+// stage sequence). Throughput follows the resident warp count (dependent
 // lookup chains), which shared memory caps: the tables take 128 KiB, each warp's ring NB*32*S bytes.
 // Shared layout (window addresses, base R0): W*NB mbarriers at R0, rings below the 32-KiB-aligned slicing
 // tables and after them (the tables sit at a 32-KiB boundary for crc_word4's (index << 7) | lb addresses).
@@ -998,7 +1000,7 @@ __global__ void __launch_bounds__(W * 32, 1) crc_ts_kernel(const Params p) {
   const uint32_t L1 = p.hlane_len;
   // producer cursor (this warp's copies): segment pidx, its stage pk of pnst; psrc = this lane's strand,
   // pbytes = its bytes below len & ~15 (the bulk-copied part); ptm / prow: the tensor path
-  uint32_t pidx = blockIdx.x * W + warp, pk = 0, pnst = 0, pseq = 0, pbytes = 0;
+  uint32_t pidx = warp * gridDim.x + blockIdx.x, pk = 0, pnst = 0, pseq = 0, pbytes = 0;
   const uint8_t* psrc = nullptr;
   const void* ptm = nullptr;
   int prow = 0;
@@ -1057,7 +1059,7 @@ __global__ void __launch_bounds__(W * 32, 1) crc_ts_kernel(const Params p) {
   const uint32_t m128 = 128u * gridDim.y;  // = 128 (gridDim.y == 1), opaque to ptxas
   const uint32_t* x2n = p.tables + TAB_X2N;
   uint32_t cseq = 0;
-  for (uint32_t idx = blockIdx.x * W + warp; idx < p.n_desc; idx += stride) {
+  for (uint32_t idx = warp * gridDim.x + blockIdx.x; idx < p.n_desc; idx += stride) {
     const SegDesc d = p.desc[idx];
     const uint64_t e = lane == 0 ? expect_early<MODE>(p, d.chunk) : 0;
     const uint32_t len = d.bytes, Ls = (uint32_t)ts_strand(len), nst = (Ls + S - 1) / S;
@@ -1127,22 +1129,24 @@ static cudaError_t launch_ts_t(const Params& p, int grid_cap, cudaStream_t s) {
     if (e != cudaSuccess) return e;
     attr_set |= 1ull << (dev & 63);
   }
-  const int grid = (int)std::max<uint32_t>(1, std::min<uint32_t>((uint32_t)grid_cap, (p.n_desc + W - 1) / W));
+  const int grid = (int)std::max<uint32_t>(1, std::min<uint32_t>((uint32_t)grid_cap, p.n_desc));
   crc_ts_kernel<MODE, W, NB, S><<<grid, W * 32, bytes, s>>>(p);
   return cudaGetLastError();
 }
 
 // CRC-32C hash-pass kernel. Default: the strand-staged kernel (19 warps, 2 x 80-B stages) when the tensor
-// maps exist, the common segment length L1 is at least 128 KiB and there are at least 16 segments per warp
-// of the grid -- +2.4..7.1 % (mean +4.7 %) over the quad-line b0f kernel on config B (1 MiB chunks) in six
-// in-process A/B blocks, +4.7 / +5.0 % with 16 / 4 MiB chunks (profiles/r02_crc_strand_staged.md) -- else
-// the quad-line b0f kernel: with short segments (a 16-KiB-segment 64 MiB image 48 vs 66 us; 4-KiB chunks
-// 2.8 vs 1.8 TB/s) or few segments per warp (1 GiB, 4096 x 256 KiB: 0.25 vs 0.39 ms, the static segment
-// deal leaves whole segments of tail) the quad-line kernel wins. SWAP_CRC_KERNEL (base | b0f | zb | zbb0f | ts | ts16; read at every launch) forces one for
+// maps exist, the common segment length L1 is at least 128 KiB and the segments either fit one round of
+// its warps (a CE_PIPE restore group's check: +12 %, profiles/r02_seg_groupchecks.md) or give every warp at
+// least 16 (the whole-image verify / hash pass: +2.4..7.1 %, mean +4.7 %, over the quad-line b0f kernel on
+// config B in six in-process A/B blocks, +4.7 / +5.0 % with 16 / 4 MiB chunks,
+// profiles/r02_crc_strand_staged.md); else the quad-line b0f kernel: with short segments (a 16-KiB-segment
+// 64 MiB image 48 vs 66 us; 4-KiB chunks 2.8 vs 1.8 TB/s) or 1-16 rounds of segments (1 GiB, 4096 x 256
+// KiB: 0.25 vs 0.37 ms -- the second round of whole segments is a tail) the quad-line kernel wins. SWAP_CRC_KERNEL (base | b0f | zb | zbb0f | ts | ts16; read at every launch) forces one for
 // A/B measurements: b0f +0.9..1.7 % over base; the Z^96 byte tables (zb) -10 % (profiles/r02_crc_variants.md).
 template <int MODE>
 static cudaError_t launch_hash(const Params& p, int grid, cudaStream_t s) {
-  int v = (p.tmaps && p.hlane_len >= (128u << 10) && p.n_desc >= 16u * 19u * (uint32_t)grid) ? 10 : 1;
+  const uint32_t slots = 19u * (uint32_t)grid;  // the strand kernel's warps
+  int v = (p.tmaps && p.hlane_len >= (128u << 10) && (p.n_desc <= slots || p.n_desc >= 16u * slots)) ? 10 : 1;
   if (const char* e = getenv("SWAP_CRC_KERNEL"))
     v = !strcmp(e, "base") ? 0 : !strcmp(e, "zb") ? 2 : !strcmp(e, "zbb0f") ? 3 : !strcmp(e, "ts") ? 10
       : !strcmp(e, "ts16") ? 11 : 1;
