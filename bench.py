@@ -702,9 +702,9 @@ def run_ours(args):
             "restore_GBps_per_gpu_slowest": round(payload / (max(restore_steps) * 1e-3) / GB, 3),
             "checkpoint_GBps_per_gpu": round(payload / (ckpt_ms * 1e-3) / GB, 3),
             # roofline = the HBM verify pass (a8), the kernel on the swap-in's critical path (~10 ms after the
-            # ~950 ms link transfer). In the serialised ncu launch list (profiles/r02_ncu_launches_bench_B_ts.md)
-            # the CE_PIPE restore's per-group checks hold the largest summed share, but they run on a side stream
-            # under the copy engine's H2D copies, off the critical path: roofline_group_checks times them live
+            # ~950 ms link transfer); the same kernel runs the CE_PIPE restore's per-group checks (side stream,
+            # under the copy engine's H2D copies): together the dominant kernel of the serialised ncu launch list
+            # (profiles/r02_ncu_launches_bench_B_ts2.md); roofline_group_checks times the group checks live
             "roofline": {"bound": "hbm", "kernel": VERIFY_KERNEL[args.checksum],
                          "achieved": round(payload / (verify_ms * 1e-3) / GB, 1), "peak": hbm_peak,
                          "unit": "GB/s", "frac": round(payload / (verify_ms * 1e-3) / GB / hbm_peak, 4),
