@@ -99,6 +99,7 @@ def parse():
     ap.add_argument("--checksum", default="crc32c", choices=["crc32c", "xxh64"])
     ap.add_argument("--chunk", type=int, default=1 << 20)
     ap.add_argument("--seg-bytes", type=int, default=0, help="CRC-32C segment size (0: the library's auto rule)")
+    ap.add_argument("--pipe-mib", type=int, default=0, help="CE_PIPE group size in MiB (0: the library's auto rule)")
     ap.add_argument("--grid", type=int, default=0)
     ap.add_argument("--no-compare", action="store_true", help="skip the other-mechanism comparison")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -503,7 +504,7 @@ def run_ours(args):
     kind = swap.SWAP_CHECKSUM_CRC32C if args.checksum == "crc32c" else swap.SWAP_CHECKSUM_XXH64
     t0 = time.perf_counter()
     sw = swap.Swapper(regions, chunk_bytes=args.chunk, checksum=kind, mechanism=args.mechanism, device=local_dev,
-                      rank=rank, world=world, grid_ctas=args.grid, seg_bytes=args.seg_bytes)
+                      rank=rank, world=world, grid_ctas=args.grid, seg_bytes=args.seg_bytes, pipe_mib=args.pipe_mib)
     t_register = time.perf_counter() - t0
     eff_mech = sw.mechanism("restore")
     eff_mech_ckpt = sw.mechanism("checkpoint")
@@ -689,7 +690,7 @@ def run_ours(args):
             "dtype": "u8", "data": "synthetic",
             "config": {"workload": workload_name,
                        "regions_per_rank": len(specs),
-                       "payload_bytes_per_rank": payload, "chunk_bytes": args.chunk, "seg_bytes": args.seg_bytes or "auto", "checksum": args.checksum,
+                       "payload_bytes_per_rank": payload, "chunk_bytes": args.chunk, "seg_bytes": args.seg_bytes or "auto", "pipe_mib": args.pipe_mib or "auto", "checksum": args.checksum,
                        "mechanism": f"{args.mechanism} -> restore {eff_mech}, checkpoint {eff_mech_ckpt}",
                        "l2": "no flush: every step moves the whole image (>> 126 MB L2)",
                        "parallelism": "single GPU" if world == 1 else f"tp{world} shard per rank (no data collective)",

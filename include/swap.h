@@ -103,7 +103,7 @@ typedef struct {
   uint32_t seg_bytes;   /* CRC32C work split inside a chunk: power of 2, >= 4096; 0 -> auto (at registration:
                            one segment per warp slot of the GPU, 4 KiB .. 256 KiB) */
   uint32_t pipe_mib;    /* SWAP_MECH_CE_PIPE group size in MiB (rounded up to whole chunks); 0 -> auto: payload/32
-                           clamped to [16, 256] MiB */
+                           clamped to [16, 512] MiB */
   int32_t host_numa;    /* host NUMA placement of the image (per-GPU topology fixed at init):
                            0 -> auto: the node sysfs reports for the device's PCI function
                            (/sys/bus/pci/devices/<bus id>/numa_node), preferred policy (mbind

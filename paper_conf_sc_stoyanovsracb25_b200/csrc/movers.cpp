@@ -430,10 +430,12 @@ static swap_status build_set(swap_ctx* c, DescSet* S, Pick pick, bool zero_src) 
   const swp::Plan& P = c->plan;
   const uint64_t seg = P.kind == SWAP_CHECKSUM_XXH64 ? P.C : std::min<uint64_t>(P.C, c->seg);
   std::vector<swk::SegDesc> desc;
-  // group size: cfg.pipe_mib, or auto = payload / 32 clamped to [16 MiB, 256 MiB] (smaller groups cost
-  // more in per-copy and per-launch overhead than they gain in overlap)
+  // group size: cfg.pipe_mib, or auto = payload / 32 clamped to [16 MiB, 512 MiB] (smaller groups cost
+  // more in per-copy and per-launch overhead than they gain in overlap; config B, profiles/r02_pipe_groups.md:
+  // swap-in 54.76-54.90 GB/s for 256 MiB - 1 GiB groups, the side-stream group checks 2.05 / 3.40 / 4.33 TB/s
+  // at 256 / 512 / 1024 MiB -- more segments per launch; 512 keeps ~12 groups per replica for 8 DP stripes)
   uint64_t target = (uint64_t)c->cfg.pipe_mib << 20;
-  if (!target) target = std::min<uint64_t>(256ull << 20, std::max<uint64_t>(16ull << 20, c->plan.payload_bytes / 32));
+  if (!target) target = std::min<uint64_t>(512ull << 20, std::max<uint64_t>(16ull << 20, c->plan.payload_bytes / 32));
   Group cur{0, 0, {}};
   uint64_t cur_bytes = 0;
   for (size_t i = 0; i < P.regions.size(); ++i) {
