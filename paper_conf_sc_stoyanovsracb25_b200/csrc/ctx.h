@@ -84,9 +84,8 @@ struct swap_ctx {
   // read the expected checksums from HBM, not over a host link saturated by the restore's own copies
   uint8_t* d_exp = nullptr;
   bool exp_valid = false;  // d_exp matches the manifest (cleared by checkpoint / import)
-  void* d_tmaps = nullptr;             // strand-staged CRC kernel: per-region tensor maps (null: none)
-  uint32_t* d_chunk_region = nullptr;  // [n_chunks] region index
-  ulonglong2* d_reg_span = nullptr;    // [n_regions] {device base, bytes}
+  void* d_tmaps = nullptr;                      // strand-staged CRC kernel: per-chunk tensor maps (null: none)
+  unsigned long long* d_chunk_dev = nullptr;    // [n_chunks] chunk g's device address (0: no map)
   uint32_t zinit_c = 0, xseg = 0;
   uint32_t seg = 0;  // CRC-32C segment size in use (cfg.seg_bytes, or chosen at registration when 0)
   uint32_t cur_mech = SWAP_MECH_SM;  // mechanism of the call in progress (resolve_mech)

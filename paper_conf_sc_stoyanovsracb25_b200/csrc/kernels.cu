@@ -904,10 +904,12 @@ static cudaError_t launch_hash_t(const Params& p, int grid, cudaStream_t s) {
 // across stages, so its register only takes slicing-by-4 word steps -- no Z shift until the final fold by
 // x^(8 * bytes after the strand) (TAB_SLANE for the common length L1): 32 lookup + 8 LDS.128 wavefronts per
 // KiB per warp. S is an odd multiple of 16 B, so the 8 lanes of an LDS.128 phase hit 8 distinct 16-B bank
-// groups. Standard segments (len == L1 at a multiple of L1 inside their region: every full segment) are
-// staged with ONE 2-D tensor copy per stage -- the region viewed as rows of P = L1/32 bytes, box {S, 32} at
-// column k*S, row offset/P; columns past P (a strand's last partial stage) are out of bounds, zero-filled,
-// never read from memory. Other segments (ragged region tails, DISCARD chunks hashed from the zero buffer)
+// groups. Standard segments (len == L1 at their place in the chunk: every full segment) are staged with ONE
+// 2-D tensor copy per stage -- the chunk viewed as rows of P = L1/32 bytes, box {S, 32} at column k*S, row
+// 32 * (segment index in the chunk); columns past P (a strand's last partial stage) are out of bounds,
+// zero-filled, never read from memory. The maps are per chunk, not per region: a scheduler swap-out releases
+// a victim's VMM slabs group by group while later groups are still hashed, and a TMA load through a map whose
+// tensor reaches into a released slab faults even when its box does not. Other segments (ragged region tails, DISCARD chunks hashed from the zero buffer)
 // take per-lane 1-D bulk copies: ptxas issues those through an ELECT loop (~10 issue slots per lane and
 // stage), half the speed if every segment took them (profiles/r02_crc_strand_staged.md), fine for the few
 // ragged ones. Segments are dealt warp-major across the CTAs (w * grid + cta, then + W * grid), so that a
@@ -1016,13 +1018,12 @@ __global__ void __launch_bounds__(W * 32, 1) crc_ts_kernel(const Params p) {
       psrc = reinterpret_cast<const uint8_t*>(dev) + a0;
       pk = 0;
       ptm = nullptr;
-      if (p.tmaps && len == L1) {
-        const uint32_t r = __ldg(p.chunk_region + __ldg(&p.desc[pidx].chunk));
-        const ulonglong2 rs = __ldg(p.reg_span + r);
-        const uint64_t off = dev - rs.x;
-        if (dev >= rs.x && off + len <= rs.y && off % L1 == 0) {
-          ptm = reinterpret_cast<const uint8_t*>(p.tmaps) + 128ull * r;
-          prow = (int)(off / (L1 / 32));
+      if (p.tmaps && len == L1) {  // segment s of chunk g starts at chunk_dev[g] + s * L1 (L1 = min(C, seg))
+        const uint32_t g = __ldg(&p.desc[pidx].chunk), s = __ldg(&p.desc[pidx].seg);
+        const unsigned long long cb = __ldg(p.chunk_dev + g);
+        if (cb && dev == cb + (uint64_t)s * L1) {
+          ptm = reinterpret_cast<const uint8_t*>(p.tmaps) + 128ull * g;
+          prow = (int)(s * 32u);
         }
       }
       return;

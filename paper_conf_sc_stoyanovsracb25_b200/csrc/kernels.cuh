@@ -65,9 +65,8 @@ struct Params {
   uint32_t xseg;                 // x^(8*seg_bytes) mod P
   uint32_t hlane_len;            // L1: the segment length TAB_HLANE was built for
   unsigned int* ticket;          // dynamic XXH64 lane kernel: chunk counter, zeroed before each launch
-  const void* tmaps;             // [n_regions] CUtensorMap of the strand-staged CRC kernel's tensor path, or null
-  const uint32_t* chunk_region;  // [n_chunks] region index of chunk g
-  const ulonglong2* reg_span;    // [n_regions] {device base, bytes}
+  const void* tmaps;             // [n_chunks] CUtensorMap of the strand-staged CRC kernel's tensor path, or null
+  const unsigned long long* chunk_dev;  // [n_chunks] device address of chunk g's first byte (0: no map)
 };
 
 void build_tables(uint32_t* tab /* TAB_WORDS */, uint64_t common_seg_len, uint64_t seg_bytes);
@@ -93,10 +92,12 @@ __host__ __device__ inline uint64_t ts_lane_end(uint64_t len, int lane) {
   if (a0 >= len) return 0;
   return a0 + Ls < len ? a0 + Ls : len;
 }
-// Its tensor path: region r viewed as rows of L1/32 bytes (u8, row pitch L1/32), box {TS_S, 32}; map r at
-// tmaps + 128 * r. out: n * 128 bytes (host); a region smaller than one row gets a zeroed map (never used:
-// its segments are not standard). Returns false if the driver entry point is missing or an encode fails
-// (the kernel then takes per-lane bulk copies, or launch_hash the quad-line kernel).
+// Its tensor path: one map per chunk (its whole extent inside the chunk: a scheduler swap-out releases a
+// victim's VMM slabs group by group while later groups are still hashed, and a TMA load through a map whose
+// tensor reaches into a released slab faults even if the box does not), chunk viewed as rows of L1/32 bytes
+// (u8, row pitch L1/32), box {TS_S, 32}; map g at tmaps + 128 * g. out: n * 128 bytes (host); a chunk
+// smaller than one row gets a zeroed map. Returns false if the driver entry point is missing or an encode
+// fails (the kernel then takes per-lane bulk copies, or launch_hash the quad-line kernel).
 constexpr int TS_S = 80;
 bool encode_tmaps(void* out, const uint64_t* base, const uint64_t* bytes, int n, uint64_t L1);
 uint32_t host_x2nmodp(uint64_t n, unsigned k, const uint32_t* x2n);

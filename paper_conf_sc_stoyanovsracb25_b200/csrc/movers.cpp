@@ -37,8 +37,7 @@ swk::Params base_params(swap_ctx* c, const DescSet& S) {
   p.hlane_len = (uint32_t)std::min<uint64_t>(c->plan.C, c->seg);
   p.ticket = &c->d_status->ticket;
   p.tmaps = c->d_tmaps;
-  p.chunk_region = c->d_chunk_region;
-  p.reg_span = c->d_reg_span;
+  p.chunk_dev = c->d_chunk_dev;
   return p;
 }
 
@@ -319,32 +318,25 @@ swap_status upload_tables(swap_ctx* c) {
   const uint32_t* x2n = tab.data() + swk::TAB_X2N;
   c->zinit_c = swk::host_multmodp(swk::host_x2nmodp(c->cfg.chunk_bytes, 3, x2n), 0xFFFFFFFFu);
   c->xseg = swk::host_x2nmodp(c->seg, 3, x2n);
-  // strand-staged CRC kernel's tensor path: a map per region, the region of every chunk
-  const size_t nr = c->plan.regions.size();
-  if (c->plan.kind == SWAP_CHECKSUM_CRC32C && nr && !c->d_tmaps) {
-    std::vector<uint64_t> base(nr), bytes(nr);
-    std::vector<ulonglong2> span(nr);
-    std::vector<uint32_t> creg(c->plan.n_chunks);
-    for (size_t r = 0; r < nr; ++r) {
-      const auto& R = c->plan.regions[r];
-      base[r] = R.r.dev_addr;
-      bytes[r] = R.r.bytes;
-      span[r] = make_ulonglong2(R.r.dev_addr, R.r.bytes);
-      for (uint64_t g = R.first; g < R.first + R.nchunks; ++g) creg[g] = (uint32_t)r;
-    }
-    std::vector<uint8_t> maps(nr * 128);
-    if (swk::encode_tmaps(maps.data(), base.data(), bytes.data(), (int)nr, std::min<uint64_t>(c->plan.C, c->seg))) {
-      for (size_t r = 0; r < nr; ++r)  // a region without a map (smaller than one row, or > 2^31 rows) never
-        if (std::all_of(maps.begin() + r * 128, maps.begin() + (r + 1) * 128, [](uint8_t b) { return b == 0; }))
-          span[r].y = 0;  // takes the tensor path: its span is empty for the kernel's range check
+  // strand-staged CRC kernel's tensor path (only used for segments of >= 128 KiB): a map per chunk
+  const uint64_t L1 = std::min<uint64_t>(c->plan.C, c->seg);
+  const uint64_t nc = c->plan.n_chunks;
+  if (c->plan.kind == SWAP_CHECKSUM_CRC32C && nc && L1 >= (128u << 10) && !c->d_tmaps) {
+    std::vector<uint64_t> base(nc), bytes(nc);
+    for (const auto& R : c->plan.regions)
+      for (uint64_t j = 0; j < R.nchunks; ++j) {
+        base[R.first + j] = R.r.dev_addr + j * c->plan.C;
+        bytes[R.first + j] = std::min<uint64_t>(c->plan.C, R.r.bytes - j * c->plan.C);
+      }
+    std::vector<uint8_t> maps(nc * 128);
+    if (swk::encode_tmaps(maps.data(), base.data(), bytes.data(), (int)nc, L1)) {
+      for (uint64_t g = 0; g < nc; ++g)  // a chunk without a map (shorter than one row) never takes the tensor path
+        if (std::all_of(maps.begin() + g * 128, maps.begin() + (g + 1) * 128, [](uint8_t v) { return v == 0; }))
+          base[g] = 0;
       CUDA_TRY(c, cudaMalloc(&c->d_tmaps, maps.size()));
       CUDA_TRY(c, cudaMemcpy(c->d_tmaps, maps.data(), maps.size(), cudaMemcpyHostToDevice));
-      CUDA_TRY(c, cudaMalloc(&c->d_reg_span, nr * sizeof(ulonglong2)));
-      CUDA_TRY(c, cudaMemcpy(c->d_reg_span, span.data(), nr * sizeof(ulonglong2), cudaMemcpyHostToDevice));
-      if (!creg.empty()) {
-        CUDA_TRY(c, cudaMalloc(&c->d_chunk_region, creg.size() * 4));
-        CUDA_TRY(c, cudaMemcpy(c->d_chunk_region, creg.data(), creg.size() * 4, cudaMemcpyHostToDevice));
-      }
+      CUDA_TRY(c, cudaMalloc(&c->d_chunk_dev, nc * 8));
+      CUDA_TRY(c, cudaMemcpy(c->d_chunk_dev, base.data(), nc * 8, cudaMemcpyHostToDevice));
     }
   }
   return SWAP_OK;
@@ -407,8 +399,7 @@ void release(swap_ctx* c) {
   if (c->d_tables) cudaFree(c->d_tables);
   if (c->d_exp) cudaFree(c->d_exp);
   if (c->d_tmaps) cudaFree(c->d_tmaps);
-  if (c->d_chunk_region) cudaFree(c->d_chunk_region);
-  if (c->d_reg_span) cudaFree(c->d_reg_span);
+  if (c->d_chunk_dev) cudaFree(c->d_chunk_dev);
   for (auto& e : c->ev)
     if (e) cudaEventDestroy(e);
   for (auto& e : c->chk_ev)

@@ -1,4 +1,4 @@
-"""Each CRC-32C HBM hash kernel (quad-line: base / b0f / zb; strand-staged with the per-region tensor-map
+"""Each CRC-32C HBM hash kernel (quad-line: base / b0f / zb; strand-staged with the per-chunk tensor-map
 path and per-lane bulk copies for other segments: ts (19 warps), ts16) forced in turn through SWAP_CRC_KERNEL, in
 a subprocess: the checkpoint's hash pass (HASH_STORE, copy-engine movers) must give the oracle's image byte
 for byte, the restore's per-group checks and the HBM verify (HASH_CHECK) must pass, and a single flipped
