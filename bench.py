@@ -45,9 +45,9 @@ RESTORE_KERNEL = {
     "ce_chunk": "restore phase: cudaMemcpyAsync per chunk + HBM hash pass",
     "ce_batch": "restore phase: coalesced cudaMemcpyAsync runs + HBM hash pass",
 }
-VERIFY_KERNEL = {"crc32c": "crc_ts_kernel<HASH_CHECK> (CRC-32C strand-staged: one TMA tensor box of 32 lane strands x 80 B per "
-                           "stage, per-lane replicated slice-by-4 tables; the quad-line hash_kernel below 128 KiB "
-                           "segments or 16 segments per warp)",
+VERIFY_KERNEL = {"crc32c": "crc_mx_kernel<HASH_CHECK> (CRC-32C, per SM 16 strand-staged warps -- 32 lane strands x 80 B "
+                           "per stage by one TMA tensor box -- and 12 quad-line warps over per-lane replicated "
+                           "slice-by-4 tables; the quad-line hash_kernel below 128 KiB segments)",
                  "xxh64": "xxh_quad_kernel<HASH_CHECK> (XXH64: a lane quad per chunk, per-chunk TMA rings in shared memory; "
                           "lane kernels below 256 KiB chunks)"}
 PCIE_GEN5_X16_GBPS = 63.015  # 64 GB/s x 128/130 (nominal, per direction)
@@ -76,8 +76,8 @@ def group_checks(rec: dict, payload: int, hbm_peak: float, mech: str):
         return None
     n = statistics.mean(rec["restore_launches"])
     t = statistics.mean(ms)
-    return {"bound": "hbm", "kernel": "HBM hash kernel <HASH_CHECK> per restore group (CRC-32C: the strand-staged "
-                                      "crc_ts_kernel, one round of its warps per group)",
+    return {"bound": "hbm", "kernel": "HBM hash kernel <HASH_CHECK> per restore group (CRC-32C: crc_mx_kernel, the verify's "
+                                      "kernel, one round of its warps per group)",
             "launches_per_restore": round(n, 1), "algorithmic_bytes_per_launch": round(payload / n),
             "achieved": round(payload / (t * 1e-3) / GB, 1), "peak": hbm_peak, "unit": "GB/s",
             "frac": round(payload / (t * 1e-3) / GB / hbm_peak, 4),

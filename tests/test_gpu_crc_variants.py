@@ -70,7 +70,7 @@ print("variant ok")
 '''
 
 
-@pytest.mark.parametrize("variant", ["base", "b0f", "zb", "ts", "ts16"])
+@pytest.mark.parametrize("variant", ["base", "b0f", "zb", "ts", "ts16", "mx", "mx16"])
 def test_crc32c_kernel_variant(variant):
     env = dict(os.environ, SWAP_CRC_KERNEL=variant)
     out = subprocess.run([sys.executable, "-c", SCRIPT, ROOT], capture_output=True, text=True, env=env, timeout=600)

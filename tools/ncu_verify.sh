@@ -4,7 +4,7 @@
 cd "${GRAFT_REPO_ROOT:-.}"
 mkdir -p gpurun_out
 for ck in ${@:-crc32c xxh64}; do
-  k=$([ $ck = crc32c ] && echo "regex:hash_kernel|crc_ts_kernel" || echo regex:xxh_)
+  k=$([ $ck = crc32c ] && echo "regex:hash_kernel|crc_ts_kernel|crc_mx_kernel" || echo regex:xxh_)
   timeout 1200 ncu --set full --clock-control none --import-source on -k $k -c 1 -o gpurun_out/ncu_verify_B_$ck -f \
     python tools/prof_case.py --config B --mechanism sm --checksum $ck --reps 1 > gpurun_out/ncu_verify_B_$ck.log 2>&1
   echo "$ck rc=$?"

@@ -66,7 +66,7 @@ os.environ.pop("SWAP_XXH_KERNEL")
 # CRC-32C hash kernel variants (fixed shared layout at the 0x400 dynamic base; the strand-staged ts kernels
 # with their tensor-map path on standard segments and per-lane bulk copies on ragged ones, also with
 # 128 KiB segments of 1 MiB chunks)
-for v in ("base", "b0f", "zb", "zbb0f", "ts", "ts16"):
+for v in ("base", "b0f", "zb", "zbb0f", "ts", "ts16", "mx", "mx16"):
     os.environ["SWAP_CRC_KERNEL"] = v
     for C, seg in ((1 << 16, 0), (1 << 20, 1 << 17)):
         with swap.Swapper(regions, chunk_bytes=C, checksum=1, mechanism="ce_region", seg_bytes=seg) as sw, \
