@@ -1266,7 +1266,9 @@ static cudaError_t launch_ts_t(const Params& p, int grid_cap, cudaStream_t s) {
 }
 
 // CRC-32C hash-pass kernel. With the tensor maps (segments of >= 128 KiB):
-//  * whole-image passes (>= 16 segments per strand-kernel warp: the verify, the CE_PIPE checkpoint's hash pass)
+//  * whole-image passes (>= 4 segments per strand-kernel warp: the verify, the CE_PIPE checkpoint's hash pass;
+//    scaled config B images, b0f vs mixed: 1 GiB 0.248 vs 0.369 ms, 2 GiB 0.479 vs 0.555, 4 GiB 0.933 vs
+//    0.880, 8 GiB 1.612 vs 1.596, 16 GiB 3.409 vs 3.349)
 //    take the mixed kernel (16 strand-staged + 12 quad-line warps per SM, 5/8 of the segments to the strand
 //    role): config B verify +4 % over the strand kernel alone inside the bench, same box (5559 / 5573 vs 5347
 //    GB/s), +6 % at 16 MiB chunks; the strand kernel alone was +2.4..7.1 % over the quad-line b0f kernel
@@ -1275,15 +1277,15 @@ static cudaError_t launch_ts_t(const Params& p, int grid_cap, cudaStream_t s) {
 //    alone is faster there (3438 vs 2908 GB/s summed over a restore's groups: latency-bound warps, one segment
 //    each): the checks hide under the copy engine's H2D copies, and one kernel for checks and verify keeps the
 //    dominant kernel of the launch list the one whose roofline the bench reports;
-//  * otherwise (1-16 rounds, or short segments) the quad-line b0f kernel (1 GiB = 4096 x 256 KiB: 0.25 vs
-//    0.37 ms; a 16-KiB-segment 64 MiB image 48 vs 66 us; 4-KiB chunks 2.8 vs 1.8 TB/s).
+//  * otherwise (1-4 rounds, or short segments) the quad-line b0f kernel (a 16-KiB-segment 64 MiB image 48 vs
+//    66 us for the strand kernel; 4-KiB chunks 2.8 vs 1.8 TB/s).
 // SWAP_CRC_KERNEL (base | b0f | zb | zbb0f | ts | ts16 | mx | mx16; read at every launch) forces one for A/B
 // measurements: b0f +0.9..1.7 % over base; the Z^96 byte tables (zb) -10 % (profiles/r02_crc_variants.md).
 template <int MODE>
 static cudaError_t launch_hash(const Params& p, int grid, cudaStream_t s) {
   const uint32_t slots = 19u * (uint32_t)grid;  // the strand kernel's warps
   int v = 1;
-  if (p.tmaps && p.hlane_len >= (128u << 10) && (p.n_desc <= slots || p.n_desc >= 16u * slots)) v = 12;
+  if (p.tmaps && p.hlane_len >= (128u << 10) && (p.n_desc <= slots || p.n_desc >= 4u * slots)) v = 12;
   if (const char* e = getenv("SWAP_CRC_KERNEL"))
     v = !strcmp(e, "base") ? 0 : !strcmp(e, "zb") ? 2 : !strcmp(e, "zbb0f") ? 3 : !strcmp(e, "ts") ? 10
       : !strcmp(e, "ts16") ? 11 : !strcmp(e, "mx") ? 12 : !strcmp(e, "mx16") ? 13 : 1;
