@@ -1016,6 +1016,10 @@ __device__ __forceinline__ void ts_role(const Params& p, uint32_t tab, uint32_t 
         if (cb && dev == cb + (uint64_t)s * L1) {
           ptm = reinterpret_cast<const uint8_t*>(p.tmaps) + 128ull * g;
           prow = (int)(s * 32u);
+          // the maps were written to global memory by the host (cudaMemcpy at registration): make them
+          // visible to the tensormap proxy before the TMA unit reads them (a ctx's maps can reuse the
+          // address of a destroyed ctx's maps)
+          if (lane == 0) asm volatile("fence.proxy.tensormap::generic.acquire.gpu [%0], 128;" ::"l"(ptm) : "memory");
         }
       }
       return;
